@@ -1,0 +1,147 @@
+/*
+ * dfs.h — C ABI of the B200-native unordered-DFS library (libdfs.so).
+ *
+ * Operation (DiggerBees, PPoPP '26; "P:a-b" = /root/reference/PAPER.md lines):
+ *   Given a CSR graph and a root r, discover every vertex reachable from r and build a DFS tree
+ *   (§2.1).  Output semantics are Table 2's "DiggerBees" row: the visited
+ *   set and the parent array of a valid DFS tree, lexicographic order NOT enforced ("Unordered").
+ *   The traversal is the paper's hierarchical work-stealing DFS (§3) re-designed for
+ *   sm_100a: a persistent kernel, per-warp two-level stacks (shared-memory HotRing + global
+ *   ColdSeg, §3.2), warp-level expansion with atomic claims (§3.3), intra-block (§3.4, Alg 3)
+ *   and inter-block (§3.5, Alg 4) stealing, and a global termination detector.
+ *
+ * Graph convention
+ *   row_ptr[n+1] (int64), col_idx[m] (int32): directed out-adjacency in CSR.
+ *   An undirected graph is passed with both directions.  Self loops and duplicates are allowed
+ *   (a self loop is never a tree edge; for duplicates the first occurrence is the tree position).
+ *   Requirements: 1 <= n <= 2^31 - 3, 0 <= m < 2^32, row_ptr[0] == 0, row_ptr non-decreasing,
+ *   row_ptr[n] == m, 0 <= col_idx[j] < n.  Violations -> DFS_EINVAL.
+ *
+ * Output convention (parent_out, int32[n])
+ *   parent_out[root] = DFS_ROOT_PARENT (-1)  (Alg 1 line 1)
+ *   parent_out[v]    = DFS_UNREACHED (-2)    for every vertex not reachable from root
+ *   parent_out[v]    = u                     otherwise: (u,v) is an edge and u is v's DFS-tree parent
+ *   visited(v) <=> parent_out[v] != DFS_UNREACHED.  The result satisfies checks I1-I6 of
+ *   DESIGN.md (scan-order-consistent DFS tree); with dfs_options.deterministic = 1 it equals
+ *   Alg 1's lexicographic tree exactly.
+ *
+ * Memory / ownership
+ *   Input and output pointers may be host or device memory (detected per call with
+ *   cudaPointerGetAttributes).  dfs_graph_create COPIES the CSR to the current CUDA device; the
+ *   caller keeps ownership of its arrays and may free them after the call.  The handle owns all
+ *   device memory it uses (graph, visited bitmap, stack-chunk pool sized from n, counters);
+ *   runs never allocate device memory, except an internal parent buffer allocated on first use
+ *   when parent_out is host memory.  Output buffers are caller-allocated and fully overwritten
+ *   on DFS_OK; their contents are unspecified on error.
+ *
+ * Synchronisation / threading
+ *   Every call is synchronous: it is stream-ordered on the handle's stream (default: the legacy
+ *   default stream; see dfs_set_stream) and returns after the outputs are written.  One call at
+ *   a time per handle; distinct handles are independent.  All calls must be made with the
+ *   handle's device current (else DFS_EDEVICE).
+ *
+ * Errors
+ *   Functions returning int return DFS_OK (0) or a negative dfs_status.  dfs_graph_create
+ *   returns NULL on failure.  dfs_last_error() returns the status of the last failing call on
+ *   the calling thread.  dfs_graph_destroy(NULL) is a no-op.
+ */
+#ifndef B200_DFS_H
+#define B200_DFS_H
+
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef struct dfs_graph dfs_graph;   /* opaque */
+
+enum dfs_status {
+    DFS_OK        =  0,
+    DFS_EINVAL    = -1,   /* NULL pointer, bad sizes, root out of range, malformed CSR        */
+    DFS_ENOMEM    = -2,   /* device allocation failed or stack-chunk pool exhausted            */
+    DFS_ECUDA     = -3,   /* CUDA runtime error (launch failure, no device, ...)               */
+    DFS_EDEVICE   = -4,   /* current device differs from the handle's device                   */
+    DFS_ETIMEOUT  = -5,   /* traversal watchdog fired (dfs_options.timeout_ms)                 */
+    DFS_EINTERNAL = -6    /* internal consistency check failed                                 */
+};
+
+#define DFS_ROOT_PARENT (-1)
+#define DFS_UNREACHED   (-2)
+
+/* Victim-block policies for inter-block stealing (Alg 4 step 1). */
+enum dfs_victim_policy {
+    DFS_VICTIM_RANDOM     = 0,   /* uniform random active block (Fig 9 baseline) */
+    DFS_VICTIM_TWO_CHOICE = 1    /* power-of-two-choices by cumulative ColdSeg load (default) */
+};
+
+/* Tuning / ablation options.  Zero-initialise, then call dfs_options_default. */
+typedef struct dfs_options {
+    int32_t blocks;          /* persistent grid size; 0 = (#SMs x resident blocks per SM)          */
+    int32_t warps_per_block; /* 1..32; 0 = 32                                                      */
+    int32_t hot_cutoff;      /* Alg 3 threshold: steal h_s = hot_cutoff/2; default 32     */
+    int32_t cold_cutoff;     /* Alg 4 threshold: steal c_s = cold_cutoff/2; default 64    */
+    int32_t deterministic;   /* 1: one warp, no stealing: result == Alg 1 lexicographic tree       */
+    int32_t intra_steal;     /* 1: enable Alg 3 (default)                                          */
+    int32_t inter_steal;     /* 1: enable Alg 4 (default)                                          */
+    int32_t victim_policy;   /* dfs_victim_policy; default DFS_VICTIM_TWO_CHOICE                   */
+    int32_t timeout_ms;      /* watchdog; default 120000                                           */
+    uint32_t seed;           /* RNG seed for victim selection                                      */
+    int32_t collect_stats;   /* 1: fill the counters of dfs_stats (small overhead)                 */
+    int32_t reserved[5];
+} dfs_options;
+
+typedef struct dfs_stats {
+    float   kernel_ms;       /* device time of reset + traversal + finalize (CUDA events)          */
+    float   traversal_ms;    /* device time of the persistent traversal kernel alone               */
+    int32_t blocks, warps_per_block;
+    int64_t n_visited;       /* |visited|                                                          */
+    int64_t m_visited;       /* sum of out-degrees of visited vertices (TEPS numerator)            */
+    /* counters (collect_stats = 1) */
+    int64_t claims, failed_claims, flushes, refills, intra_steals, inter_steals, steal_attempts,
+            chunks_allocated, windows;
+} dfs_stats;
+
+void dfs_options_default(dfs_options *opt);
+
+/* Create a graph handle on the current CUDA device (copies and validates the CSR).
+ * Returns NULL on failure (see dfs_last_error). */
+dfs_graph *dfs_graph_create(const int64_t *row_ptr, const int32_t *col_idx, int64_t n, int64_t m);
+
+/* One unordered DFS from root (Alg 2 skeleton P:249-286 with §3's hierarchy).  parent_out: n
+ * int32, host or device.  Default options. */
+int dfs_run(dfs_graph *g, int32_t root, int32_t *parent_out);
+
+/* num_roots independent traversals; row i of parents_out (num_roots x n, row-major, host or
+ * device) receives the result for roots[i] (roots: host or device).  North-star batch entry;
+ * multi-GPU batches partition roots across processes above this call. */
+int dfs_run_batch(dfs_graph *g, const int32_t *roots, int32_t num_roots, int32_t *parents_out);
+
+/* dfs_run with explicit options (may be NULL = defaults) and optional stats (may be NULL). */
+int dfs_run_ex(dfs_graph *g, int32_t root, int32_t *parent_out, const dfs_options *opt,
+               dfs_stats *stats);
+
+/* Batch with explicit options; stats (may be NULL) accumulates over the batch. */
+int dfs_run_batch_ex(dfs_graph *g, const int32_t *roots, int32_t num_roots, int32_t *parents_out,
+                     const dfs_options *opt, dfs_stats *stats);
+
+/* Stream all subsequent calls on this handle are ordered on (a cudaStream_t; NULL = legacy
+ * default stream). */
+int dfs_set_stream(dfs_graph *g, void *cuda_stream);
+
+/* n, m, device ordinal of a handle (any pointer may be NULL). */
+int dfs_graph_info(const dfs_graph *g, int64_t *n, int64_t *m, int32_t *device);
+
+/* Number of this library's kernels launched on the handle since creation (reset, traversal,
+ * finalize, ...): the bench's "gpu_launches" count. */
+int64_t dfs_launch_count(const dfs_graph *g);
+
+void dfs_graph_destroy(dfs_graph *g);
+
+int dfs_last_error(void);
+const char *dfs_strerror(int code);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* B200_DFS_H */

@@ -1,0 +1,276 @@
+"""ctypes binding of libdfs.so (include/dfs.h) — argument marshalling only.
+
+PyTorch supplies device memory, the current CUDA stream and (in bench.py) process groups; the
+traversal itself is the persistent sm_100a kernel behind ``dfs_run``/``dfs_run_batch``.
+Function names follow the C ABI: :meth:`Graph.run` -> ``dfs_run_ex``, :meth:`Graph.run_batch`
+-> ``dfs_run_batch_ex``, construction -> ``dfs_graph_create``, :meth:`Graph.close` ->
+``dfs_graph_destroy``.
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+from dataclasses import dataclass, fields
+from typing import Optional
+
+import numpy as np
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+_SO = os.path.join(_HERE, "libdfs.so")
+
+DFS_ROOT_PARENT = -1
+DFS_UNREACHED = -2
+
+STATUS = {0: "DFS_OK", -1: "DFS_EINVAL", -2: "DFS_ENOMEM", -3: "DFS_ECUDA", -4: "DFS_EDEVICE",
+          -5: "DFS_ETIMEOUT", -6: "DFS_EINTERNAL"}
+
+#: every symbol include/dfs.h declares (checked by tests/test_capi.py)
+EXPORTS = ["dfs_options_default", "dfs_graph_create", "dfs_run", "dfs_run_batch", "dfs_run_ex",
+           "dfs_run_batch_ex", "dfs_set_stream", "dfs_graph_info", "dfs_launch_count",
+           "dfs_graph_destroy", "dfs_last_error", "dfs_strerror"]
+
+
+class DfsError(RuntimeError):
+    def __init__(self, code: int, what: str = ""):
+        self.code = code
+        super().__init__(f"{what}: {STATUS.get(code, code)} ({_strerror(code)})")
+
+
+class _Options(ctypes.Structure):
+    _fields_ = [("blocks", ctypes.c_int32), ("warps_per_block", ctypes.c_int32),
+                ("hot_cutoff", ctypes.c_int32), ("cold_cutoff", ctypes.c_int32),
+                ("deterministic", ctypes.c_int32), ("intra_steal", ctypes.c_int32),
+                ("inter_steal", ctypes.c_int32), ("victim_policy", ctypes.c_int32),
+                ("timeout_ms", ctypes.c_int32), ("seed", ctypes.c_uint32),
+                ("collect_stats", ctypes.c_int32), ("reserved", ctypes.c_int32 * 5)]
+
+
+class _Stats(ctypes.Structure):
+    _fields_ = [("kernel_ms", ctypes.c_float), ("traversal_ms", ctypes.c_float),
+                ("blocks", ctypes.c_int32), ("warps_per_block", ctypes.c_int32),
+                ("n_visited", ctypes.c_int64), ("m_visited", ctypes.c_int64),
+                ("claims", ctypes.c_int64), ("failed_claims", ctypes.c_int64),
+                ("flushes", ctypes.c_int64), ("refills", ctypes.c_int64),
+                ("intra_steals", ctypes.c_int64), ("inter_steals", ctypes.c_int64),
+                ("steal_attempts", ctypes.c_int64), ("chunks_allocated", ctypes.c_int64),
+                ("windows", ctypes.c_int64)]
+
+
+@dataclass
+class Options:
+    """Mirror of ``struct dfs_options`` (None = library default)."""
+    blocks: Optional[int] = None
+    warps_per_block: Optional[int] = None
+    hot_cutoff: Optional[int] = None
+    cold_cutoff: Optional[int] = None
+    deterministic: Optional[bool] = None
+    intra_steal: Optional[bool] = None
+    inter_steal: Optional[bool] = None
+    victim_policy: Optional[int] = None
+    timeout_ms: Optional[int] = None
+    seed: Optional[int] = None
+    collect_stats: Optional[bool] = None
+
+    def to_c(self) -> _Options:
+        o = _Options()
+        load_library().dfs_options_default(ctypes.byref(o))
+        for f in fields(self):
+            v = getattr(self, f.name)
+            if v is not None:
+                setattr(o, f.name, int(v))
+        return o
+
+
+@dataclass
+class Stats:
+    kernel_ms: float
+    traversal_ms: float
+    blocks: int
+    warps_per_block: int
+    n_visited: int
+    m_visited: int
+    claims: int
+    failed_claims: int
+    flushes: int
+    refills: int
+    intra_steals: int
+    inter_steals: int
+    steal_attempts: int
+    chunks_allocated: int
+    windows: int
+
+
+_lib = None
+
+
+def lib_path() -> str:
+    return _SO
+
+
+def load_library():
+    """Load libdfs.so; raises if it is missing (no fallback path exists)."""
+    global _lib
+    if _lib is None:
+        if not os.path.exists(_SO):
+            raise ImportError(f"{_SO} is missing: run `python __graft_entry__.py` (build()) first; "
+                              "there is no CPU fallback")
+        lib = ctypes.CDLL(_SO)
+        P, I32, I64 = ctypes.c_void_p, ctypes.c_int32, ctypes.c_int64
+        lib.dfs_options_default.argtypes = [ctypes.POINTER(_Options)]
+        lib.dfs_options_default.restype = None
+        lib.dfs_graph_create.argtypes = [P, P, I64, I64]
+        lib.dfs_graph_create.restype = P
+        lib.dfs_run.argtypes = [P, I32, P]
+        lib.dfs_run.restype = ctypes.c_int
+        lib.dfs_run_batch.argtypes = [P, P, I32, P]
+        lib.dfs_run_batch.restype = ctypes.c_int
+        lib.dfs_run_ex.argtypes = [P, I32, P, ctypes.POINTER(_Options), ctypes.POINTER(_Stats)]
+        lib.dfs_run_ex.restype = ctypes.c_int
+        lib.dfs_run_batch_ex.argtypes = [P, P, I32, P, ctypes.POINTER(_Options), ctypes.POINTER(_Stats)]
+        lib.dfs_run_batch_ex.restype = ctypes.c_int
+        lib.dfs_set_stream.argtypes = [P, P]
+        lib.dfs_set_stream.restype = ctypes.c_int
+        lib.dfs_graph_info.argtypes = [P, ctypes.POINTER(I64), ctypes.POINTER(I64), ctypes.POINTER(I32)]
+        lib.dfs_graph_info.restype = ctypes.c_int
+        lib.dfs_launch_count.argtypes = [P]
+        lib.dfs_launch_count.restype = I64
+        lib.dfs_graph_destroy.argtypes = [P]
+        lib.dfs_graph_destroy.restype = None
+        lib.dfs_last_error.argtypes = []
+        lib.dfs_last_error.restype = ctypes.c_int
+        lib.dfs_strerror.argtypes = [ctypes.c_int]
+        lib.dfs_strerror.restype = ctypes.c_char_p
+        _lib = lib
+    return _lib
+
+
+def _strerror(code: int) -> str:
+    try:
+        return load_library().dfs_strerror(code).decode()
+    except Exception:  # pragma: no cover
+        return "?"
+
+
+def _ptr(x):
+    """(data pointer, keep-alive) of a contiguous torch tensor or numpy array."""
+    try:
+        import torch
+        if isinstance(x, torch.Tensor):
+            if not x.is_contiguous():
+                x = x.contiguous()
+            return x.data_ptr(), x
+    except ImportError:  # pragma: no cover
+        pass
+    a = np.ascontiguousarray(x)
+    return a.ctypes.data, a
+
+
+def _as(x, np_dtype, torch_dtype):
+    try:
+        import torch
+        if isinstance(x, torch.Tensor):
+            return x.to(torch_dtype).contiguous()
+    except ImportError:  # pragma: no cover
+        pass
+    return np.ascontiguousarray(x, dtype=np_dtype)
+
+
+class Graph:
+    """A CSR graph resident on the current CUDA device (``dfs_graph_create``).
+
+    ``row_ptr`` (int64[n+1]) and ``col_idx`` (int32[m]) may be numpy arrays or torch tensors on
+    the CPU or on the current GPU; they are copied, so the caller may drop them afterwards.
+    """
+
+    def __init__(self, row_ptr, col_idx):
+        import torch
+        self._lib = load_library()
+        rp = _as(row_ptr, np.int64, torch.int64)
+        ci = _as(col_idx, np.int32, torch.int32)
+        n = int(rp.shape[0]) - 1
+        m = int(ci.shape[0])
+        prp, _k1 = _ptr(rp)
+        pci, _k2 = _ptr(ci) if m > 0 else (None, None)
+        self._h = self._lib.dfs_graph_create(prp, pci, n, m)
+        if not self._h:
+            raise DfsError(self._lib.dfs_last_error(), "dfs_graph_create")
+        self.n, self.m = n, m
+        self.device = torch.cuda.current_device()
+
+    # -- helpers ------------------------------------------------------------------------
+    def _stream(self):
+        import torch
+        rc = self._lib.dfs_set_stream(self._h, torch.cuda.current_stream().cuda_stream)
+        if rc != 0:
+            raise DfsError(rc, "dfs_set_stream")
+
+    @staticmethod
+    def _opts(options: Optional[Options], stats: bool):
+        if options is None and not stats:
+            return None
+        o = (options or Options()).to_c()
+        if stats:
+            o.collect_stats = 1
+        return o
+
+    # -- API ----------------------------------------------------------------------------
+    def run(self, root: int, out=None, options: Optional[Options] = None, stats: bool = False):
+        """One unordered DFS from ``root`` (``dfs_run_ex``).  Returns the int32 parent tensor
+        (``out`` if given; host or device) and, with ``stats=True``, a :class:`Stats`."""
+        import torch
+        if out is None:
+            out = torch.empty(self.n, dtype=torch.int32, device="cuda")
+        assert out.dtype == torch.int32 and out.numel() == self.n
+        self._stream()
+        o = self._opts(options, stats)
+        st = _Stats() if stats else None
+        rc = self._lib.dfs_run_ex(self._h, int(root), out.data_ptr(),
+                                  ctypes.byref(o) if o is not None else None,
+                                  ctypes.byref(st) if st is not None else None)
+        if rc != 0:
+            raise DfsError(rc, "dfs_run_ex")
+        if stats:
+            return out, Stats(**{f[0]: getattr(st, f[0]) for f in _Stats._fields_})
+        return out
+
+    def run_batch(self, roots, out=None, options: Optional[Options] = None, stats: bool = False):
+        """``len(roots)`` traversals (``dfs_run_batch_ex``); row i of the (k, n) int32 result
+        belongs to ``roots[i]``."""
+        import torch
+        r = torch.as_tensor(roots, dtype=torch.int32)
+        k = int(r.numel())
+        if out is None:
+            out = torch.empty((k, self.n), dtype=torch.int32, device="cuda")
+        assert out.dtype == torch.int32 and out.numel() == k * self.n
+        self._stream()
+        o = self._opts(options, stats)
+        st = _Stats() if stats else None
+        rr = r.contiguous()
+        rc = self._lib.dfs_run_batch_ex(self._h, rr.data_ptr(), k, out.data_ptr(),
+                                        ctypes.byref(o) if o is not None else None,
+                                        ctypes.byref(st) if st is not None else None)
+        if rc != 0:
+            raise DfsError(rc, "dfs_run_batch_ex")
+        if stats:
+            return out, Stats(**{f[0]: getattr(st, f[0]) for f in _Stats._fields_})
+        return out
+
+    def launch_count(self) -> int:
+        return int(self._lib.dfs_launch_count(self._h))
+
+    def close(self):
+        if getattr(self, "_h", None):
+            self._lib.dfs_graph_destroy(self._h)
+            self._h = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:  # pragma: no cover
+            pass
+
+    def __enter__(self):
+        return self
+
+    def __exit__(self, *a):
+        self.close()

@@ -1,0 +1,222 @@
+"""GPU parity: the CUDA path (through the C ABI) against the oracle, on the same seeded inputs.
+
+Bars (DESIGN.md §"Parity"): integer work, tolerance 0.
+  * deterministic single-warp mode: parent array bit-exact with Alg 1 (oracle.dfs);
+  * tree-shaped inputs (unique spanning tree): bit-exact in every mode;
+  * full parallel mode: checks I1-I6 exact (I4 = reach set bit-exact, visited count exact);
+    I7 (classical DFS tree) reported, not required (stealing creates cross edges by design);
+  * stress: tiny cutoffs, few warps/blocks, many roots — forces flush/refill/steal races.
+"""
+import numpy as np
+import pytest
+
+import graphgen
+import oracle
+
+torch = pytest.importorskip("torch")
+pytestmark = pytest.mark.gpu
+
+if torch.cuda.is_available():
+    from paper_conf_ppopp_niul0c26_b200 import DfsError, Graph, Options
+
+
+def _exact(g, root, parent):
+    want = oracle.dfs(g.row_ptr, g.col_idx, root)
+    got = parent.cpu().numpy() if hasattr(parent, "cpu") else parent
+    if not np.array_equal(got, want):
+        bad = np.nonzero(got != want)[0]
+        raise AssertionError(f"{g.name} root {root}: {bad.size} mismatches, first {bad[:5]} "
+                             f"got {got[bad[:5]]} want {want[bad[:5]]}")
+
+
+def _valid(g, root, parent, undirected=True):
+    got = parent.cpu().numpy() if hasattr(parent, "cpu") else parent
+    r = oracle.check_tree(g.row_ptr, g.col_idx, root, got, i7=True, undirected=undirected)
+    assert all(getattr(r, k) == 1 for k in ("i1", "i2", "i3", "i4", "i5", "i6")), (g.name, root, r)
+    reach = oracle.reach(g.row_ptr, g.col_idx, root)
+    assert r.n_visited == int(reach.sum())
+    return r
+
+
+DET = None
+
+
+def det():
+    return Options(deterministic=True)
+
+
+# ------------------------------------------------------------------ deterministic = Alg 1
+@pytest.mark.parametrize("name,build,root", [
+    ("grid256", lambda: graphgen.grid(256, 256), 0),                  # depth-65,535 snake
+    ("grid_ragged", lambda: graphgen.grid(37, 53), 700),
+    ("road512", lambda: graphgen.road(512, 300, seed=5), 0),
+    ("path1e6", lambda: graphgen.path(1_000_000), 0),
+    ("pathchords", lambda: graphgen.path_chords(300_000, 3_000, seed=2), 12345),
+    ("caterpillar", lambda: graphgen.caterpillar(4096, 94), 0),
+    ("rmat16", lambda: graphgen.rmat(16, 16), None),
+    ("star", lambda: graphgen.star(100_000), 0),
+    ("random_dir", lambda: graphgen.random_graph(20_000, 60_000, seed=3, symmetric=False,
+                                                  allow_self=True, allow_dup=True), 17),
+    ("shuffled", lambda: graphgen.shuffle_lists(graphgen.random_graph(5000, 30000, seed=4), 9), 1),
+])
+def test_deterministic_bit_exact(name, build, root):
+    g = build()
+    if root is None:
+        root = int(graphgen.random_roots(g, 1, seed=1)[0])
+    with Graph(g.row_ptr, g.col_idx) as G:
+        p = G.run(root, options=det())
+        torch.cuda.synchronize()
+        _exact(g, root, p)
+
+
+# ------------------------------------------------------------------ unique trees: exact in parallel
+@pytest.mark.parametrize("name,build,roots", [
+    ("path", lambda: graphgen.path(200_001), [0, 100_000, 200_000]),
+    ("star", lambda: graphgen.star(50_000), [0, 7]),
+    ("bintree", lambda: graphgen.binary_tree((1 << 20) - 1), [0, 5, (1 << 19)]),
+    ("caterpillar", lambda: graphgen.caterpillar(1 << 14, 94), [0, 5000]),
+])
+def test_tree_inputs_bit_exact_parallel(name, build, roots):
+    g = build()
+    with Graph(g.row_ptr, g.col_idx) as G:
+        for r in roots:
+            p = G.run(r)
+            _exact(g, r, p)
+
+
+# ------------------------------------------------------------------ parallel: I1-I6 exact
+@pytest.mark.parametrize("name,build,nroots", [
+    ("grid256", lambda: graphgen.grid(256, 256), 3),
+    ("road1024", lambda: graphgen.road(1024, 1024, seed=0x5EED), 3),
+    ("road_ragged", lambda: graphgen.road(999, 777, seed=11), 2),
+    ("rmat18", lambda: graphgen.rmat(18, 16), 4),
+    ("pathchords", lambda: graphgen.path_chords(1_000_000, 10_000, seed=1), 2),
+    ("random_sparse", lambda: graphgen.random_graph(200_000, 150_000, seed=8), 4),  # many components
+])
+def test_parallel_valid(name, build, nroots):
+    g = build()
+    roots = [0] + list(graphgen.random_roots(g, nroots - 1, seed=42))
+    with Graph(g.row_ptr, g.col_idx) as G:
+        for r in roots:
+            p = G.run(int(r))
+            _valid(g, int(r), p)
+
+
+def test_parallel_directed_with_self_loops_and_duplicates():
+    g = graphgen.random_graph(100_000, 400_000, seed=77, symmetric=False, allow_self=True, allow_dup=True)
+    with Graph(g.row_ptr, g.col_idx) as G:
+        for r in graphgen.random_roots(g, 3, seed=5):
+            p = G.run(int(r))
+            _valid(g, int(r), p, undirected=False)
+
+
+# ------------------------------------------------------------------ stress
+@pytest.mark.parametrize("opts", [
+    dict(hot_cutoff=4, cold_cutoff=4),
+    dict(hot_cutoff=8, cold_cutoff=8, warps_per_block=4, blocks=8),
+    dict(hot_cutoff=4, cold_cutoff=4, warps_per_block=2, blocks=64),
+    dict(victim_policy=0),
+    dict(intra_steal=False),
+    dict(inter_steal=False),
+    dict(blocks=1),
+    dict(hot_cutoff=64, cold_cutoff=128),
+])
+def test_stress_options(opts):
+    graphs = [graphgen.road(300, 300, seed=3), graphgen.rmat(14, 8, seed=9),
+              graphgen.caterpillar(2000, 30), graphgen.path_chords(100_000, 2_000, seed=3)]
+    o = Options(**opts)
+    for g in graphs:
+        with Graph(g.row_ptr, g.col_idx) as G:
+            for r in list(graphgen.random_roots(g, 3, seed=len(opts))) + [0]:
+                p = G.run(int(r), options=o)
+                _valid(g, int(r), p)
+
+
+def test_many_small_random_graphs():
+    rng = np.random.default_rng(0)
+    for k in range(40):
+        n = int(rng.integers(2, 3000))
+        g = graphgen.random_graph(n, int(rng.integers(0, 4 * n)), seed=k, symmetric=bool(k % 2),
+                                  allow_self=bool(k % 3 == 0), allow_dup=bool(k % 5 == 0))
+        o = Options(hot_cutoff=4, cold_cutoff=4) if k % 2 else None
+        with Graph(g.row_ptr, g.col_idx) as G:
+            r = int(rng.integers(0, n))
+            p = G.run(r, options=o)
+            _valid(g, r, p, undirected=bool(k % 2))
+            if k % 4 == 0:
+                _exact(g, r, G.run(r, options=det()))
+
+
+# ------------------------------------------------------------------ API edge cases
+def test_isolated_root_single_vertex_and_empty():
+    rp = np.zeros(2, dtype=np.int64)
+    with Graph(rp, np.zeros(0, dtype=np.int32)) as G:
+        assert G.run(0).cpu().tolist() == [-1]
+    rp = np.array([0, 1, 2, 2], dtype=np.int64)
+    ci = np.array([1, 0], dtype=np.int32)
+    with Graph(rp, ci) as G:
+        assert G.run(2).cpu().tolist() == [-2, -2, -1]
+        assert G.run(0).cpu().tolist() == [-1, 0, -2]
+
+
+def test_host_and_device_buffers_and_batch():
+    g = graphgen.road(200, 150, seed=1)
+    roots = graphgen.random_roots(g, 6, seed=2)
+    rp_d = torch.from_numpy(g.row_ptr).cuda()
+    ci_d = torch.from_numpy(g.col_idx).cuda()
+    with Graph(rp_d, ci_d) as G:                                # device inputs
+        host_out = torch.empty(g.n, dtype=torch.int32).pin_memory()
+        G.run(int(roots[0]), out=host_out)                       # host output
+        _valid(g, int(roots[0]), host_out.numpy())
+        out = G.run_batch(roots)                                 # device batch output
+        for q, r in enumerate(roots):
+            _valid(g, int(r), out[q])
+        hb = torch.empty((len(roots), g.n), dtype=torch.int32)  # host batch output, device roots
+        G.run_batch(torch.from_numpy(roots).cuda(), out=hb, options=det())
+        for q, r in enumerate(roots):
+            _exact(g, int(r), hb[q].numpy())
+        assert G.launch_count() > 0
+
+
+def test_errors():
+    g = graphgen.grid(10, 10)
+    with Graph(g.row_ptr, g.col_idx) as G:
+        with pytest.raises(DfsError) as e:
+            G.run(100)
+        assert e.value.code == -1
+        with pytest.raises(DfsError):
+            G.run(0, options=Options(hot_cutoff=6))               # h_s must be even
+        with pytest.raises(DfsError):
+            G.run(0, options=Options(blocks=100000))
+    bad = g.row_ptr.copy(); bad[5] = bad[4] - 1                   # non-monotone row_ptr
+    with pytest.raises(DfsError):
+        Graph(bad, g.col_idx)
+    badc = g.col_idx.copy(); badc[3] = g.n                        # neighbour out of range
+    with pytest.raises(DfsError):
+        Graph(g.row_ptr, badc)
+    with pytest.raises(DfsError):
+        Graph(torch.from_numpy(bad).cuda(), torch.from_numpy(g.col_idx).cuda())
+
+
+def test_stats_counters():
+    g = graphgen.road(512, 512, seed=3)
+    with Graph(g.row_ptr, g.col_idx) as G:
+        p, st = G.run(0, stats=True)
+        r = _valid(g, 0, p)
+        assert st.n_visited == r.n_visited and st.m_visited == r.m_visited
+        assert st.claims == r.n_visited - 1
+        assert st.kernel_ms > 0
+
+
+def test_stream_and_repeat_consistency():
+    g = graphgen.rmat(15, 16, seed=3)
+    r = int(graphgen.random_roots(g, 1, seed=3)[0])
+    s = torch.cuda.Stream()
+    with Graph(g.row_ptr, g.col_idx) as G:
+        with torch.cuda.stream(s):
+            ps = [G.run(r) for _ in range(5)]
+        torch.cuda.synchronize()
+        vis = [(p != -2).cpu().numpy() for p in ps]
+        for p, v in zip(ps, vis):
+            assert np.array_equal(v, vis[0])
+            _valid(g, r, p)
