@@ -79,8 +79,10 @@ enum dfs_victim_policy {
 typedef struct dfs_options {
     int32_t blocks;          /* persistent grid size; 0 = (#SMs x resident blocks per SM)          */
     int32_t warps_per_block; /* 1..32; 0 = 32                                                      */
-    int32_t hot_cutoff;      /* Alg 3 threshold: steal h_s = hot_cutoff/2; default 32     */
-    int32_t cold_cutoff;     /* Alg 4 threshold: steal c_s = cold_cutoff/2; default 64    */
+    int32_t hot_cutoff;      /* Alg 3 threshold: steal h_s = hot_cutoff/2 entries when a peer holds
+                                >= hot_cutoff (even, h_s <= 32); paper 32; default 2       */
+    int32_t cold_cutoff;     /* Alg 4 threshold: steal c_s = cold_cutoff/2 (a power of two <= 64);
+                                paper 64; default 2                                        */
     int32_t deterministic;   /* 1: one warp, no stealing: result == Alg 1 lexicographic tree       */
     int32_t intra_steal;     /* 1: enable Alg 3 (default)                                          */
     int32_t inter_steal;     /* 1: enable Alg 4 (default)                                          */
@@ -88,7 +90,22 @@ typedef struct dfs_options {
     int32_t timeout_ms;      /* watchdog; default 120000                                           */
     uint32_t seed;           /* RNG seed for victim selection                                      */
     int32_t collect_stats;   /* 1: fill the counters of dfs_stats (small overhead)                 */
-    int32_t reserved[5];
+    int32_t spill;           /* 1: demand-driven spill — a busy warp whose HotRing holds >=
+                                2*cold_cutoff entries moves the oldest half to its ColdSeg when
+                                >= spill_idle warps are idle (B200 design); default 1 */
+    int32_t inter_any;       /* 1: any idle warp that finds no intra-block victim may steal
+                                inter-block; 0: only the leader warp of an idle block (Alg 4,
+                                P:1150-1152); default 1                                            */
+    int32_t spill_idle;      /* idle-warp threshold of the spill; default 32                       */
+    int32_t backoff_max_ns;  /* cap of the idle warps' exponential __nanosleep backoff; default 2048 */
+    int32_t window;          /* expansion window in positions: 32 (one neighbour per lane) or 128
+                                (four per lane, one 128-bit load); 0 = auto (128 iff m >= 8n)      */
+    int32_t pub_batch;       /* the owner publishes its HotRing head to thieves every pub_batch
+                                pushes (entries above it are private); default 1                    */
+    int32_t speculate;       /* 1: claim a freshly descended child's first non-parent neighbour
+                                in parallel with the visited probes; 0: off; 2 (default): on for
+                                32-wide windows only                                               */
+    int32_t reserved[4];
 } dfs_options;
 
 typedef struct dfs_stats {
@@ -100,6 +117,9 @@ typedef struct dfs_stats {
     /* counters (collect_stats = 1) */
     int64_t claims, failed_claims, flushes, refills, intra_steals, inter_steals, steal_attempts,
             chunks_allocated, windows;
+    int64_t idle_ns;         /* sum over warps of time spent idle (stealing / waiting)             */
+    int64_t inter_scans;     /* inter-block victim-selection rounds                                */
+    int64_t spills;          /* demand-driven spills                                               */
 } dfs_stats;
 
 void dfs_options_default(dfs_options *opt);
@@ -135,6 +155,12 @@ int dfs_graph_info(const dfs_graph *g, int64_t *n, int64_t *m, int32_t *device);
 /* Number of this library's kernels launched on the handle since creation (reset, traversal,
  * finalize, ...): the bench's "gpu_launches" count. */
 int64_t dfs_launch_count(const dfs_graph *g);
+
+/* Diagnostics: busy-warp timeline.  dfs_debug_timeline(g, len, dt_ns, NULL) enables sampling of
+ * the global busy-warp counter every dt_ns (block 0 / warp 0) into a device buffer of len
+ * samples (sample = busy + 1; 0 = no sample) for subsequent runs; calling it again with the same
+ * len and a host buffer `out` copies the last run's samples out and clears them; len = 0 disables. */
+int dfs_debug_timeline(dfs_graph *g, uint32_t len, uint32_t dt_ns, uint32_t *out);
 
 void dfs_graph_destroy(dfs_graph *g);
 

@@ -1,30 +1,38 @@
 // dfs_device.cuh — sm_100a device code of the unordered-DFS hot path.
 //
 // The method is DiggerBees (PPoPP '26); "P:a-b" = /root/reference/PAPER.md lines.  The kernel
-// re-designs the paper's H100 kernel for B200 (DESIGN.md §"Kernels"):
+// re-designs the paper's H100 kernel for B200:
 //
 //   * persistent grid, one 32-warp CTA per SM (subsystem 1; "1 block per SM")
 //   * per-warp two-level stack (subsystem 2; §3.2, Fig 2):
-//       HotRing  = circular buffer in shared memory, monotone 32-bit head/tail counters
+//       HotRing  = circular buffer in shared memory; head/tail are 16-bit counters packed in
+//                  one 32-bit word updated only by shared-memory atomics (no SC fences)
 //       ColdSeg  = per-warp virtual linear segment in global memory, backed by a chunk table
 //                  and a global chunk pool (the paper's fixed n_v/n_w capacity overflows on deep
 //                  graphs; reading S9)
-//       flush oldest H/2 entries from tail -> ColdSeg top; refill from ColdSeg top
-//   * warp-level expansion (subsystem 3; §3.3): the 32 lanes load a 32-neighbour
-//     window of col_idx, probe the visited bitmap, __ballot_sync + __ffs pick the FIRST unvisited
-//     neighbour in CSR order, one lane claims it with atomicOr on the bitmap word (the claim of
-//     Alg 1 l.9-10 made atomic).  The current top entry lives in registers; the child's
-//     row_ptr pair and its first window are loaded speculatively, overlapping the claim.
-//   * intra-block stealing (subsystem 4; §3.4, Alg 3): idle warps take h_s =
+//       flush oldest entries from tail -> ColdSeg top; refill from ColdSeg top
+//   * warp-level expansion (subsystem 3; §3.3): the 32 lanes load a VEC*32-position
+//     window of col_idx (VEC = 4: one 128-bit load per lane), probe the visited bitmap,
+//     __ballot_sync + __ffs pick the FIRST unvisited neighbour in CSR order, lane 0 claims it
+//     with atomicOr on the bitmap word (Alg 1 l.9-10 made atomic).  The top entry lives in
+//     registers; the child's row_ptr pair and first window are loaded speculatively so they
+//     overlap the probe and the claim.
+//   * intra-block stealing (subsystem 4; §3.4, Alg 3): an idle warp takes h_s =
 //     hot_cutoff/2 entries from the TAIL of the peer HotRing with max hot_rest >= hot_cutoff,
-//     under a per-warp shared-memory lock + THE-style owner/thief protocol (reading S12)
-//   * inter-block stealing (subsystem 5; §3.5, Alg 4): the leader warp of an idle
-//     block picks a victim block by two random choices weighted by cumulative ColdSeg load
-//     (reading S14), then the victim warp with max cold_rest >= cold_cutoff, reserves c_s =
-//     cold_cutoff/2 entries from the ColdSeg BOTTOM with a 64-bit CAS on the packed
-//     {top,bottom} word, and copies them into its HotRing.
+//     reserving them with a CAS on the packed head/tail word under the victim's lock (S12)
+//   * inter-block stealing (subsystem 5; §3.5, Alg 4): two random active blocks,
+//     the heavier by cumulative ColdSeg load (S14); the warp with max cold_rest >= cold_cutoff;
+//     c_s = cold_cutoff/2 entries reserved from the ColdSeg BOTTOM by a 64-bit CAS on the packed
+//     {top,bottom} word and copied into the thief's HotRing.
+//   * demand-driven spill (B200 addition): when many warps are idle, a busy warp
+//     moves the oldest half of a deep HotRing to its ColdSeg so other blocks can steal it.
 //   * global termination (unspecified in the paper, reading S13): a busy counter of warps that
 //     hold work plus registered thieves; the atomic that brings it to 0 raises `done`.
+//
+// Memory-ordering notes: CTA-scope release (MEMBAR.ALL.CTA) publishes HotRing
+// entries; CTA-scope acquire is free.  GPU-scope publication of ColdSeg data uses
+// fence.release.gpu (MEMBAR.ALL.GPU, no L1 invalidation); readers of ColdSeg data use L2
+// (.cg / .relaxed.gpu) loads whose addresses depend on the reserving atomic.
 #pragma once
 #include <cstdint>
 
@@ -35,7 +43,6 @@ constexpr uint32_t kEmptySlot = 0xffffffffu;
 constexpr int kChunkLog2 = 11;                     // ColdSeg chunk = 2048 entries (16 KB)
 constexpr uint32_t kChunk = 1u << kChunkLog2;
 constexpr int kMaxWarps = 32;                      // 32-bit warp mask
-constexpr int kPrefetchLanes = 8;                  // lanes that prefetch a candidate's row_ptr
 
 // error codes written to Ctl::status (mirrors dfs_status)
 constexpr int kStatusENOMEM = -2;
@@ -53,12 +60,12 @@ struct Ctl {
 
 enum CounterIdx {
     kCntClaims = 0, kCntFailedClaims, kCntFlushes, kCntRefills, kCntIntraSteals, kCntInterSteals,
-    kCntStealAttempts, kCntChunks, kCntWindows, kNumCounters
+    kCntStealAttempts, kCntChunks, kCntWindows, kCntIdleNs, kCntInterScans, kCntSpills, kNumCounters
 };
 
 struct KParams {
     const uint32_t* __restrict__ rp;         // n+1 (narrowed row_ptr; m < 2^32)
-    const int32_t* __restrict__ col;         // m
+    const int32_t* __restrict__ col;         // m (+8 padding)
     uint32_t* bitmap;                        // ceil(n/32) visited words
     int32_t* parent;                         // n output
     unsigned long long* cold_tb;             // n_warps: (top << 32) | bottom
@@ -75,8 +82,17 @@ struct KParams {
     int hot_cutoff, cold_cutoff;
     int intra, inter, policy;
     int collect_stats;
+    int spill;                               // demand-driven spill of oldest HotRing entries
+    int spill_idle;                          // ... when at least this many warps are idle
+    int inter_any;                           // any idle warp may steal inter-block (else leader of an idle block)
+    unsigned int backoff_max_ns;             // idle-loop exponential backoff cap
+    unsigned int* timeline;                  // optional: busy-warp samples (block 0 / warp 0)
+    unsigned int timeline_len;
+    unsigned int timeline_dt_ns;
     unsigned long long timeout_ns;
     uint32_t seed;
+    uint32_t pub_batch;                      // publish the HotRing head every pub_batch pushes
+    int speculate;                           // speculative claim of the child's first neighbour
 };
 
 // ------------------------------------------------------------------------------------------
@@ -97,19 +113,49 @@ __device__ __forceinline__ int ld_relaxed_s32(const int* p) {
     asm volatile("ld.relaxed.gpu.global.s32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
     return v;
 }
+__device__ __forceinline__ void st_relaxed_u32(uint32_t* p, uint32_t v) {
+    asm volatile("st.relaxed.gpu.global.u32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
+}
 __device__ __forceinline__ unsigned long long globaltimer() {
     unsigned long long t;
     asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
     return t;
 }
-// 16-byte L2 (coherent) load of two stack entries
-__device__ __forceinline__ void ld_cg_v2(const unsigned long long* p, unsigned long long& a,
-                                         unsigned long long& b) {
-    asm volatile("ld.global.cg.v2.u64 {%0, %1}, [%2];" : "=l"(a), "=l"(b) : "l"(p) : "memory");
+__device__ __forceinline__ unsigned long long ld_cg_u64(const unsigned long long* p) {
+    unsigned long long v;
+    asm volatile("ld.global.cg.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
+    return v;
 }
-__device__ __forceinline__ void st_cg_v2(unsigned long long* p, unsigned long long a,
-                                         unsigned long long b) {
-    asm volatile("st.global.cg.v2.u64 [%0], {%1, %2};" ::"l"(p), "l"(a), "l"(b) : "memory");
+__device__ __forceinline__ void st_cg_u64(unsigned long long* p, unsigned long long v) {
+    asm volatile("st.global.cg.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
+}
+// release fence at GPU scope without the L1 invalidation (CCTL.IVALL) of __threadfence()
+__device__ __forceinline__ void fence_release_gpu() { asm volatile("fence.release.gpu;" ::: "memory"); }
+
+// shared-memory atomics with explicit semantics (CTA scope)
+__device__ __forceinline__ uint32_t smem_addr(const void* p) { return (uint32_t)__cvta_generic_to_shared(p); }
+__device__ __forceinline__ uint32_t atom_add_release_cta(uint32_t* p, uint32_t v) {
+    uint32_t r;
+    asm volatile("atom.release.cta.shared.add.u32 %0, [%1], %2;" : "=r"(r) : "r"(smem_addr(p)), "r"(v) : "memory");
+    return r;
+}
+__device__ __forceinline__ uint32_t atom_add_relaxed_cta(uint32_t* p, uint32_t v) {
+    uint32_t r;
+    asm volatile("atom.relaxed.cta.shared.add.u32 %0, [%1], %2;" : "=r"(r) : "r"(smem_addr(p)), "r"(v) : "memory");
+    return r;
+}
+__device__ __forceinline__ uint32_t atom_cas_acquire_cta(uint32_t* p, uint32_t cmp, uint32_t v) {
+    uint32_t r;
+    asm volatile("atom.acquire.cta.shared.cas.b32 %0, [%1], %2, %3;" : "=r"(r) : "r"(smem_addr(p)), "r"(cmp), "r"(v) : "memory");
+    return r;
+}
+__device__ __forceinline__ uint32_t ld_acquire_cta(const uint32_t* p) {
+    uint32_t r;
+    asm volatile("ld.acquire.cta.shared.u32 %0, [%1];" : "=r"(r) : "r"(smem_addr(p)) : "memory");
+    return r;
+}
+__device__ __forceinline__ void st_release_cta(uint32_t* p, uint32_t v) {
+    asm volatile("st.release.cta.shared.u32 [%0], %1;" ::"r"(smem_addr(p)), "r"(v) : "memory");
 }
 
 __device__ __forceinline__ unsigned long long pack_entry(uint32_t v, uint32_t i) {
@@ -123,30 +169,29 @@ __device__ __forceinline__ uint32_t xorshift32(uint32_t& s) {
     return s;
 }
 
+// packed HotRing control word: (head << 16) | tail, 16-bit counters (H <= 2^15)
+__device__ __forceinline__ uint32_t ht_head(uint32_t x) { return x >> 16; }
+__device__ __forceinline__ uint32_t ht_tail(uint32_t x) { return x & 0xFFFFu; }
+__device__ __forceinline__ int ht_rest(uint32_t x) { return (int)(int16_t)(uint16_t)((x >> 16) - (x & 0xFFFFu)); }
+
 // ------------------------------------------------------------------------------------------
 // shared-memory control block (one per CTA)
 // ------------------------------------------------------------------------------------------
 struct SmemCtl {
-    volatile uint32_t head[kMaxWarps];    // HotRing head (next free slot); written by owner only
-    volatile uint32_t tail[kMaxWarps];    // oldest entry; thieves reserve by advancing it
-    volatile uint32_t tailf[kMaxWarps];   // slots below tailf are free for reuse (copy finished)
-    int lock[kMaxWarps];                  // per-warp lock for tail-side operations
-    unsigned int warp_mask;               // 1 = warp active
-    volatile int done;                    // block-local copy of ctl->done
+    uint32_t ht[kMaxWarps];                // HotRing (head << 16) | tail; atomics only
+    volatile uint32_t tailf[kMaxWarps];    // 16-bit: slots below tailf are free for reuse
+    uint32_t lock[kMaxWarps];              // per-warp lock for tail-side ops (thieves, flush)
+    unsigned int warp_mask;                // 1 = warp active
+    volatile int done;                     // block-local copy of ctl->done
+    uint32_t inter_token;                  // one idle warp per block scans other blocks at a time
+    unsigned long long cnt[kMaxWarps][16]; // per-warp stats counters (collect_stats)
 };
 
-__device__ __forceinline__ void smem_lock(int* l) {
-    while (atomicCAS(l, 0, 1) != 0) { }
-    __threadfence_block();
+__device__ __forceinline__ void smem_lock(uint32_t* l) {
+    while (atom_cas_acquire_cta(l, 0u, 1u) != 0u) { }
 }
-__device__ __forceinline__ bool smem_trylock(int* l) {
-    if (atomicCAS(l, 0, 1) == 0) { __threadfence_block(); return true; }
-    return false;
-}
-__device__ __forceinline__ void smem_unlock(int* l) {
-    __threadfence_block();
-    atomicExch(l, 0);
-}
+__device__ __forceinline__ bool smem_trylock(uint32_t* l) { return atom_cas_acquire_cta(l, 0u, 1u) == 0u; }
+__device__ __forceinline__ void smem_unlock(uint32_t* l) { st_release_cta(l, 0u); }
 
 // ------------------------------------------------------------------------------------------
 // chunk pool: tagged lock-free free stack + bump allocator
@@ -171,8 +216,8 @@ __device__ __forceinline__ void pool_free(const KParams& P, uint32_t idx) {
     Ctl* c = P.ctl;
     unsigned long long old = ld_relaxed_u64(&c->free_head);
     for (;;) {
-        asm volatile("st.relaxed.gpu.global.u32 [%0], %1;" ::"l"(&P.chunk_next[idx]), "r"((uint32_t)old) : "memory");
-        __threadfence();
+        st_relaxed_u32(&P.chunk_next[idx], (uint32_t)old);
+        fence_release_gpu();
         unsigned long long nw = ((unsigned long long)((uint32_t)(old >> 32) + 1u) << 32) | idx;
         unsigned long long got = atomicCAS(&c->free_head, old, nw);
         if (got == old) return;
@@ -187,14 +232,21 @@ __device__ __forceinline__ void raise_error(const KParams& P, int code) {
 }
 
 // ------------------------------------------------------------------------------------------
-// The persistent traversal kernel.  H = HotRing entries per warp (power of two).
-// Launched with blockDim.x = 32 * W (W <= 32) and dynamic shared memory
+// The persistent traversal kernel.
+//   H   = HotRing entries per warp (power of two, <= 2^15)
+//   VEC = neighbours per lane per window (1: 32-wide window; 4: 128-wide, 128-bit loads)
+//   WMAX = max warps per block (launch bounds: 32 -> 64 registers, 16 -> 128 registers)
+//   STATS = compile the diagnostic counters in
+// Launched with blockDim.x = 32 * W (W <= WMAX) and dynamic shared memory
 // sizeof(SmemCtl) (16-byte padded) + W * H * 8 bytes.
 // ------------------------------------------------------------------------------------------
-template <int H>
-__global__ void __launch_bounds__(1024, 1) dfs_persistent_kernel(const KParams P) {
-    static_assert((H & (H - 1)) == 0 && H >= 64, "H must be a power of two >= 64");
+template <int H, int VEC, int WMAX, bool STATS>
+__global__ void __launch_bounds__(32 * WMAX, 1) dfs_persistent_kernel(const KParams P) {
+    static_assert((H & (H - 1)) == 0 && H >= 64 && H <= 32768, "H must be a power of two in [64, 2^15]");
+    static_assert(VEC == 1 || VEC == 4, "VEC is 1 or 4");
     constexpr uint32_t kBatch = H / 2;              // flush batch (reading S10)
+    constexpr uint32_t kWin = 32u * VEC;            // positions per window
+    constexpr int kPfLanes = 8 / VEC;               // lanes covering the first 8 positions
     extern __shared__ __align__(16) unsigned char smem_raw[];
     SmemCtl& S = *reinterpret_cast<SmemCtl*>(smem_raw);
     constexpr int kCtlBytes = (sizeof(SmemCtl) + 15) & ~15;
@@ -211,28 +263,33 @@ __global__ void __launch_bounds__(1024, 1) dfs_persistent_kernel(const KParams P
     const uint32_t cs = (uint32_t)P.cold_cutoff >> 1;       // c_s (Alg 4 l.17)
 
     if (threadIdx.x < kMaxWarps) {
-        S.head[threadIdx.x] = 0; S.tail[threadIdx.x] = 0; S.tailf[threadIdx.x] = 0;
-        S.lock[threadIdx.x] = 0;
+        S.ht[threadIdx.x] = 0; S.tailf[threadIdx.x] = 0; S.lock[threadIdx.x] = 0;
     }
-    if (threadIdx.x == 0) { S.warp_mask = (blockIdx.x == 0) ? 1u : 0u; S.done = 0; }
+    if (threadIdx.x == 0) { S.warp_mask = (blockIdx.x == 0) ? 1u : 0u; S.done = 0; S.inter_token = 0; }
+    unsigned long long* const cnt = S.cnt[w];     // lane 0 updates its warp's counters
+    if (STATS && lane < 16) cnt[lane] = 0;
     __syncthreads();
 
     // ---- per-warp state (warp-uniform registers) ----
     bool has_top = false;        // a current top entry <u, i> lives in registers
-    bool have_win = false;       // nb holds the window starting at i
+    bool have_win = false;       // nbv holds the window starting at i
     bool need_end = false;       // end must be re-read from row_ptr
     uint32_t u = 0, i = 0, end = 0;
-    int nb = -1;                 // this lane's neighbour in the current window
-    uint32_t my_head = 0;        // owner copy of S.head[w]
+    int nbv[VEC];                // this lane's neighbours in the current window
+#pragma unroll
+    for (int e = 0; e < VEC; ++e) nbv[e] = -1;
+    uint32_t my_head = 0;        // owner's true HotRing head (16-bit wrap)
+    uint32_t pub = 0;            // head value published in S.ht (entries in [pub, my_head) are
+                                 // private: pushed/popped without synchronisation)
+    bool spec_ok = false;        // current window is a freshly descended child's first window
+    uint32_t par = kFull;        // parent of u when spec_ok
     uint32_t my_top = 0;         // owner copy of ColdSeg top
     uint32_t hi = 0;             // ColdSeg chunks [.., hi) mapped by this warp
     bool active = false;
     uint32_t rng = P.seed ^ (0x9E3779B9u * (uint32_t)(gw + 1));
     if (rng == 0) rng = 1;
-    unsigned long long cnt[kNumCounters];
-#pragma unroll
-    for (int k = 0; k < kNumCounters; ++k) cnt[k] = 0;
     const unsigned long long t_start = globaltimer();
+    unsigned long long t_idle0 = 0;
     uint32_t iter = 0;
 
     if (blockIdx.x == 0 && w == 0) {
@@ -241,15 +298,47 @@ __global__ void __launch_bounds__(1024, 1) dfs_persistent_kernel(const KParams P
         u = (uint32_t)P.root; i = __ldg(P.rp + u); end = __ldg(P.rp + u + 1);
     }
 
+    // window loader: lane holds positions base + VEC*lane + e, e < VEC
+    auto load_window = [&](uint32_t base, uint32_t limit, int* out) {
+        const uint32_t q = base + (uint32_t)VEC * lane;
+        if constexpr (VEC == 4) {
+            int4 x = make_int4(-1, -1, -1, -1);
+            if (q < limit) x = __ldg(reinterpret_cast<const int4*>(P.col + q));   // col padded
+            out[0] = x.x; out[1] = x.y; out[2] = x.z; out[3] = x.w;
+        } else {
+            out[0] = (q < limit) ? __ldg(P.col + q) : -1;
+        }
+    };
+
     // ---------------------------------------------------------------- owner stack operations
-    // flush: move the kBatch oldest HotRing entries to ColdSeg top (Fig 2(e))
-    auto flush = [&]() -> bool {
-        if (lane == 0) smem_lock(&S.lock[w]);
-        __syncwarp();
-        const uint32_t t = __shfl_sync(kFull, S.tail[w], 0);
-        // map chunks covering [my_top, my_top + kBatch)
+    // publish the private entries [pub, my_head) to thieves (CTA-scope release)
+    auto publish = [&]() {
+        if (my_head != pub) {
+            if (lane == 0) atom_add_release_cta(&S.ht[w], ((my_head - pub) & 0xFFFFu) << 16);
+            pub = my_head;
+        }
+    };
+
+    // flush: move up to `want` of the oldest HotRing entries to ColdSeg top, keeping at least
+    // `keep` in the ring (Fig 2(e): want = batch, keep = 0 when the ring is full;
+    // the demand-driven spill uses want = keep = rest/2)
+    auto flush = [&](uint32_t want, uint32_t keep) -> bool {
+        publish();
+        uint32_t t = 0;
+        if (lane == 0) { smem_lock(&S.lock[w]); t = ht_tail(ld_acquire_cta(&S.ht[w])); }
+        t = __shfl_sync(kFull, t, 0);
+        __syncwarp();                                 // ring entries written by lane 0 -> all lanes
+        const uint32_t rest = (my_head - t) & 0xFFFFu;
+        uint32_t kf = rest > keep ? rest - keep : 0u;
+        if (kf > want) kf = want;
+        if (kf == 0) {
+            if (lane == 0) smem_unlock(&S.lock[w]);
+            __syncwarp();
+            return true;
+        }
+        // map chunks covering [my_top, my_top + kf)
         bool ok = true;
-        while (ok && (unsigned long long)hi * kChunk < (unsigned long long)my_top + kBatch) {
+        while (ok && (unsigned long long)hi * kChunk < (unsigned long long)my_top + kf) {
             uint32_t c = 0;
             if (lane == 0) {
                 c = pool_alloc(P);
@@ -261,79 +350,83 @@ __global__ void __launch_bounds__(1024, 1) dfs_persistent_kernel(const KParams P
                         __nanosleep(64);
                     }
                     if (c != kEmptySlot) {
-                        P.chunk_consumed[c] = 0;
-                        asm volatile("st.relaxed.gpu.global.u32 [%0], %1;" ::"l"(slot), "r"(c) : "memory");
+                        st_relaxed_u32(&P.chunk_consumed[c], 0u);
+                        st_relaxed_u32(slot, c);
                     }
                 }
             }
             c = __shfl_sync(kFull, c, 0);
-            if (c == kEmptySlot) ok = false; else { ++hi; ++cnt[kCntChunks]; }
+            if (c == kEmptySlot) ok = false; else { ++hi; if (STATS && lane == 0) ++cnt[kCntChunks]; }
         }
         if (!ok) {
             if (lane == 0) { raise_error(P, kStatusENOMEM); smem_unlock(&S.lock[w]); }
             __syncwarp();
             return false;
         }
-        // vectorised copy: each lane moves pairs of entries (16 B); t and my_top are even
-        for (uint32_t q = 2u * lane; q < kBatch; q += 64u) {
-            const unsigned long long* src = ring + ((t + q) & (H - 1));
-            unsigned long long a = src[0], b = src[1];
-            uint32_t p = my_top + q;
-            uint32_t c = ld_relaxed_u32(&my_tab[(p >> kChunkLog2) & tmask]);
-            st_cg_v2(P.pool + ((size_t)c << kChunkLog2) + (p & (kChunk - 1)), a, b);
+        // warp copy, one 8-byte entry per lane per step
+        for (uint32_t q = lane; q < kf; q += 32u) {
+            const unsigned long long e = ring[(t + q) & (H - 1)];
+            const uint32_t p = my_top + q;
+            const uint32_t c = ld_relaxed_u32(&my_tab[(p >> kChunkLog2) & tmask]);
+            st_cg_u64(P.pool + ((size_t)c << kChunkLog2) + (p & (kChunk - 1)), e);
         }
-        __threadfence();
+        fence_release_gpu();                          // every lane: its stores before the publish
         __syncwarp();
         if (lane == 0) {
-            atomicAdd(&P.cold_tb[gw], (unsigned long long)kBatch << 32);   // publish top (release)
-            atomicAdd(&P.block_cold[blockIdx.x], (int)kBatch);
-            S.tail[w] = t + kBatch;
-            S.tailf[w] = t + kBatch;
+            atomicAdd(&P.cold_tb[gw], (unsigned long long)kf << 32);       // publish top
+            atomicAdd(&P.block_cold[blockIdx.x], (int)kf);
+            // advance tail (thieves are locked out; head is ours)
+            uint32_t old = ld_acquire_cta(&S.ht[w]);
+            for (;;) {
+                const uint32_t nw = (old & 0xFFFF0000u) | ((t + kf) & 0xFFFFu);
+                const uint32_t got = atom_cas_acquire_cta(&S.ht[w], old, nw);
+                if (got == old) break;
+                old = got;
+            }
+            S.tailf[w] = (t + kf) & 0xFFFFu;
             smem_unlock(&S.lock[w]);
         }
         __syncwarp();
-        my_top += kBatch;
-        ++cnt[kCntFlushes];
+        my_top += kf;
+        if (STATS && lane == 0) ++cnt[kCntFlushes];
         return true;
     };
 
     // push <v, idx> at head (Fig 2(c)); flushes first when full
     auto push = [&](uint32_t v, uint32_t idx) -> bool {
-        if (__shfl_sync(kFull, (int)(my_head - S.tailf[w]) >= H, 0)) {
-            if (!flush()) return false;
+        int full = 0;
+        if (lane == 0) full = ((my_head - S.tailf[w]) & 0xFFFFu) >= (uint32_t)H;
+        if (__shfl_sync(kFull, full, 0)) {
+            if (!flush(kBatch, 0u)) return false;
         }
-        if (lane == 0) {
-            ring[my_head & (H - 1)] = pack_entry(v, idx);
-            __threadfence_block();
-            S.head[w] = my_head + 1;
-        }
-        __syncwarp();
+        if (lane == 0) ring[my_head & (H - 1)] = pack_entry(v, idx);
         ++my_head;
+        if (((my_head - pub) & 0xFFFFu) >= P.pub_batch) publish();
         return true;
     };
 
-    // pop the newest HotRing entry (Fig 2(d)); THE protocol against tail-side thieves
+    // pop the newest HotRing entry (Fig 2(d)).  A private entry needs no synchronisation; at
+    // the published head one atomic decrement resolves the race with tail-side thieves (their
+    // CAS fails if the word changed)
     auto pop = [&](uint32_t& v, uint32_t& idx) -> bool {
         unsigned long long e = 0;
         int got = 0;
+        if (my_head != pub) {
+            if (lane == 0) e = ring[(my_head - 1u) & (H - 1)];
+            e = __shfl_sync(kFull, e, 0);
+            --my_head;
+            v = entry_v(e); idx = entry_i(e);
+            return true;
+        }
         if (lane == 0) {
-            const uint32_t h = my_head - 1;
-            S.head[w] = h;
-            __threadfence_block();
-            if ((int)(h - S.tail[w]) >= 0) { e = ring[h & (H - 1)]; got = 1; }
-            else {
-                // possible conflict with a thief (or empty): decide under the lock, where tail is
-                // final — a thief may still roll its reservation back (reading S12)
-                S.head[w] = h + 1;
-                smem_lock(&S.lock[w]);
-                if ((int)(h - S.tail[w]) >= 0) { S.head[w] = h; e = ring[h & (H - 1)]; got = 1; }
-                smem_unlock(&S.lock[w]);
-            }
+            const uint32_t old = atom_add_relaxed_cta(&S.ht[w], 0xFFFF0000u);   // head--
+            if (ht_rest(old) >= 1) { e = ring[(ht_head(old) - 1u) & (H - 1)]; got = 1; }
+            else atom_add_relaxed_cta(&S.ht[w], 0x10000u);                       // empty: undo
         }
         got = __shfl_sync(kFull, got, 0);
         if (!got) return false;
         e = __shfl_sync(kFull, e, 0);
-        --my_head;
+        --my_head; --pub;
         v = entry_v(e); idx = entry_i(e);
         return true;
     };
@@ -357,22 +450,19 @@ __global__ void __launch_bounds__(1024, 1) dfs_persistent_kernel(const KParams P
         k = __shfl_sync(kFull, k, 0);
         if (k == 0) return 0;
         const uint32_t base = my_top - k;
-        // ring is empty: my_head == tail (even); place entries oldest first
-        for (uint32_t q = 2u * lane; q < k; q += 64u) {
-            uint32_t p = base + q;
-            uint32_t c = ld_relaxed_u32(&my_tab[(p >> kChunkLog2) & tmask]);
-            unsigned long long a, b;
-            ld_cg_v2(P.pool + ((size_t)c << kChunkLog2) + (p & (kChunk - 1)), a, b);
-            unsigned long long* dst = ring + ((my_head + q) & (H - 1));
-            dst[0] = a; dst[1] = b;
+        // ring is empty (my_head == tail); place entries oldest first
+        for (uint32_t q = lane; q < k; q += 32u) {
+            const uint32_t p = base + q;
+            const uint32_t c = ld_relaxed_u32(&my_tab[(p >> kChunkLog2) & tmask]);
+            ring[(my_head + q) & (H - 1)] = ld_cg_u64(P.pool + ((size_t)c << kChunkLog2) + (p & (kChunk - 1)));
         }
         my_top = base;
         // release chunks that lie wholly above top + one spare chunk (never read by thieves)
         while (hi > 0 && (unsigned long long)(hi - 1) * kChunk >= (unsigned long long)my_top + kChunk) {
             if (lane == 0) {
                 uint32_t* slot = &my_tab[(hi - 1) & tmask];
-                uint32_t c = ld_relaxed_u32(slot);
-                asm volatile("st.relaxed.gpu.global.u32 [%0], %1;" ::"l"(slot), "r"(kEmptySlot) : "memory");
+                const uint32_t c = ld_relaxed_u32(slot);
+                st_relaxed_u32(slot, kEmptySlot);
                 pool_free(P, c);
             }
             --hi;
@@ -380,75 +470,207 @@ __global__ void __launch_bounds__(1024, 1) dfs_persistent_kernel(const KParams P
         __syncwarp();
         if (lane == 0) {
             atomicSub(&P.block_cold[blockIdx.x], (int)k);
-            __threadfence_block();
-            S.head[w] = my_head + k;
+            atom_add_release_cta(&S.ht[w], k << 16);              // publish (ring was empty)
         }
-        __syncwarp();
-        my_head += k;
-        ++cnt[kCntRefills];
+        my_head += k; pub = my_head;
+        if (STATS && lane == 0) ++cnt[kCntRefills];
         return k;
     };
 
     auto set_done_local = [&]() {
         if (lane == 0) S.done = 1;
     };
+    auto deregister = [&]() {      // lane 0: leave the busy count; the last one raises done
+        if (atomicSub(&P.ctl->busy, 1u) == 1u) { atomicExch(&P.ctl->done, 1u); S.done = 1; }
+    };
+
+    // diagnostics: block 0 / warp 0 samples the busy counter every timeline_dt_ns
+    unsigned int tl_next = 0;
+    auto sample = [&]() {
+        if (P.timeline && blockIdx.x == 0 && w == 0 && lane == 0) {
+            const unsigned long long now = globaltimer() - t_start;
+            const unsigned int slot = (unsigned int)(now / P.timeline_dt_ns);
+            if (slot >= tl_next && slot < P.timeline_len) {
+                P.timeline[slot] = *(volatile unsigned int*)&P.ctl->busy + 1u;   // 0 = no sample
+                tl_next = slot + 1;
+            }
+        }
+    };
 
     // ---------------------------------------------------------------- main loop (Alg 2)
     for (;;) {
         if (has_top) {
-            // ===== warp-level expansion step (Alg 1 l.5-12 over a 32-wide window) =====
+            // ===== warp-level expansion step (Alg 1 l.5-12 over one window) =====
+            // Window = positions [a, a + kWin), a = i rounded down to a multiple of VEC; lane k
+            // holds positions a+VEC*k .. a+VEC*k+VEC-1.  Positions outside [i, end) are masked.
             if (!have_win) {
                 const uint32_t e2 = need_end ? __ldg(P.rp + u + 1) : end;
-                const uint32_t idx = i + lane;
-                nb = (idx < P.m) ? __ldg(P.col + idx) : -1;
+                load_window(i & ~(uint32_t)(VEC - 1), P.m, nbv);
                 end = e2; need_end = false;
             }
-            ++cnt[kCntWindows];
-            const bool valid = (i + lane) < end;
-            uint32_t wbits = kFull, prs = 0, pre = 0;
-            if (valid) {
-                wbits = __ldcg(P.bitmap + ((uint32_t)nb >> 5));
-                if (lane < kPrefetchLanes) { prs = __ldg(P.rp + nb); pre = __ldg(P.rp + nb + 1); }
+            if (STATS && lane == 0) ++cnt[kCntWindows];
+            const uint32_t a = i & ~(uint32_t)(VEC - 1);
+            const uint32_t q0 = a + (uint32_t)VEC * lane;
+            // long list (hubs): load the next window now so it is in flight while this window's
+            // probes resolve (a sequential scan then costs one probe round trip per window)
+            int nxt[VEC];
+            const bool have_nxt = a + kWin < end;
+            if (have_nxt) load_window(a + kWin, P.m, nxt);
+            // speculative claim (fresh child only): the first position whose neighbour is not the
+            // parent we came from is, if unvisited, exactly Alg 1's next tree edge; claiming it
+            // in parallel with the probes removes the probe -> claim round trip
+            int sk = -1, se = 0;
+            uint32_t sv = 0, s_old = 0, s_rs = 0, s_re = 0;
+            if ((P.speculate == 1 || (P.speculate == 2 && VEC == 1)) && spec_ok) {
+                uint32_t vm = 0;
+#pragma unroll
+                for (int e = 0; e < VEC; ++e) {
+                    const uint32_t p = q0 + e;
+                    if (p >= i && p < end && (uint32_t)nbv[e] != par) vm |= 1u << e;
+                }
+                const uint32_t vb = __ballot_sync(kFull, vm != 0);
+                if (vb) {
+                    sk = __ffs(vb) - 1;
+                    se = __ffs(__shfl_sync(kFull, vm, sk)) - 1;
+                    int pick = nbv[0];
+#pragma unroll
+                    for (int f = 1; f < VEC; ++f) if (se == f) pick = nbv[f];
+                    sv = (uint32_t)__shfl_sync(kFull, pick, sk);
+                    if (lane == 0) s_old = atomicOr(P.bitmap + (sv >> 5), 1u << (sv & 31));
+                    s_rs = __ldg(P.rp + sv); s_re = __ldg(P.rp + sv + 1);
+                }
             }
-            const bool cand = valid && !((wbits >> (nb & 31)) & 1u);
-            uint32_t unv = __ballot_sync(kFull, cand);
+            // probe visited bits; the lanes holding the first 8 positions also prefetch their
+            // candidates' row_ptr pairs so a claim can load the child's window immediately
+            uint32_t m4 = 0;
+            uint32_t prs[VEC], pre[VEC];
+#pragma unroll
+            for (int e = 0; e < VEC; ++e) {
+                const uint32_t p = q0 + e;
+                const int x = nbv[e];
+                prs[e] = 0; pre[e] = 0;
+                if (p >= i && p < end) {
+                    const uint32_t word = __ldcg(P.bitmap + ((uint32_t)x >> 5));
+                    if (lane < kPfLanes) { prs[e] = __ldg(P.rp + x); pre[e] = __ldg(P.rp + x + 1); }
+                    if (!((word >> (x & 31)) & 1u)) m4 |= 1u << e;
+                }
+            }
             bool descended = false;
-            while (unv) {
-                const int j = __ffs(unv) - 1;                    // first unvisited in CSR order
-                const uint32_t v = (uint32_t)__shfl_sync(kFull, nb, j);
-                uint32_t vrs = __shfl_sync(kFull, prs, j), vre = __shfl_sync(kFull, pre, j);
-                if (j >= kPrefetchLanes) { vrs = __ldg(P.rp + v); vre = __ldg(P.rp + v + 1); }
+            if (sk >= 0) {
+                if (lane == sk) m4 &= ~(1u << se);               // p0 is claimed either way
+                s_old = __shfl_sync(kFull, s_old, 0);
+                if (!(s_old & (1u << (sv & 31)))) {
+                    // speculative claim won: <u, next candidate> below, child on top
+                    int cnb[VEC];
+                    load_window(s_rs & ~(uint32_t)(VEC - 1), s_re, cnb);
+                    if (STATS && lane == 0) ++cnt[kCntClaims];
+                    if (lane == 0) P.parent[sv] = (int32_t)u;                       // Alg 1 l.10
+                    const uint32_t mine = (lane == sk) ? (m4 & ~((2u << se) - 1u)) : (lane > sk ? m4 : 0u);
+                    const uint32_t later = __ballot_sync(kFull, mine != 0);
+                    uint32_t ni = a + kWin;
+                    if (later) {
+                        const int k2 = __ffs(later) - 1;
+                        const uint32_t m2 = __shfl_sync(kFull, mine, k2);
+                        ni = a + (uint32_t)VEC * (uint32_t)k2 + (uint32_t)(__ffs(m2) - 1);
+                    }
+                    if (ni < end) {
+                        if (!push(u, ni)) goto exit_loop;
+                    }
+                    par = u;
+                    u = sv; i = s_rs; end = s_re; have_win = true; need_end = false; spec_ok = true;
+#pragma unroll
+                    for (int f = 0; f < VEC; ++f) nbv[f] = cnb[f];
+                    descended = true;
+                } else if (lane == 0) {
+                    ++cnt[kCntFailedClaims];
+                }
+            }
+            uint32_t any = descended ? 0u : __ballot_sync(kFull, m4 != 0);
+            while (any) {
+                const int k = __ffs(any) - 1;                      // first lane with a candidate
+                const uint32_t mk = __shfl_sync(kFull, m4, k);
+                const int e = __ffs(mk) - 1;                       // first candidate in CSR order
+                int mine_nb = nbv[0];
+                uint32_t mine_rs = prs[0], mine_re = pre[0];
+#pragma unroll
+                for (int f = 1; f < VEC; ++f)
+                    if (e == f) { mine_nb = nbv[f]; mine_rs = prs[f]; mine_re = pre[f]; }
+                const uint32_t v = (uint32_t)__shfl_sync(kFull, mine_nb, k);
+                uint32_t vrs, vre;
+                if (k < kPfLanes) {
+                    vrs = __shfl_sync(kFull, mine_rs, k); vre = __shfl_sync(kFull, mine_re, k);
+                } else {
+                    vrs = __ldg(P.rp + v); vre = __ldg(P.rp + v + 1);
+                }
                 const uint32_t bit = 1u << (v & 31);
                 uint32_t old = 0;
                 if (lane == 0) old = atomicOr(P.bitmap + (v >> 5), bit);          // claim
                 // speculative load of the child's first window, overlapping the claim
-                const uint32_t cidx = vrs + lane;
-                const int cnb = (cidx < P.m) ? __ldg(P.col + cidx) : -1;
+                int cnb[VEC];
+                load_window(vrs & ~(uint32_t)(VEC - 1), vre, cnb);
                 old = __shfl_sync(kFull, old, 0);
                 if (!(old & bit)) {
-                    ++cnt[kCntClaims];
+                    if (STATS && lane == 0) ++cnt[kCntClaims];
                     if (lane == 0) P.parent[v] = (int32_t)u;                        // Alg 1 l.10
-                    const uint32_t ni = i + (uint32_t)j + 1u;
-                    // Alg 1 l.8 + l.11: keep <u, ni> below the child unless u is exhausted
+                    // Alg 1 l.8 + l.11: keep <u, ni> below the child unless u is exhausted.
+                    // Positions after the claimed one whose probe saw a claimed target stay
+                    // claimed (claims are monotone), so scanning them again cannot change
+                    // anything: resume at the next still-unvisited candidate, or past the window.
+                    const uint32_t mine = (lane == k) ? (m4 & ~((2u << e) - 1u)) : (lane > k ? m4 : 0u);
+                    const uint32_t later = __ballot_sync(kFull, mine != 0);
+                    uint32_t ni = a + kWin;
+                    if (later) {
+                        const int k2 = __ffs(later) - 1;
+                        const uint32_t m2 = __shfl_sync(kFull, mine, k2);
+                        ni = a + (uint32_t)VEC * (uint32_t)k2 + (uint32_t)(__ffs(m2) - 1);
+                    }
                     if (ni < end) {
                         if (!push(u, ni)) goto exit_loop;
                     }
-                    u = v; i = vrs; end = vre; nb = cnb; have_win = true; need_end = false;
+                    par = u;
+                    u = v; i = vrs; end = vre; have_win = true; need_end = false; spec_ok = true;
+#pragma unroll
+                    for (int f = 0; f < VEC; ++f) nbv[f] = cnb[f];
                     descended = true;
                     break;
                 }
-                ++cnt[kCntFailedClaims];
-                unv &= unv - 1;                                   // lost the race: next candidate
+                if (STATS && lane == 0) ++cnt[kCntFailedClaims];
+                if (lane == k) m4 &= ~(1u << e);                  // lost the race: next candidate
+                any = __ballot_sync(kFull, m4 != 0);
             }
             if (!descended) {
-                i += 32;
-                have_win = false;
-                if (i >= end) {                                   // Alg 1 l.14: pop
+                i = a + kWin;
+                spec_ok = false;
+                if (have_nxt) {                                   // next window already loaded
+#pragma unroll
+                    for (int f = 0; f < VEC; ++f) nbv[f] = nxt[f];
+                    have_win = true;
+                } else {
+                    have_win = false;                             // i >= end: Alg 1 l.14: pop
                     has_top = pop(u, i);
                     need_end = true;
                 }
             }
-            if ((++iter & 1023u) == 0) {
+            ++iter;
+            if ((iter & 31u) == 0) sample();
+            if (P.spill && (iter & 31u) == 0) {
+                // demand-driven spill: many warps idle and a deep HotRing -> make the oldest half
+                // of it visible to other blocks (Alg 4 steals ColdSeg bottoms only)
+                uint32_t want = 0;
+                if (lane == 0) {
+                    const uint32_t rest = (my_head - ht_tail(ld_acquire_cta(&S.ht[w]))) & 0xFFFFu;
+                    if (rest >= 2u * (uint32_t)P.cold_cutoff) {
+                        const uint32_t busy = *(volatile unsigned int*)&P.ctl->busy;
+                        if ((int)(gridDim.x * W - busy) >= P.spill_idle) want = rest / 2;
+                    }
+                }
+                want = __shfl_sync(kFull, want, 0);
+                if (want) {
+                    if (!flush(want, want)) break;
+                    if (STATS && lane == 0) ++cnt[kCntSpills];
+                }
+            }
+            if ((iter & 1023u) == 0) {
                 const int stop = __shfl_sync(kFull, (int)(*(volatile unsigned int*)&P.ctl->done), 0);
                 if (stop) { set_done_local(); break; }
                 if (__shfl_sync(kFull, (int)(globaltimer() - t_start > P.timeout_ns), 0)) {
@@ -472,12 +694,13 @@ __global__ void __launch_bounds__(1024, 1) dfs_persistent_kernel(const KParams P
             active = false;
             if (lane == 0) {
                 atomicAnd(&S.warp_mask, ~(1u << w));
-                if (atomicSub(&P.ctl->busy, 1u) == 1u) { atomicExch(&P.ctl->done, 1u); S.done = 1; }
+                deregister();
             }
             __syncwarp();
         }
         bool got_work = false;
         uint32_t backoff = 32;
+        t_idle0 = STATS ? globaltimer() : 0ull;
         while (!got_work) {
             if (__shfl_sync(kFull, S.done, 0)) goto exit_loop;
             if (w == 0) {
@@ -494,52 +717,57 @@ __global__ void __launch_bounds__(1024, 1) dfs_persistent_kernel(const KParams P
             // ---- Alg 3: intra-block stealing from the peer HotRing with max hot_rest ----
             if (P.intra && W > 1) {
                 int rest = -1;
-                if (lane < W && lane != w) rest = (int)(S.head[lane] - S.tail[lane]);
+                if (lane < W && lane != w) rest = ht_rest(*(volatile uint32_t*)&S.ht[lane]);
                 const int best = __reduce_max_sync(kFull, rest);
                 if (best >= P.hot_cutoff) {
                     const int vwarp = __ffs(__ballot_sync(kFull, rest == best)) - 1;
-                    ++cnt[kCntStealAttempts];
+                    if (STATS && lane == 0) ++cnt[kCntStealAttempts];
                     uint32_t ok = 0, t = 0;
                     if (lane == 0) {
                         atomicAdd(&P.ctl->busy, 1u);                 // register before reserving
                         if (smem_trylock(&S.lock[vwarp])) {
-                            t = S.tail[vwarp];
-                            if ((int)(S.head[vwarp] - t) >= P.hot_cutoff) {
-                                S.tail[vwarp] = t + hs;              // reserve (Alg 3 l.13-15)
-                                __threadfence_block();
-                                if ((int)(S.head[vwarp] - (t + hs)) >= 0) ok = 1;
-                                else S.tail[vwarp] = t;              // owner raced us: roll back
+                            uint32_t old = *(volatile uint32_t*)&S.ht[vwarp];
+                            for (int tries = 0; tries < 8; ++tries) {
+                                if (ht_rest(old) < P.hot_cutoff) break;
+                                t = ht_tail(old);
+                                const uint32_t nw = (old & 0xFFFF0000u) | ((t + hs) & 0xFFFFu);
+                                const uint32_t got = atom_cas_acquire_cta(&S.ht[vwarp], old, nw);   // reserve
+                                if (got == old) { ok = 1; break; }
+                                old = got;
                             }
                             if (!ok) smem_unlock(&S.lock[vwarp]);
                         }
-                        if (!ok) {
-                            if (atomicSub(&P.ctl->busy, 1u) == 1u) { atomicExch(&P.ctl->done, 1u); S.done = 1; }
-                        }
+                        if (!ok) deregister();
                     }
                     ok = __shfl_sync(kFull, ok, 0);
                     if (ok) {
                         t = __shfl_sync(kFull, t, 0);
+                        __syncwarp();                                // lane 0's acquire -> all lanes
                         const unsigned long long* vring = rings + (size_t)vwarp * H;
                         if (lane < (int)hs) ring[(my_head + lane) & (H - 1)] = vring[(t + lane) & (H - 1)];
                         __syncwarp();
                         if (lane == 0) {
-                            __threadfence_block();
-                            S.tailf[vwarp] = t + hs;                 // slots reusable by the owner
+                            S.tailf[vwarp] = (t + hs) & 0xFFFFu;     // slots reusable by the owner
                             smem_unlock(&S.lock[vwarp]);
-                            S.head[w] = my_head + hs;
+                            atom_add_release_cta(&S.ht[w], hs << 16); // publish into our ring
                             atomicOr(&S.warp_mask, 1u << w);         // mark active
                         }
                         __syncwarp();
-                        my_head += hs;
-                        ++cnt[kCntIntraSteals];
+                        my_head += hs; pub = my_head;
+                        if (STATS && lane == 0) ++cnt[kCntIntraSteals];
                         got_work = true;
                         break;
                     }
                 }
             }
-            // ---- Alg 4: leader warp of an idle block steals from a remote ColdSeg bottom ----
-            if (P.inter && w == 0 && gridDim.x > 1 &&
-                __shfl_sync(kFull, *(volatile unsigned int*)&S.warp_mask, 0) == 0u) {
+            // ---- Alg 4: steal c_s entries from a remote ColdSeg bottom ----
+            int token = 0;
+            if (P.inter && gridDim.x > 1 &&
+                (P.inter_any || (w == 0 && __shfl_sync(kFull, *(volatile unsigned int*)&S.warp_mask, 0) == 0u))) {
+                if (lane == 0) token = smem_trylock(&S.inter_token) ? 1 : 0;
+                token = __shfl_sync(kFull, token, 0);
+            }
+            if (token) {
                 const int nB = gridDim.x;
                 // cumulative ColdSeg load per block (reading S14); active = load > 0
                 int vb = -1;
@@ -547,7 +775,7 @@ __global__ void __launch_bounds__(1024, 1) dfs_persistent_kernel(const KParams P
                     int nact = 0;
                     for (int b0 = 0; b0 < nB; b0 += 32) {
                         const int b = b0 + lane;
-                        const bool a = b < nB && b != (int)blockIdx.x && ld_relaxed_s32(&P.block_cold[b]) > 0;
+                        const bool a = b < nB && (P.inter_any || b != (int)blockIdx.x) && ld_relaxed_s32(&P.block_cold[b]) > 0;
                         nact += __popc(__ballot_sync(kFull, a));
                     }
                     if (nact > 0) {
@@ -558,7 +786,7 @@ __global__ void __launch_bounds__(1024, 1) dfs_persistent_kernel(const KParams P
                         int pick1 = -1, pick2 = -1, load1 = 0, load2 = 0, seen = 0;
                         for (int b0 = 0; b0 < nB && (pick1 < 0 || pick2 < 0); b0 += 32) {
                             const int b = b0 + lane;
-                            const int load = (b < nB && b != (int)blockIdx.x) ? ld_relaxed_s32(&P.block_cold[b]) : 0;
+                            const int load = (b < nB && (P.inter_any || b != (int)blockIdx.x)) ? ld_relaxed_s32(&P.block_cold[b]) : 0;
                             const uint32_t m = __ballot_sync(kFull, load > 0);
                             const int c = __popc(m);
                             for (int which = 0; which < 2; ++which) {
@@ -575,20 +803,20 @@ __global__ void __launch_bounds__(1024, 1) dfs_persistent_kernel(const KParams P
                         else vb = (load2 > load1 || (load2 == load1 && pick2 < pick1)) ? pick2 : pick1;
                     }
                 }
+                if (STATS && lane == 0) ++cnt[kCntInterScans];
                 if (vb >= 0) {
                     // victim warp: max cold_rest = top - bottom (Alg 4 l.9-15)
                     const int WV = W;                 // all blocks have W warps
                     int rest = -1;
-                    unsigned long long word = 0;
                     if (lane < WV) {
-                        word = ld_relaxed_u64(&P.cold_tb[vb * WV + lane]);
+                        const unsigned long long word = ld_relaxed_u64(&P.cold_tb[vb * WV + lane]);
                         rest = (int)((uint32_t)(word >> 32) - (uint32_t)word);
                     }
                     const int best = __reduce_max_sync(kFull, rest);
                     if (best >= P.cold_cutoff) {
                         const int vwl = __ffs(__ballot_sync(kFull, rest == best)) - 1;
                         const int vwg = vb * WV + vwl;
-                        ++cnt[kCntStealAttempts];
+                        if (STATS && lane == 0) ++cnt[kCntStealAttempts];
                         uint32_t ok = 0, bot = 0;
                         if (lane == 0) {
                             atomicAdd(&P.ctl->busy, 1u);
@@ -597,60 +825,58 @@ __global__ void __launch_bounds__(1024, 1) dfs_persistent_kernel(const KParams P
                                 const uint32_t top = (uint32_t)(old >> 32), b = (uint32_t)old;
                                 if ((int)(top - b) < P.cold_cutoff) break;
                                 const unsigned long long nw = ((unsigned long long)top << 32) | (uint32_t)(b + cs);
-                                const unsigned long long got = atomicCAS(&P.cold_tb[vwg], old, nw);
+                                const unsigned long long got = atomicCAS(&P.cold_tb[vwg], old, nw);   // reserve
                                 if (got == old) { ok = 1; bot = b; break; }
                                 old = got;
                             }
-                            if (!ok) {
-                                if (atomicSub(&P.ctl->busy, 1u) == 1u) { atomicExch(&P.ctl->done, 1u); S.done = 1; }
-                            }
+                            if (!ok) deregister();
                         }
                         ok = __shfl_sync(kFull, ok, 0);
                         if (ok) {
                             bot = __shfl_sync(kFull, bot, 0);
-                            __threadfence();                                    // acquire (Alg 4 l.21)
+                            // remote transfer (Alg 4 l.21-22): L2 loads, addresses from the CAS
                             uint32_t* vtab = P.chunk_tab + ((size_t)vwg << P.tab_log2);
                             uint32_t* slot = &vtab[(bot >> kChunkLog2) & tmask];
                             const uint32_t c = ld_relaxed_u32(slot);
                             const unsigned long long* src = P.pool + ((size_t)c << kChunkLog2) + (bot & (kChunk - 1));
-                            if (2u * lane < cs) {
-                                unsigned long long a, b;
-                                ld_cg_v2(src + 2 * lane, a, b);
-                                unsigned long long* dst = ring + ((my_head + 2u * lane) & (H - 1));
-                                dst[0] = a; dst[1] = b;
-                            }
+                            for (uint32_t q = lane; q < cs; q += 32u)
+                                ring[(my_head + q) & (H - 1)] = ld_cg_u64(src + q);
                             __syncwarp();
                             if (lane == 0) {
-                                __threadfence();
                                 const uint32_t before = atomicAdd(&P.chunk_consumed[c], cs);
                                 if (before + cs == kChunk) {                   // chunk fully consumed
-                                    asm volatile("st.relaxed.gpu.global.u32 [%0], %1;" ::"l"(slot), "r"(kEmptySlot) : "memory");
+                                    st_relaxed_u32(slot, kEmptySlot);
                                     pool_free(P, c);
                                 }
                                 atomicSub(&P.block_cold[vb], (int)cs);
-                                __threadfence_block();
-                                S.head[w] = my_head + cs;
+                                atom_add_release_cta(&S.ht[w], cs << 16);      // publish into our ring
                                 atomicOr(&S.warp_mask, 1u << w);               // mark w, b active
                             }
                             __syncwarp();
-                            my_head += cs;
-                            ++cnt[kCntInterSteals];
+                            my_head += cs; pub = my_head;
+                            if (STATS && lane == 0) ++cnt[kCntInterSteals];
+                            if (lane == 0) smem_unlock(&S.inter_token);
                             got_work = true;
                             break;
                         }
                     }
                 }
             }
+            if (token && lane == 0) smem_unlock(&S.inter_token);
+            sample();
             __nanosleep(backoff);
-            if (backoff < 2048) backoff <<= 1;
+            if (backoff < P.backoff_max_ns) backoff <<= 1;
         }
         // got work: it is in the HotRing
+        if (STATS && lane == 0) cnt[kCntIdleNs] += globaltimer() - t_idle0;
+        t_idle0 = 0;
         active = true;
         has_top = pop(u, i);
         need_end = true; have_win = false;
     }
 exit_loop:
     __syncwarp();
+    if (STATS && !active && t_idle0 && lane == 0) cnt[kCntIdleNs] += globaltimer() - t_idle0;
     // release the ColdSeg chunks still mapped by this warp so the chunk table is all-empty
     // for the next run (thieves free the chunks they fully consume)
     {
@@ -659,16 +885,14 @@ exit_loop:
         const uint32_t lo = bot >> kChunkLog2;     // chunks below were freed by the thieves
         for (uint32_t k = lo + lane; k < hi; k += 32) {
             uint32_t* slot = &my_tab[k & tmask];
-            const uint32_t c = ld_relaxed_u32(slot);
-            if (c != kEmptySlot) {
-                asm volatile("st.relaxed.gpu.global.u32 [%0], %1;" ::"l"(slot), "r"(kEmptySlot) : "memory");
-            }
+            if (ld_relaxed_u32(slot) != kEmptySlot) st_relaxed_u32(slot, kEmptySlot);
         }
     }
-    if (P.collect_stats) {
+    if (STATS) {
 #pragma unroll
         for (int k = 0; k < kNumCounters; ++k)
             if (lane == 0 && cnt[k]) atomicAdd(&P.ctl->counters[k], cnt[k]);
+        __syncwarp();
     }
 }
 

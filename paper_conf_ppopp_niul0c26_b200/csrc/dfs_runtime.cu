@@ -32,6 +32,16 @@ bool is_device_ptr(const void* p) {
     return a.type == cudaMemoryTypeDevice || a.type == cudaMemoryTypeManaged;
 }
 
+// the 8 instantiations of the persistent kernel: [vec128][wmax16][stats]
+const void* const* kernel_table() {
+    static const void* const t[8] = {
+        (const void*)dfs_persistent_kernel<kRing, 1, 32, false>, (const void*)dfs_persistent_kernel<kRing, 1, 32, true>,
+        (const void*)dfs_persistent_kernel<kRing, 1, 16, false>, (const void*)dfs_persistent_kernel<kRing, 1, 16, true>,
+        (const void*)dfs_persistent_kernel<kRing, 4, 32, false>, (const void*)dfs_persistent_kernel<kRing, 4, 32, true>,
+        (const void*)dfs_persistent_kernel<kRing, 4, 16, false>, (const void*)dfs_persistent_kernel<kRing, 4, 16, true>};
+    return t;
+}
+
 size_t smem_bytes(int warps) {
     return ((sizeof(SmemCtl) + 15) & ~size_t(15)) + (size_t)warps * kRing * sizeof(unsigned long long);
 }
@@ -62,6 +72,8 @@ struct dfs_graph {
     bool tab_dirty = false;
     int64_t launches = 0;
     cudaEvent_t ev0 = nullptr, ev1 = nullptr, evk0 = nullptr, evk1 = nullptr;
+    unsigned int* d_timeline = nullptr;   // diagnostics (dfs_debug_timeline)
+    unsigned int timeline_len = 0, timeline_dt_ns = 0;
 };
 
 static void free_graph(dfs_graph* g) {
@@ -72,6 +84,7 @@ static void free_graph(dfs_graph* g) {
     cudaFree(g->d_rp); cudaFree(g->d_col); cudaFree(g->d_bitmap); cudaFree(g->d_parent);
     cudaFree(g->d_cold_tb); cudaFree(g->d_tab); cudaFree(g->d_pool); cudaFree(g->d_consumed);
     cudaFree(g->d_next); cudaFree(g->d_block_cold); cudaFree(g->d_ctl); cudaFree(g->d_count2);
+    cudaFree(g->d_timeline);
     if (g->ev0) cudaEventDestroy(g->ev0);
     if (g->ev1) cudaEventDestroy(g->ev1);
     if (g->evk0) cudaEventDestroy(g->evk0);
@@ -87,8 +100,8 @@ void dfs_options_default(dfs_options* o) {
     std::memset(o, 0, sizeof(*o));
     o->blocks = 0;
     o->warps_per_block = 32;
-    o->hot_cutoff = 32;
-    o->cold_cutoff = 64;
+    o->hot_cutoff = 2;           // paper: 32; B200 sweep: 2
+    o->cold_cutoff = 2;          // paper: 64; B200 sweep: 2
     o->deterministic = 0;
     o->intra_steal = 1;
     o->inter_steal = 1;
@@ -96,6 +109,13 @@ void dfs_options_default(dfs_options* o) {
     o->timeout_ms = 120000;
     o->seed = 0x5EEDu;
     o->collect_stats = 0;
+    o->spill = 1;
+    o->inter_any = 1;
+    o->spill_idle = 32;
+    o->backoff_max_ns = 2048;
+    o->window = 0;
+    o->pub_batch = 1;
+    o->speculate = 2;
 }
 
 int dfs_last_error(void) { return g_last_error; }
@@ -127,12 +147,15 @@ dfs_graph* dfs_graph_create(const int64_t* row_ptr, const int32_t* col_idx, int6
     if (cudaGetDeviceProperties(&prop, g->device) != cudaSuccess) { cudaGetLastError(); delete g; fail(DFS_ECUDA); return nullptr; }
     g->sms = prop.multiProcessorCount;
     const size_t sm32 = smem_bytes(32);
-    if (cudaFuncSetAttribute(dfs_persistent_kernel<kRing>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                             (int)sm32) != cudaSuccess) {
-        cudaGetLastError(); delete g; fail(DFS_ECUDA); return nullptr;
+    bool attr_ok = true;
+    for (int kf = 0; kf < 8; ++kf) {
+        const void* f = kernel_table()[kf];
+        if (f && cudaFuncSetAttribute(f, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm32) != cudaSuccess)
+            attr_ok = false;
     }
+    if (!attr_ok) { cudaGetLastError(); delete g; fail(DFS_ECUDA); return nullptr; }
     int per_sm = 0;
-    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, dfs_persistent_kernel<kRing>, 1024, sm32) !=
+    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, dfs_persistent_kernel<kRing, 4, 32, false>, 1024, sm32) !=
             cudaSuccess || per_sm < 1) {
         cudaGetLastError(); per_sm = 1;
     }
@@ -151,7 +174,7 @@ dfs_graph* dfs_graph_create(const int64_t* row_ptr, const int32_t* col_idx, int6
     bool ok = true;
     auto A = [&](void** p, size_t bytes) { if (ok && cudaMalloc(p, bytes ? bytes : 16) != cudaSuccess) ok = false; };
     A((void**)&g->d_rp, (size_t)(n + 1) * sizeof(uint32_t));
-    A((void**)&g->d_col, (size_t)m * sizeof(int32_t));
+    A((void**)&g->d_col, (size_t)(m + 8) * sizeof(int32_t));     // padded for 128-bit window loads
     A((void**)&g->d_bitmap, nwords * sizeof(uint32_t));
     A((void**)&g->d_cold_tb, (size_t)n_warps * sizeof(unsigned long long));
     A((void**)&g->d_tab, g->tab_words * sizeof(uint32_t));
@@ -197,6 +220,7 @@ dfs_graph* dfs_graph_create(const int64_t* row_ptr, const int32_t* col_idx, int6
     if (cudaGetLastError() != cudaSuccess) { free_graph(g); fail(DFS_ECUDA); return nullptr; }
     if (bad || hbad) { free_graph(g); fail(DFS_EINVAL); return nullptr; }
     cudaMemset(g->d_tab, 0xFF, g->tab_words * sizeof(uint32_t));   // all chunk slots empty
+    cudaMemset(g->d_col + m, 0xFF, 8 * sizeof(int32_t));            // padding (never a valid position)
     if (cudaDeviceSynchronize() != cudaSuccess) { cudaGetLastError(); free_graph(g); fail(DFS_ECUDA); return nullptr; }
     return g;
 }
@@ -218,6 +242,35 @@ int dfs_graph_info(const dfs_graph* g, int64_t* n, int64_t* m, int32_t* device) 
 }
 
 int64_t dfs_launch_count(const dfs_graph* g) { return g ? g->launches : -1; }
+
+int dfs_debug_timeline(dfs_graph* g, uint32_t len, uint32_t dt_ns, uint32_t* out) {
+    if (!g || (len > 0 && dt_ns == 0)) return fail(DFS_EINVAL);
+    if (len == 0) {                       // disable
+        cudaFree(g->d_timeline);
+        g->d_timeline = nullptr; g->timeline_len = 0;
+        return DFS_OK;
+    }
+    if (g->d_timeline && g->timeline_len == len && out == nullptr) return DFS_OK;
+    if (!g->d_timeline || g->timeline_len != len) {
+        cudaFree(g->d_timeline);
+        g->d_timeline = nullptr;
+        if (cudaMalloc(&g->d_timeline, (size_t)len * sizeof(uint32_t)) != cudaSuccess) {
+            cudaGetLastError();
+            g->timeline_len = 0;
+            return fail(DFS_ENOMEM);
+        }
+        cudaMemset(g->d_timeline, 0, (size_t)len * sizeof(uint32_t));
+        g->timeline_len = len; g->timeline_dt_ns = dt_ns;
+        return DFS_OK;
+    }
+    // copy out the samples of the last run, then clear
+    if (cudaMemcpy(out, g->d_timeline, (size_t)len * sizeof(uint32_t), cudaMemcpyDeviceToHost) != cudaSuccess) {
+        cudaGetLastError();
+        return fail(DFS_ECUDA);
+    }
+    cudaMemset(g->d_timeline, 0, (size_t)len * sizeof(uint32_t));
+    return DFS_OK;
+}
 
 }  // extern "C"
 
@@ -246,11 +299,21 @@ static int launch_one(dfs_graph* g, int32_t root, int32_t* d_out, const dfs_opti
     P.hot_cutoff = o.hot_cutoff; P.cold_cutoff = o.cold_cutoff;
     P.intra = o.intra_steal; P.inter = o.inter_steal; P.policy = o.victim_policy;
     P.collect_stats = o.collect_stats;
+    P.spill = o.spill;
+    P.spill_idle = o.spill_idle > 0 ? o.spill_idle : 32;
+    P.inter_any = o.inter_any;
+    P.backoff_max_ns = o.backoff_max_ns > 0 ? (unsigned)o.backoff_max_ns : 2048u;
+    P.pub_batch = o.pub_batch > 0 ? (uint32_t)o.pub_batch : 4u;
+    P.speculate = o.speculate;
+    P.timeline = g->d_timeline;
+    P.timeline_len = g->timeline_len;
+    P.timeline_dt_ns = g->timeline_dt_ns;
     P.timeout_ns = (unsigned long long)o.timeout_ms * 1000000ull;
     P.seed = o.seed;
     void* args[] = {(void*)&P};
     if (timed) cudaEventRecord(g->evk0, s);
-    cudaError_t e = cudaLaunchCooperativeKernel((const void*)dfs_persistent_kernel<kRing>, dim3(blocks),
+    const void* kfn = kernel_table()[(o.window == 128 ? 4 : 0) + (warps <= 16 ? 2 : 0) + (o.collect_stats ? 1 : 0)];
+    cudaError_t e = cudaLaunchCooperativeKernel(kfn, dim3(blocks),
                                                 dim3(32 * warps), args, smem_bytes(warps), s);
     if (e != cudaSuccess) { cudaGetLastError(); return DFS_ECUDA; }
     if (timed) cudaEventRecord(g->evk1, s);
@@ -264,14 +327,17 @@ static int launch_one(dfs_graph* g, int32_t root, int32_t* d_out, const dfs_opti
 static int resolve_options(const dfs_graph* g, const dfs_options* in, dfs_options& o, int& blocks, int& warps) {
     dfs_options_default(&o);
     if (in) o = *in;
-    if (o.hot_cutoff == 0) o.hot_cutoff = 32;
-    if (o.cold_cutoff == 0) o.cold_cutoff = 64;
+    if (o.hot_cutoff == 0) o.hot_cutoff = 2;
+    if (o.cold_cutoff == 0) o.cold_cutoff = 2;
     if (o.timeout_ms <= 0) o.timeout_ms = 120000;
-    // h_s must be even, <= 32 lanes; c_s even power of two dividing the chunk (tail/bottom parity)
+    // h_s = hot_cutoff/2 in [1, 32] (one lane per entry); c_s = cold_cutoff/2 a power of two
+    // <= 64 (dividing the ColdSeg chunk, so a steal never straddles chunks)
     const int hs = o.hot_cutoff / 2, cs = o.cold_cutoff / 2;
-    if (o.hot_cutoff % 4 != 0 || hs < 2 || hs > 32) return DFS_EINVAL;
-    if (o.cold_cutoff % 4 != 0 || cs < 2 || cs > 64 || (cs & (cs - 1)) != 0) return DFS_EINVAL;
+    if (o.hot_cutoff % 2 != 0 || hs < 1 || hs > 32) return DFS_EINVAL;
+    if (o.cold_cutoff % 2 != 0 || cs < 1 || cs > 64 || (cs & (cs - 1)) != 0) return DFS_EINVAL;
     if (o.victim_policy != 0 && o.victim_policy != 1) return DFS_EINVAL;
+    if (o.window == 0) o.window = (g->n > 0 && g->m >= 8 * g->n) ? 128 : 32;   // wide windows for dense lists
+    if (o.window != 32 && o.window != 128) return DFS_EINVAL;
     warps = o.warps_per_block <= 0 ? 32 : o.warps_per_block;
     if (warps > 32) return DFS_EINVAL;
     blocks = o.blocks <= 0 ? g->max_blocks : o.blocks;
@@ -359,6 +425,9 @@ static int run_many(dfs_graph* g, const int32_t* roots_host, int32_t k, int32_t*
         stats->steal_attempts = (int64_t)counters[kCntStealAttempts];
         stats->chunks_allocated = (int64_t)counters[kCntChunks];
         stats->windows = (int64_t)counters[kCntWindows];
+        stats->idle_ns = (int64_t)counters[kCntIdleNs];
+        stats->inter_scans = (int64_t)counters[kCntInterScans];
+        stats->spills = (int64_t)counters[kCntSpills];
     }
     return DFS_OK;
 }

@@ -27,7 +27,7 @@ STATUS = {0: "DFS_OK", -1: "DFS_EINVAL", -2: "DFS_ENOMEM", -3: "DFS_ECUDA", -4: 
 #: every symbol include/dfs.h declares (checked by tests/test_capi.py)
 EXPORTS = ["dfs_options_default", "dfs_graph_create", "dfs_run", "dfs_run_batch", "dfs_run_ex",
            "dfs_run_batch_ex", "dfs_set_stream", "dfs_graph_info", "dfs_launch_count",
-           "dfs_graph_destroy", "dfs_last_error", "dfs_strerror"]
+           "dfs_graph_destroy", "dfs_last_error", "dfs_strerror", "dfs_debug_timeline"]
 
 
 class DfsError(RuntimeError):
@@ -42,7 +42,11 @@ class _Options(ctypes.Structure):
                 ("deterministic", ctypes.c_int32), ("intra_steal", ctypes.c_int32),
                 ("inter_steal", ctypes.c_int32), ("victim_policy", ctypes.c_int32),
                 ("timeout_ms", ctypes.c_int32), ("seed", ctypes.c_uint32),
-                ("collect_stats", ctypes.c_int32), ("reserved", ctypes.c_int32 * 5)]
+                ("collect_stats", ctypes.c_int32), ("spill", ctypes.c_int32),
+                ("inter_any", ctypes.c_int32), ("spill_idle", ctypes.c_int32),
+                ("backoff_max_ns", ctypes.c_int32), ("window", ctypes.c_int32),
+                ("pub_batch", ctypes.c_int32), ("speculate", ctypes.c_int32),
+                ("reserved", ctypes.c_int32 * 4)]
 
 
 class _Stats(ctypes.Structure):
@@ -53,7 +57,8 @@ class _Stats(ctypes.Structure):
                 ("flushes", ctypes.c_int64), ("refills", ctypes.c_int64),
                 ("intra_steals", ctypes.c_int64), ("inter_steals", ctypes.c_int64),
                 ("steal_attempts", ctypes.c_int64), ("chunks_allocated", ctypes.c_int64),
-                ("windows", ctypes.c_int64)]
+                ("windows", ctypes.c_int64), ("idle_ns", ctypes.c_int64),
+                ("inter_scans", ctypes.c_int64), ("spills", ctypes.c_int64)]
 
 
 @dataclass
@@ -70,6 +75,13 @@ class Options:
     timeout_ms: Optional[int] = None
     seed: Optional[int] = None
     collect_stats: Optional[bool] = None
+    spill: Optional[bool] = None
+    inter_any: Optional[bool] = None
+    spill_idle: Optional[int] = None
+    backoff_max_ns: Optional[int] = None
+    window: Optional[int] = None
+    pub_batch: Optional[int] = None
+    speculate: Optional[bool] = None
 
     def to_c(self) -> _Options:
         o = _Options()
@@ -98,6 +110,9 @@ class Stats:
     steal_attempts: int
     chunks_allocated: int
     windows: int
+    idle_ns: int
+    inter_scans: int
+    spills: int
 
 
 _lib = None
@@ -134,6 +149,8 @@ def load_library():
         lib.dfs_graph_info.restype = ctypes.c_int
         lib.dfs_launch_count.argtypes = [P]
         lib.dfs_launch_count.restype = I64
+        lib.dfs_debug_timeline.argtypes = [P, ctypes.c_uint32, ctypes.c_uint32, P]
+        lib.dfs_debug_timeline.restype = ctypes.c_int
         lib.dfs_graph_destroy.argtypes = [P]
         lib.dfs_graph_destroy.restype = None
         lib.dfs_last_error.argtypes = []
@@ -254,6 +271,20 @@ class Graph:
         if stats:
             return out, Stats(**{f[0]: getattr(st, f[0]) for f in _Stats._fields_})
         return out
+
+    def timeline(self, len_: int = 0, dt_ns: int = 10_000, fetch: bool = False):
+        """Diagnostics (dfs_debug_timeline): enable with len_ > 0; fetch=True returns the last
+        run's busy-warp samples as a numpy array (-1 = no sample)."""
+        if not fetch:
+            rc = self._lib.dfs_debug_timeline(self._h, len_, dt_ns, None)
+            if rc != 0:
+                raise DfsError(rc, "dfs_debug_timeline")
+            return None
+        buf = np.zeros(len_, dtype=np.uint32)
+        rc = self._lib.dfs_debug_timeline(self._h, len_, dt_ns, buf.ctypes.data)
+        if rc != 0:
+            raise DfsError(rc, "dfs_debug_timeline")
+        return buf.astype(np.int64) - 1
 
     def launch_count(self) -> int:
         return int(self._lib.dfs_launch_count(self._h))

@@ -64,9 +64,10 @@ def test_deterministic_bit_exact(name, build, root):
     if root is None:
         root = int(graphgen.random_roots(g, 1, seed=1)[0])
     with Graph(g.row_ptr, g.col_idx) as G:
-        p = G.run(root, options=det())
-        torch.cuda.synchronize()
-        _exact(g, root, p)
+        for win in (32, 128):
+            p = G.run(root, options=Options(deterministic=True, window=win))
+            torch.cuda.synchronize()
+            _exact(g, root, p)
 
 
 # ------------------------------------------------------------------ unique trees: exact in parallel
@@ -113,13 +114,19 @@ def test_parallel_directed_with_self_loops_and_duplicates():
 # ------------------------------------------------------------------ stress
 @pytest.mark.parametrize("opts", [
     dict(hot_cutoff=4, cold_cutoff=4),
+    dict(hot_cutoff=2, cold_cutoff=2),
+    dict(hot_cutoff=6, cold_cutoff=2, spill_idle=1),
+    dict(hot_cutoff=2, cold_cutoff=2, warps_per_block=3, blocks=5, spill=False),
     dict(hot_cutoff=8, cold_cutoff=8, warps_per_block=4, blocks=8),
+    dict(inter_any=False, spill=False),
     dict(hot_cutoff=4, cold_cutoff=4, warps_per_block=2, blocks=64),
     dict(victim_policy=0),
     dict(intra_steal=False),
     dict(inter_steal=False),
     dict(blocks=1),
     dict(hot_cutoff=64, cold_cutoff=128),
+    dict(hot_cutoff=2, cold_cutoff=2, window=128),
+    dict(hot_cutoff=4, cold_cutoff=8, window=32),
 ])
 def test_stress_options(opts):
     graphs = [graphgen.road(300, 300, seed=3), graphgen.rmat(14, 8, seed=9),
@@ -185,7 +192,9 @@ def test_errors():
             G.run(100)
         assert e.value.code == -1
         with pytest.raises(DfsError):
-            G.run(0, options=Options(hot_cutoff=6))               # h_s must be even
+            G.run(0, options=Options(hot_cutoff=3))               # h_s = hot_cutoff/2 needs even cutoff
+        with pytest.raises(DfsError):
+            G.run(0, options=Options(cold_cutoff=6))              # c_s must be a power of two
         with pytest.raises(DfsError):
             G.run(0, options=Options(blocks=100000))
     bad = g.row_ptr.copy(); bad[5] = bad[4] - 1                   # non-monotone row_ptr
