@@ -79,10 +79,10 @@ enum dfs_victim_policy {
 typedef struct dfs_options {
     int32_t blocks;          /* persistent grid size; 0 = (#SMs x resident blocks per SM)          */
     int32_t warps_per_block; /* 1..32; 0 = 32                                                      */
-    int32_t hot_cutoff;      /* Alg 3 threshold: steal h_s = hot_cutoff/2 entries when a peer holds
-                                >= hot_cutoff (even, h_s <= 32); paper 32; default 2       */
-    int32_t cold_cutoff;     /* Alg 4 threshold: steal c_s = cold_cutoff/2 (a power of two <= 64);
-                                paper 64; default 2                                        */
+    int32_t hot_cutoff;      /* Alg 3 threshold: steal h_s = max(1, hot_cutoff/2) entries when a peer
+                                holds >= hot_cutoff (h_s <= 32); paper 32; default 1      */
+    int32_t cold_cutoff;     /* Alg 4 threshold: steal c_s = max(1, cold_cutoff/2) entries (<= 64)
+                                when a ColdSeg holds >= cold_cutoff; paper 64; default 1   */
     int32_t deterministic;   /* 1: one warp, no stealing: result == Alg 1 lexicographic tree       */
     int32_t intra_steal;     /* 1: enable Alg 3 (default)                                          */
     int32_t inter_steal;     /* 1: enable Alg 4 (default)                                          */
@@ -105,7 +105,10 @@ typedef struct dfs_options {
     int32_t speculate;       /* 1: claim a freshly descended child's first non-parent neighbour
                                 in parallel with the visited probes; 0: off; 2 (default): on for
                                 32-wide windows only                                               */
-    int32_t reserved[4];
+    int32_t steal_half;      /* 1 (default): a thief takes max(h_s, rest/2) <= 32 HotRing entries
+                                (resp. max(c_s, rest/2) <= 64 ColdSeg entries); 0: exactly h_s/c_s
+                                as in Alg 3/4                                                       */
+    int32_t reserved[3];
 } dfs_options;
 
 typedef struct dfs_stats {

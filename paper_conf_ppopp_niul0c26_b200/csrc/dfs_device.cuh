@@ -93,6 +93,7 @@ struct KParams {
     uint32_t seed;
     uint32_t pub_batch;                      // publish the HotRing head every pub_batch pushes
     int speculate;                           // speculative claim of the child's first neighbour
+    int steal_half;                          // steal max(h_s, rest/2) (resp. c_s) entries
 };
 
 // ------------------------------------------------------------------------------------------
@@ -259,8 +260,8 @@ __global__ void __launch_bounds__(32 * WMAX, 1) dfs_persistent_kernel(const KPar
     unsigned long long* const ring = rings + (size_t)w * H;
     const uint32_t tmask = (1u << P.tab_log2) - 1u;
     uint32_t* const my_tab = P.chunk_tab + ((size_t)gw << P.tab_log2);
-    const uint32_t hs = (uint32_t)P.hot_cutoff >> 1;        // h_s (Alg 3 l.12)
-    const uint32_t cs = (uint32_t)P.cold_cutoff >> 1;       // c_s (Alg 4 l.17)
+    const uint32_t hs = P.hot_cutoff >= 2 ? (uint32_t)P.hot_cutoff >> 1 : 1u;   // h_s (Alg 3 l.12)
+    const uint32_t cs = P.cold_cutoff >= 2 ? (uint32_t)P.cold_cutoff >> 1 : 1u; // c_s (Alg 4 l.17)
 
     if (threadIdx.x < kMaxWarps) {
         S.ht[threadIdx.x] = 0; S.tailf[threadIdx.x] = 0; S.lock[threadIdx.x] = 0;
@@ -722,15 +723,20 @@ __global__ void __launch_bounds__(32 * WMAX, 1) dfs_persistent_kernel(const KPar
                 if (best >= P.hot_cutoff) {
                     const int vwarp = __ffs(__ballot_sync(kFull, rest == best)) - 1;
                     if (STATS && lane == 0) ++cnt[kCntStealAttempts];
-                    uint32_t ok = 0, t = 0;
+                    uint32_t ok = 0, t = 0, kst = 0;
                     if (lane == 0) {
                         atomicAdd(&P.ctl->busy, 1u);                 // register before reserving
                         if (smem_trylock(&S.lock[vwarp])) {
                             uint32_t old = *(volatile uint32_t*)&S.ht[vwarp];
                             for (int tries = 0; tries < 8; ++tries) {
-                                if (ht_rest(old) < P.hot_cutoff) break;
+                                const int r = ht_rest(old);
+                                if (r < P.hot_cutoff) break;
                                 t = ht_tail(old);
-                                const uint32_t nw = (old & 0xFFFF0000u) | ((t + hs) & 0xFFFFu);
+                                kst = hs;
+                                if (P.steal_half && (uint32_t)(r / 2) > kst) kst = (uint32_t)(r / 2);
+                                if (kst > 32u) kst = 32u;
+                                if ((int)kst > r) kst = (uint32_t)r;
+                                const uint32_t nw = (old & 0xFFFF0000u) | ((t + kst) & 0xFFFFu);
                                 const uint32_t got = atom_cas_acquire_cta(&S.ht[vwarp], old, nw);   // reserve
                                 if (got == old) { ok = 1; break; }
                                 old = got;
@@ -742,18 +748,19 @@ __global__ void __launch_bounds__(32 * WMAX, 1) dfs_persistent_kernel(const KPar
                     ok = __shfl_sync(kFull, ok, 0);
                     if (ok) {
                         t = __shfl_sync(kFull, t, 0);
+                        kst = __shfl_sync(kFull, kst, 0);
                         __syncwarp();                                // lane 0's acquire -> all lanes
                         const unsigned long long* vring = rings + (size_t)vwarp * H;
-                        if (lane < (int)hs) ring[(my_head + lane) & (H - 1)] = vring[(t + lane) & (H - 1)];
+                        if (lane < (int)kst) ring[(my_head + lane) & (H - 1)] = vring[(t + lane) & (H - 1)];
                         __syncwarp();
                         if (lane == 0) {
-                            S.tailf[vwarp] = (t + hs) & 0xFFFFu;     // slots reusable by the owner
+                            S.tailf[vwarp] = (t + kst) & 0xFFFFu;    // slots reusable by the owner
                             smem_unlock(&S.lock[vwarp]);
-                            atom_add_release_cta(&S.ht[w], hs << 16); // publish into our ring
+                            atom_add_release_cta(&S.ht[w], kst << 16); // publish into our ring
                             atomicOr(&S.warp_mask, 1u << w);         // mark active
                         }
                         __syncwarp();
-                        my_head += hs; pub = my_head;
+                        my_head += kst; pub = my_head;
                         if (STATS && lane == 0) ++cnt[kCntIntraSteals];
                         got_work = true;
                         break;
@@ -817,14 +824,19 @@ __global__ void __launch_bounds__(32 * WMAX, 1) dfs_persistent_kernel(const KPar
                         const int vwl = __ffs(__ballot_sync(kFull, rest == best)) - 1;
                         const int vwg = vb * WV + vwl;
                         if (STATS && lane == 0) ++cnt[kCntStealAttempts];
-                        uint32_t ok = 0, bot = 0;
+                        uint32_t ok = 0, bot = 0, kst = 0;
                         if (lane == 0) {
                             atomicAdd(&P.ctl->busy, 1u);
                             unsigned long long old = ld_relaxed_u64(&P.cold_tb[vwg]);
                             for (int tries = 0; tries < 4; ++tries) {
                                 const uint32_t top = (uint32_t)(old >> 32), b = (uint32_t)old;
-                                if ((int)(top - b) < P.cold_cutoff) break;
-                                const unsigned long long nw = ((unsigned long long)top << 32) | (uint32_t)(b + cs);
+                                const int r = (int)(top - b);
+                                if (r < P.cold_cutoff) break;
+                                kst = cs;
+                                if (P.steal_half && (uint32_t)(r / 2) > kst) kst = (uint32_t)(r / 2);
+                                if (kst > 64u) kst = 64u;
+                                if ((int)kst > r) kst = (uint32_t)r;
+                                const unsigned long long nw = ((unsigned long long)top << 32) | (uint32_t)(b + kst);
                                 const unsigned long long got = atomicCAS(&P.cold_tb[vwg], old, nw);   // reserve
                                 if (got == old) { ok = 1; bot = b; break; }
                                 old = got;
@@ -834,26 +846,38 @@ __global__ void __launch_bounds__(32 * WMAX, 1) dfs_persistent_kernel(const KPar
                         ok = __shfl_sync(kFull, ok, 0);
                         if (ok) {
                             bot = __shfl_sync(kFull, bot, 0);
-                            // remote transfer (Alg 4 l.21-22): L2 loads, addresses from the CAS
+                            kst = __shfl_sync(kFull, kst, 0);
+                            // remote transfer (Alg 4 l.21-22): L2 loads, addresses from the CAS;
+                            // the range [bot, bot+kst) may straddle two ColdSeg chunks
                             uint32_t* vtab = P.chunk_tab + ((size_t)vwg << P.tab_log2);
-                            uint32_t* slot = &vtab[(bot >> kChunkLog2) & tmask];
-                            const uint32_t c = ld_relaxed_u32(slot);
-                            const unsigned long long* src = P.pool + ((size_t)c << kChunkLog2) + (bot & (kChunk - 1));
-                            for (uint32_t q = lane; q < cs; q += 32u)
-                                ring[(my_head + q) & (H - 1)] = ld_cg_u64(src + q);
+                            for (uint32_t q = lane; q < kst; q += 32u) {
+                                const uint32_t p = bot + q;
+                                const uint32_t c = ld_relaxed_u32(&vtab[(p >> kChunkLog2) & tmask]);
+                                ring[(my_head + q) & (H - 1)] = ld_cg_u64(P.pool + ((size_t)c << kChunkLog2) + (p & (kChunk - 1)));
+                            }
                             __syncwarp();
                             if (lane == 0) {
-                                const uint32_t before = atomicAdd(&P.chunk_consumed[c], cs);
-                                if (before + cs == kChunk) {                   // chunk fully consumed
-                                    st_relaxed_u32(slot, kEmptySlot);
-                                    pool_free(P, c);
+                                // chunk accounting: every position below bottom is passed by
+                                // exactly one steal; the thief completing a chunk frees it
+                                uint32_t p = bot, left = kst;
+                                while (left) {
+                                    const uint32_t in_chunk = kChunk - (p & (kChunk - 1));
+                                    const uint32_t part = left < in_chunk ? left : in_chunk;
+                                    uint32_t* slot = &vtab[(p >> kChunkLog2) & tmask];
+                                    const uint32_t c = ld_relaxed_u32(slot);
+                                    const uint32_t before = atomicAdd(&P.chunk_consumed[c], part);
+                                    if (before + part == kChunk) {             // chunk fully consumed
+                                        st_relaxed_u32(slot, kEmptySlot);
+                                        pool_free(P, c);
+                                    }
+                                    p += part; left -= part;
                                 }
-                                atomicSub(&P.block_cold[vb], (int)cs);
-                                atom_add_release_cta(&S.ht[w], cs << 16);      // publish into our ring
+                                atomicSub(&P.block_cold[vb], (int)kst);
+                                atom_add_release_cta(&S.ht[w], kst << 16);     // publish into our ring
                                 atomicOr(&S.warp_mask, 1u << w);               // mark w, b active
                             }
                             __syncwarp();
-                            my_head += cs; pub = my_head;
+                            my_head += kst; pub = my_head;
                             if (STATS && lane == 0) ++cnt[kCntInterSteals];
                             if (lane == 0) smem_unlock(&S.inter_token);
                             got_work = true;

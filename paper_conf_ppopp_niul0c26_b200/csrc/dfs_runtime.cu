@@ -100,8 +100,8 @@ void dfs_options_default(dfs_options* o) {
     std::memset(o, 0, sizeof(*o));
     o->blocks = 0;
     o->warps_per_block = 32;
-    o->hot_cutoff = 2;           // paper: 32; B200 sweep: 2
-    o->cold_cutoff = 2;          // paper: 64; B200 sweep: 2
+    o->hot_cutoff = 1;           // paper: 32; B200 sweep: 1
+    o->cold_cutoff = 1;          // paper: 64; B200 sweep: 1
     o->deterministic = 0;
     o->intra_steal = 1;
     o->inter_steal = 1;
@@ -116,6 +116,7 @@ void dfs_options_default(dfs_options* o) {
     o->window = 0;
     o->pub_batch = 1;
     o->speculate = 2;
+    o->steal_half = 1;
 }
 
 int dfs_last_error(void) { return g_last_error; }
@@ -305,6 +306,7 @@ static int launch_one(dfs_graph* g, int32_t root, int32_t* d_out, const dfs_opti
     P.backoff_max_ns = o.backoff_max_ns > 0 ? (unsigned)o.backoff_max_ns : 2048u;
     P.pub_batch = o.pub_batch > 0 ? (uint32_t)o.pub_batch : 4u;
     P.speculate = o.speculate;
+    P.steal_half = o.steal_half;
     P.timeline = g->d_timeline;
     P.timeline_len = g->timeline_len;
     P.timeline_dt_ns = g->timeline_dt_ns;
@@ -327,14 +329,13 @@ static int launch_one(dfs_graph* g, int32_t root, int32_t* d_out, const dfs_opti
 static int resolve_options(const dfs_graph* g, const dfs_options* in, dfs_options& o, int& blocks, int& warps) {
     dfs_options_default(&o);
     if (in) o = *in;
-    if (o.hot_cutoff == 0) o.hot_cutoff = 2;
-    if (o.cold_cutoff == 0) o.cold_cutoff = 2;
+    if (o.hot_cutoff == 0) o.hot_cutoff = 1;
+    if (o.cold_cutoff == 0) o.cold_cutoff = 1;
     if (o.timeout_ms <= 0) o.timeout_ms = 120000;
-    // h_s = hot_cutoff/2 in [1, 32] (one lane per entry); c_s = cold_cutoff/2 a power of two
-    // <= 64 (dividing the ColdSeg chunk, so a steal never straddles chunks)
-    const int hs = o.hot_cutoff / 2, cs = o.cold_cutoff / 2;
-    if (o.hot_cutoff % 2 != 0 || hs < 1 || hs > 32) return DFS_EINVAL;
-    if (o.cold_cutoff % 2 != 0 || cs < 1 || cs > 64 || (cs & (cs - 1)) != 0) return DFS_EINVAL;
+    // thresholds >= 1; h_s = max(1, hot_cutoff/2) <= 32 (one lane per entry);
+    // c_s = max(1, cold_cutoff/2) <= 64
+    if (o.hot_cutoff < 1 || o.hot_cutoff / 2 > 32) return DFS_EINVAL;
+    if (o.cold_cutoff < 1 || o.cold_cutoff / 2 > 64) return DFS_EINVAL;
     if (o.victim_policy != 0 && o.victim_policy != 1) return DFS_EINVAL;
     if (o.window == 0) o.window = (g->n > 0 && g->m >= 8 * g->n) ? 128 : 32;   // wide windows for dense lists
     if (o.window != 32 && o.window != 128) return DFS_EINVAL;

@@ -46,7 +46,7 @@ class _Options(ctypes.Structure):
                 ("inter_any", ctypes.c_int32), ("spill_idle", ctypes.c_int32),
                 ("backoff_max_ns", ctypes.c_int32), ("window", ctypes.c_int32),
                 ("pub_batch", ctypes.c_int32), ("speculate", ctypes.c_int32),
-                ("reserved", ctypes.c_int32 * 4)]
+                ("steal_half", ctypes.c_int32), ("reserved", ctypes.c_int32 * 3)]
 
 
 class _Stats(ctypes.Structure):
@@ -81,7 +81,8 @@ class Options:
     backoff_max_ns: Optional[int] = None
     window: Optional[int] = None
     pub_batch: Optional[int] = None
-    speculate: Optional[bool] = None
+    speculate: Optional[int] = None
+    steal_half: Optional[bool] = None
 
     def to_c(self) -> _Options:
         o = _Options()

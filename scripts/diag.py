@@ -85,6 +85,11 @@ VARIANTS = {
     "paperdef": dict(hot_cutoff=32, cold_cutoff=64, spill=False, inter_any=False, pub_batch=1, speculate=False),
     "spec1": dict(speculate=1),
     "spec0": dict(speculate=0),
+    "nohalf": dict(steal_half=False),
+    "h1c1": dict(hot_cutoff=1, cold_cutoff=1),
+    "h1c2": dict(hot_cutoff=1, cold_cutoff=2),
+    "h4c4": dict(hot_cutoff=4, cold_cutoff=4),
+    "h1c1nohalf": dict(hot_cutoff=1, cold_cutoff=1, steal_half=False),
 }
 
 

@@ -73,7 +73,7 @@ def test_null_handle_is_einval(lib):
 def test_options_default(lib):
     o = dfs._Options()
     lib.dfs_options_default(ctypes.byref(o))
-    assert (o.hot_cutoff, o.cold_cutoff, o.warps_per_block) == (2, 2, 32)     # B200 sweep
+    assert (o.hot_cutoff, o.cold_cutoff, o.warps_per_block) == (1, 1, 32)     # B200 sweep
     assert o.victim_policy == 1 and o.intra_steal == 1 and o.inter_steal == 1
 
 

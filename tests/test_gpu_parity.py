@@ -127,6 +127,10 @@ def test_parallel_directed_with_self_loops_and_duplicates():
     dict(hot_cutoff=64, cold_cutoff=128),
     dict(hot_cutoff=2, cold_cutoff=2, window=128),
     dict(hot_cutoff=4, cold_cutoff=8, window=32),
+    dict(hot_cutoff=1, cold_cutoff=1),
+    dict(hot_cutoff=3, cold_cutoff=5, steal_half=False),
+    dict(hot_cutoff=1, cold_cutoff=1, warps_per_block=2, blocks=3, spill_idle=1, pub_batch=3),
+    dict(speculate=1, window=128, steal_half=False),
 ])
 def test_stress_options(opts):
     graphs = [graphgen.road(300, 300, seed=3), graphgen.rmat(14, 8, seed=9),
@@ -192,9 +196,11 @@ def test_errors():
             G.run(100)
         assert e.value.code == -1
         with pytest.raises(DfsError):
-            G.run(0, options=Options(hot_cutoff=3))               # h_s = hot_cutoff/2 needs even cutoff
+            G.run(0, options=Options(hot_cutoff=66))              # h_s > 32 lanes
         with pytest.raises(DfsError):
-            G.run(0, options=Options(cold_cutoff=6))              # c_s must be a power of two
+            G.run(0, options=Options(cold_cutoff=130))            # c_s > 64
+        with pytest.raises(DfsError):
+            G.run(0, options=Options(window=64))
         with pytest.raises(DfsError):
             G.run(0, options=Options(blocks=100000))
     bad = g.row_ptr.copy(); bad[5] = bad[4] - 1                   # non-monotone row_ptr
