@@ -108,7 +108,10 @@ typedef struct dfs_options {
     int32_t steal_half;      /* 1 (default): a thief takes max(h_s, rest/2) <= 32 HotRing entries
                                 (resp. max(c_s, rest/2) <= 64 ColdSeg entries); 0: exactly h_s/c_s
                                 as in Alg 3/4                                                       */
-    int32_t reserved[3];
+    int32_t probe_mode;      /* visited probes: 0 = L2 (ld.global.cg, default), 1 = L1-cached,
+                                2 = ld.relaxed.gpu.  A stale probe can only say "unvisited" for a
+                                claimed vertex; the atomic claim decides, so all are exact         */
+    int32_t reserved[2];
 } dfs_options;
 
 typedef struct dfs_stats {
@@ -123,6 +126,9 @@ typedef struct dfs_stats {
     int64_t idle_ns;         /* sum over warps of time spent idle (stealing / waiting)             */
     int64_t inter_scans;     /* inter-block victim-selection rounds                                */
     int64_t spills;          /* demand-driven spills                                               */
+    /* SM-cycle breakdown of the expansion step summed over windows (collect_stats; diagnostics):
+       wait for the window data, wait for the probes, wait for the speculative claim, rest */
+    int64_t cyc_window, cyc_probe, cyc_claim, cyc_tail;
 } dfs_stats;
 
 void dfs_options_default(dfs_options *opt);

@@ -60,12 +60,13 @@ struct Ctl {
 
 enum CounterIdx {
     kCntClaims = 0, kCntFailedClaims, kCntFlushes, kCntRefills, kCntIntraSteals, kCntInterSteals,
-    kCntStealAttempts, kCntChunks, kCntWindows, kCntIdleNs, kCntInterScans, kCntSpills, kNumCounters
+    kCntStealAttempts, kCntChunks, kCntWindows, kCntIdleNs, kCntInterScans, kCntSpills,
+    kCntTWin, kCntTProbe, kCntTClaim, kCntTTail, kNumCounters
 };
 
 struct KParams {
     const uint32_t* __restrict__ rp;         // n+1 (narrowed row_ptr; m < 2^32)
-    const int32_t* __restrict__ col;         // m (+8 padding)
+    const uint2* __restrict__ adj;           // m (+8 padding): {neighbour v, row_ptr[v]} per CSR entry
     uint32_t* bitmap;                        // ceil(n/32) visited words
     int32_t* parent;                         // n output
     unsigned long long* cold_tb;             // n_warps: (top << 32) | bottom
@@ -94,6 +95,7 @@ struct KParams {
     uint32_t pub_batch;                      // publish the HotRing head every pub_batch pushes
     int speculate;                           // speculative claim of the child's first neighbour
     int steal_half;                          // steal max(h_s, rest/2) (resp. c_s) entries
+    int probe_mode;                          // 0: L2 (.cg) probes; 1: L1-cached probes; 2: .relaxed.gpu
 };
 
 // ------------------------------------------------------------------------------------------
@@ -116,6 +118,12 @@ __device__ __forceinline__ int ld_relaxed_s32(const int* p) {
 }
 __device__ __forceinline__ void st_relaxed_u32(uint32_t* p, uint32_t v) {
     asm volatile("st.relaxed.gpu.global.u32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
+}
+// SM clock read that waits for `dep` to be ready (scoreboard dependency on the asm input)
+__device__ __forceinline__ long long clock_after(uint32_t dep) {
+    long long t;
+    asm volatile("mov.u64 %0, %%clock64;" : "=l"(t) : "r"(dep) : "memory");
+    return t;
 }
 __device__ __forceinline__ unsigned long long globaltimer() {
     unsigned long long t;
@@ -186,6 +194,7 @@ struct SmemCtl {
     volatile int done;                     // block-local copy of ctl->done
     uint32_t inter_token;                  // one idle warp per block scans other blocks at a time
     unsigned long long cnt[kMaxWarps][16]; // per-warp stats counters (collect_stats)
+    static_assert(kNumCounters <= 16, "counter slots");
 };
 
 __device__ __forceinline__ void smem_lock(uint32_t* l) {
@@ -247,7 +256,6 @@ __global__ void __launch_bounds__(32 * WMAX, 1) dfs_persistent_kernel(const KPar
     static_assert(VEC == 1 || VEC == 4, "VEC is 1 or 4");
     constexpr uint32_t kBatch = H / 2;              // flush batch (reading S10)
     constexpr uint32_t kWin = 32u * VEC;            // positions per window
-    constexpr int kPfLanes = 8 / VEC;               // lanes covering the first 8 positions
     extern __shared__ __align__(16) unsigned char smem_raw[];
     SmemCtl& S = *reinterpret_cast<SmemCtl*>(smem_raw);
     constexpr int kCtlBytes = (sizeof(SmemCtl) + 15) & ~15;
@@ -276,9 +284,10 @@ __global__ void __launch_bounds__(32 * WMAX, 1) dfs_persistent_kernel(const KPar
     bool have_win = false;       // nbv holds the window starting at i
     bool need_end = false;       // end must be re-read from row_ptr
     uint32_t u = 0, i = 0, end = 0;
-    int nbv[VEC];                // this lane's neighbours in the current window
+    int nbv[VEC];                // this lane's neighbours in the current window ...
+    uint32_t rsv[VEC];           // ... and their row_ptr values (edge-annotated adjacency)
 #pragma unroll
-    for (int e = 0; e < VEC; ++e) nbv[e] = -1;
+    for (int e = 0; e < VEC; ++e) { nbv[e] = -1; rsv[e] = 0; }
     uint32_t my_head = 0;        // owner's true HotRing head (16-bit wrap)
     uint32_t pub = 0;            // head value published in S.ht (entries in [pub, my_head) are
                                  // private: pushed/popped without synchronisation)
@@ -299,15 +308,23 @@ __global__ void __launch_bounds__(32 * WMAX, 1) dfs_persistent_kernel(const KPar
         u = (uint32_t)P.root; i = __ldg(P.rp + u); end = __ldg(P.rp + u + 1);
     }
 
-    // window loader: lane holds positions base + VEC*lane + e, e < VEC
-    auto load_window = [&](uint32_t base, uint32_t limit, int* out) {
+    // window loader: lane holds positions base + VEC*lane + e, e < VEC.  Each entry is
+    // {v, row_ptr[v]}, so the child's window address is known as soon as its id is: one
+    // dependent load per DFS level instead of two (col_idx then row_ptr).
+    auto load_window = [&](uint32_t base, int* nb, uint32_t* rs) {
         const uint32_t q = base + (uint32_t)VEC * lane;
         if constexpr (VEC == 4) {
-            int4 x = make_int4(-1, -1, -1, -1);
-            if (q < limit) x = __ldg(reinterpret_cast<const int4*>(P.col + q));   // col padded
-            out[0] = x.x; out[1] = x.y; out[2] = x.z; out[3] = x.w;
+            uint4 x0 = make_uint4(kFull, 0u, kFull, 0u), x1 = x0;
+            if (q < P.m) {                                                   // adj padded
+                x0 = __ldg(reinterpret_cast<const uint4*>(P.adj + q));
+                x1 = __ldg(reinterpret_cast<const uint4*>(P.adj + q + 2));
+            }
+            nb[0] = (int)x0.x; rs[0] = x0.y; nb[1] = (int)x0.z; rs[1] = x0.w;
+            nb[2] = (int)x1.x; rs[2] = x1.y; nb[3] = (int)x1.z; rs[3] = x1.w;
         } else {
-            out[0] = (q < limit) ? __ldg(P.col + q) : -1;
+            uint2 x = make_uint2(kFull, 0u);
+            if (q < P.m) x = __ldg(P.adj + q);
+            nb[0] = (int)x.x; rs[0] = x.y;
         }
     };
 
@@ -506,22 +523,27 @@ __global__ void __launch_bounds__(32 * WMAX, 1) dfs_persistent_kernel(const KPar
             // holds positions a+VEC*k .. a+VEC*k+VEC-1.  Positions outside [i, end) are masked.
             if (!have_win) {
                 const uint32_t e2 = need_end ? __ldg(P.rp + u + 1) : end;
-                load_window(i & ~(uint32_t)(VEC - 1), P.m, nbv);
+                load_window(i & ~(uint32_t)(VEC - 1), nbv, rsv);
                 end = e2; need_end = false;
             }
             if (STATS && lane == 0) ++cnt[kCntWindows];
+            long long tc0 = 0, tc1 = 0;
+            if (STATS) { tc0 = clock_after(0u); tc1 = clock_after((uint32_t)nbv[0] ^ end); }
             const uint32_t a = i & ~(uint32_t)(VEC - 1);
             const uint32_t q0 = a + (uint32_t)VEC * lane;
             // long list (hubs): load the next window now so it is in flight while this window's
             // probes resolve (a sequential scan then costs one probe round trip per window)
             int nxt[VEC];
+            uint32_t nxr[VEC];
             const bool have_nxt = a + kWin < end;
-            if (have_nxt) load_window(a + kWin, P.m, nxt);
+            if (have_nxt) load_window(a + kWin, nxt, nxr);
             // speculative claim (fresh child only): the first position whose neighbour is not the
-            // parent we came from is, if unvisited, exactly Alg 1's next tree edge; claiming it
-            // in parallel with the probes removes the probe -> claim round trip
+            // parent we came from is, if unvisited, exactly Alg 1's next tree edge.  Its claim,
+            // its end offset and its first window are all issued in parallel with the probes.
             int sk = -1, se = 0;
             uint32_t sv = 0, s_old = 0, s_rs = 0, s_re = 0;
+            int cnb[VEC];
+            uint32_t cnr[VEC];
             if ((P.speculate == 1 || (P.speculate == 2 && VEC == 1)) && spec_ok) {
                 uint32_t vm = 0;
 #pragma unroll
@@ -534,55 +556,68 @@ __global__ void __launch_bounds__(32 * WMAX, 1) dfs_persistent_kernel(const KPar
                     sk = __ffs(vb) - 1;
                     se = __ffs(__shfl_sync(kFull, vm, sk)) - 1;
                     int pick = nbv[0];
+                    uint32_t pick_rs = rsv[0];
 #pragma unroll
-                    for (int f = 1; f < VEC; ++f) if (se == f) pick = nbv[f];
+                    for (int f = 1; f < VEC; ++f) if (se == f) { pick = nbv[f]; pick_rs = rsv[f]; }
                     sv = (uint32_t)__shfl_sync(kFull, pick, sk);
+                    s_rs = __shfl_sync(kFull, pick_rs, sk);
                     if (lane == 0) s_old = atomicOr(P.bitmap + (sv >> 5), 1u << (sv & 31));
-                    s_rs = __ldg(P.rp + sv); s_re = __ldg(P.rp + sv + 1);
+                    s_re = __ldg(P.rp + sv + 1);
+                    load_window(s_rs & ~(uint32_t)(VEC - 1), cnb, cnr);
                 }
             }
-            // probe visited bits; the lanes holding the first 8 positions also prefetch their
-            // candidates' row_ptr pairs so a claim can load the child's window immediately
+            // probe the visited bits of every position in the window
             uint32_t m4 = 0;
-            uint32_t prs[VEC], pre[VEC];
 #pragma unroll
             for (int e = 0; e < VEC; ++e) {
                 const uint32_t p = q0 + e;
                 const int x = nbv[e];
-                prs[e] = 0; pre[e] = 0;
                 if (p >= i && p < end) {
-                    const uint32_t word = __ldcg(P.bitmap + ((uint32_t)x >> 5));
-                    if (lane < kPfLanes) { prs[e] = __ldg(P.rp + x); pre[e] = __ldg(P.rp + x + 1); }
+                    // a probe that reads "visited" is always right (bits are only ever set), so a
+                    // possibly-stale cached copy is a valid filter: the atomic claim decides
+                    const uint32_t* wp = P.bitmap + ((uint32_t)x >> 5);
+                    const uint32_t word = P.probe_mode == 1 ? *wp
+                                        : P.probe_mode == 2 ? ld_relaxed_u32(wp) : __ldcg(wp);
                     if (!((word >> (x & 31)) & 1u)) m4 |= 1u << e;
                 }
             }
             bool descended = false;
+            long long tc2 = 0;
+            if (STATS) tc2 = clock_after(m4);
+            // descend into child v found at window slot (k, e): push <u, next candidate> (Alg 1
+            // l.8 + l.11) unless u is exhausted, then make v the register top.  Positions after
+            // (k, e) whose probe saw a claimed target stay claimed (claims are monotone), so
+            // scanning them again cannot change anything: resume at the next still-unvisited
+            // candidate, or past the window.
+            auto descend = [&](int k, int e, uint32_t v, uint32_t vrs, uint32_t vre) -> bool {
+                if (STATS && lane == 0) ++cnt[kCntClaims];
+                if (lane == 0) P.parent[v] = (int32_t)u;                            // Alg 1 l.10
+                const uint32_t mine = (lane == k) ? (m4 & ~((2u << e) - 1u)) : (lane > k ? m4 : 0u);
+                const uint32_t later = __ballot_sync(kFull, mine != 0);
+                uint32_t ni = a + kWin;
+                if (later) {
+                    const int k2 = __ffs(later) - 1;
+                    const uint32_t m2 = __shfl_sync(kFull, mine, k2);
+                    ni = a + (uint32_t)VEC * (uint32_t)k2 + (uint32_t)(__ffs(m2) - 1);
+                }
+                if (ni < end) {
+                    if (!push(u, ni)) return false;
+                }
+                par = u;
+                u = v; i = vrs; end = vre; have_win = true; need_end = false; spec_ok = true;
+#pragma unroll
+                for (int f = 0; f < VEC; ++f) { nbv[f] = cnb[f]; rsv[f] = cnr[f]; }
+                descended = true;
+                return true;
+            };
+            long long tc3 = tc2;
             if (sk >= 0) {
                 if (lane == sk) m4 &= ~(1u << se);               // p0 is claimed either way
                 s_old = __shfl_sync(kFull, s_old, 0);
-                if (!(s_old & (1u << (sv & 31)))) {
-                    // speculative claim won: <u, next candidate> below, child on top
-                    int cnb[VEC];
-                    load_window(s_rs & ~(uint32_t)(VEC - 1), s_re, cnb);
-                    if (STATS && lane == 0) ++cnt[kCntClaims];
-                    if (lane == 0) P.parent[sv] = (int32_t)u;                       // Alg 1 l.10
-                    const uint32_t mine = (lane == sk) ? (m4 & ~((2u << se) - 1u)) : (lane > sk ? m4 : 0u);
-                    const uint32_t later = __ballot_sync(kFull, mine != 0);
-                    uint32_t ni = a + kWin;
-                    if (later) {
-                        const int k2 = __ffs(later) - 1;
-                        const uint32_t m2 = __shfl_sync(kFull, mine, k2);
-                        ni = a + (uint32_t)VEC * (uint32_t)k2 + (uint32_t)(__ffs(m2) - 1);
-                    }
-                    if (ni < end) {
-                        if (!push(u, ni)) goto exit_loop;
-                    }
-                    par = u;
-                    u = sv; i = s_rs; end = s_re; have_win = true; need_end = false; spec_ok = true;
-#pragma unroll
-                    for (int f = 0; f < VEC; ++f) nbv[f] = cnb[f];
-                    descended = true;
-                } else if (lane == 0) {
+                if (STATS) tc3 = clock_after(s_old);
+                if (!(s_old & (1u << (sv & 31)))) {              // speculative claim won
+                    if (!descend(sk, se, sv, s_rs, s_re)) goto exit_loop;
+                } else if (STATS && lane == 0) {
                     ++cnt[kCntFailedClaims];
                 }
             }
@@ -592,59 +627,38 @@ __global__ void __launch_bounds__(32 * WMAX, 1) dfs_persistent_kernel(const KPar
                 const uint32_t mk = __shfl_sync(kFull, m4, k);
                 const int e = __ffs(mk) - 1;                       // first candidate in CSR order
                 int mine_nb = nbv[0];
-                uint32_t mine_rs = prs[0], mine_re = pre[0];
+                uint32_t mine_rs = rsv[0];
 #pragma unroll
                 for (int f = 1; f < VEC; ++f)
-                    if (e == f) { mine_nb = nbv[f]; mine_rs = prs[f]; mine_re = pre[f]; }
+                    if (e == f) { mine_nb = nbv[f]; mine_rs = rsv[f]; }
                 const uint32_t v = (uint32_t)__shfl_sync(kFull, mine_nb, k);
-                uint32_t vrs, vre;
-                if (k < kPfLanes) {
-                    vrs = __shfl_sync(kFull, mine_rs, k); vre = __shfl_sync(kFull, mine_re, k);
-                } else {
-                    vrs = __ldg(P.rp + v); vre = __ldg(P.rp + v + 1);
-                }
+                const uint32_t vrs = __shfl_sync(kFull, mine_rs, k);
                 const uint32_t bit = 1u << (v & 31);
                 uint32_t old = 0;
                 if (lane == 0) old = atomicOr(P.bitmap + (v >> 5), bit);          // claim
-                // speculative load of the child's first window, overlapping the claim
-                int cnb[VEC];
-                load_window(vrs & ~(uint32_t)(VEC - 1), vre, cnb);
+                // the child's end offset and first window load overlap the claim
+                const uint32_t vre = __ldg(P.rp + v + 1);
+                load_window(vrs & ~(uint32_t)(VEC - 1), cnb, cnr);
                 old = __shfl_sync(kFull, old, 0);
                 if (!(old & bit)) {
-                    if (STATS && lane == 0) ++cnt[kCntClaims];
-                    if (lane == 0) P.parent[v] = (int32_t)u;                        // Alg 1 l.10
-                    // Alg 1 l.8 + l.11: keep <u, ni> below the child unless u is exhausted.
-                    // Positions after the claimed one whose probe saw a claimed target stay
-                    // claimed (claims are monotone), so scanning them again cannot change
-                    // anything: resume at the next still-unvisited candidate, or past the window.
-                    const uint32_t mine = (lane == k) ? (m4 & ~((2u << e) - 1u)) : (lane > k ? m4 : 0u);
-                    const uint32_t later = __ballot_sync(kFull, mine != 0);
-                    uint32_t ni = a + kWin;
-                    if (later) {
-                        const int k2 = __ffs(later) - 1;
-                        const uint32_t m2 = __shfl_sync(kFull, mine, k2);
-                        ni = a + (uint32_t)VEC * (uint32_t)k2 + (uint32_t)(__ffs(m2) - 1);
-                    }
-                    if (ni < end) {
-                        if (!push(u, ni)) goto exit_loop;
-                    }
-                    par = u;
-                    u = v; i = vrs; end = vre; have_win = true; need_end = false; spec_ok = true;
-#pragma unroll
-                    for (int f = 0; f < VEC; ++f) nbv[f] = cnb[f];
-                    descended = true;
+                    if (!descend(k, e, v, vrs, vre)) goto exit_loop;
                     break;
                 }
                 if (STATS && lane == 0) ++cnt[kCntFailedClaims];
                 if (lane == k) m4 &= ~(1u << e);                  // lost the race: next candidate
                 any = __ballot_sync(kFull, m4 != 0);
             }
+            if (STATS && lane == 0) {
+                const long long tc4 = clock_after((uint32_t)nbv[0] ^ i);
+                cnt[kCntTWin] += tc1 - tc0; cnt[kCntTProbe] += tc2 - tc1;
+                cnt[kCntTClaim] += tc3 - tc2; cnt[kCntTTail] += tc4 - tc3;
+            }
             if (!descended) {
                 i = a + kWin;
                 spec_ok = false;
                 if (have_nxt) {                                   // next window already loaded
 #pragma unroll
-                    for (int f = 0; f < VEC; ++f) nbv[f] = nxt[f];
+                    for (int f = 0; f < VEC; ++f) { nbv[f] = nxt[f]; rsv[f] = nxr[f]; }
                     have_win = true;
                 } else {
                     have_win = false;                             // i >= end: Alg 1 l.14: pop
@@ -982,6 +996,16 @@ __global__ void dfs_validate_rowptr_kernel(const int64_t* __restrict__ rp64, uin
         if (v < (size_t)n) ok = ok && rp64[v + 1] >= a;
         if (!ok) atomicExch(bad, 1);
         rp32[v] = (uint32_t)a;
+    }
+}
+
+// edge-annotated adjacency: adj[j] = {col_idx[j], row_ptr[col_idx[j]]} (step a1)
+__global__ void dfs_build_adj_kernel(const int32_t* __restrict__ col, const uint32_t* __restrict__ rp,
+                                     uint2* adj, int64_t m) {
+    const size_t stride = (size_t)gridDim.x * blockDim.x;
+    for (size_t j = blockIdx.x * (size_t)blockDim.x + threadIdx.x; j < (size_t)m; j += stride) {
+        const int32_t c = col[j];
+        adj[j] = make_uint2((uint32_t)c, __ldg(rp + c));
     }
 }
 

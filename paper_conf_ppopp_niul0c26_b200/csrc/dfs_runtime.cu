@@ -55,7 +55,7 @@ struct dfs_graph {
     int sms = 0;
     int max_blocks = 0;          // co-resident 32-warp blocks (allocation bound)
     uint32_t* d_rp = nullptr;
-    int32_t* d_col = nullptr;
+    uint2* d_adj = nullptr;      // {col_idx[j], row_ptr[col_idx[j]]} per CSR entry (+8 padding)
     uint32_t* d_bitmap = nullptr;
     int32_t* d_parent = nullptr; // lazily allocated for host outputs
     unsigned long long* d_cold_tb = nullptr;
@@ -81,7 +81,7 @@ static void free_graph(dfs_graph* g) {
     int cur = 0;
     cudaGetDevice(&cur);
     cudaSetDevice(g->device);
-    cudaFree(g->d_rp); cudaFree(g->d_col); cudaFree(g->d_bitmap); cudaFree(g->d_parent);
+    cudaFree(g->d_rp); cudaFree(g->d_adj); cudaFree(g->d_bitmap); cudaFree(g->d_parent);
     cudaFree(g->d_cold_tb); cudaFree(g->d_tab); cudaFree(g->d_pool); cudaFree(g->d_consumed);
     cudaFree(g->d_next); cudaFree(g->d_block_cold); cudaFree(g->d_ctl); cudaFree(g->d_count2);
     cudaFree(g->d_timeline);
@@ -117,6 +117,7 @@ void dfs_options_default(dfs_options* o) {
     o->pub_batch = 1;
     o->speculate = 2;
     o->steal_half = 1;
+    o->probe_mode = 0;
 }
 
 int dfs_last_error(void) { return g_last_error; }
@@ -175,7 +176,7 @@ dfs_graph* dfs_graph_create(const int64_t* row_ptr, const int32_t* col_idx, int6
     bool ok = true;
     auto A = [&](void** p, size_t bytes) { if (ok && cudaMalloc(p, bytes ? bytes : 16) != cudaSuccess) ok = false; };
     A((void**)&g->d_rp, (size_t)(n + 1) * sizeof(uint32_t));
-    A((void**)&g->d_col, (size_t)(m + 8) * sizeof(int32_t));     // padded for 128-bit window loads
+    A((void**)&g->d_adj, (size_t)(m + 8) * sizeof(uint2));       // padded for 128-bit window loads
     A((void**)&g->d_bitmap, nwords * sizeof(uint32_t));
     A((void**)&g->d_cold_tb, (size_t)n_warps * sizeof(unsigned long long));
     A((void**)&g->d_tab, g->tab_words * sizeof(uint32_t));
@@ -209,19 +210,29 @@ dfs_graph* dfs_graph_create(const int64_t* row_ptr, const int32_t* col_idx, int6
         }
         if (!bad) cudaMemcpy(g->d_rp, rp32.data(), (size_t)(n + 1) * sizeof(uint32_t), cudaMemcpyHostToDevice);
     }
+    int32_t* d_col = nullptr;   // staging copy of col_idx (freed after the adjacency is built)
     if (!bad && m > 0) {
-        cudaMemcpy(g->d_col, col_idx, (size_t)m * sizeof(int32_t), cudaMemcpyDefault);
+        if (cudaMalloc(&d_col, (size_t)m * sizeof(int32_t)) != cudaSuccess) {
+            cudaGetLastError(); cudaFree(d_bad); free_graph(g); fail(DFS_ENOMEM); return nullptr;
+        }
+        cudaMemcpy(d_col, col_idx, (size_t)m * sizeof(int32_t), cudaMemcpyDefault);
         const int blocks = (int)std::min<int64_t>((m + 255) / 256, 65535);
-        dfs_validate_col_kernel<<<blocks, 256>>>(g->d_col, m, n, d_bad);
+        dfs_validate_col_kernel<<<blocks, 256>>>(d_col, m, n, d_bad);
         g->launches++;
     }
     int hbad = 0;
     cudaMemcpy(&hbad, d_bad, sizeof(int), cudaMemcpyDeviceToHost);
     cudaFree(d_bad);
+    if (!bad && !hbad && m > 0) {
+        const int blocks = (int)std::min<int64_t>((m + 255) / 256, 65535);
+        dfs_build_adj_kernel<<<blocks, 256>>>(d_col, g->d_rp, g->d_adj, m);
+        g->launches++;
+    }
+    cudaFree(d_col);
     if (cudaGetLastError() != cudaSuccess) { free_graph(g); fail(DFS_ECUDA); return nullptr; }
     if (bad || hbad) { free_graph(g); fail(DFS_EINVAL); return nullptr; }
     cudaMemset(g->d_tab, 0xFF, g->tab_words * sizeof(uint32_t));   // all chunk slots empty
-    cudaMemset(g->d_col + m, 0xFF, 8 * sizeof(int32_t));            // padding (never a valid position)
+    cudaMemset(g->d_adj + m, 0xFF, 8 * sizeof(uint2));              // padding (never a valid position)
     if (cudaDeviceSynchronize() != cudaSuccess) { cudaGetLastError(); free_graph(g); fail(DFS_ECUDA); return nullptr; }
     return g;
 }
@@ -291,7 +302,7 @@ static int launch_one(dfs_graph* g, int32_t root, int32_t* d_out, const dfs_opti
     g->tab_dirty = false;
 
     KParams P;
-    P.rp = g->d_rp; P.col = g->d_col; P.bitmap = g->d_bitmap; P.parent = d_out;
+    P.rp = g->d_rp; P.adj = g->d_adj; P.bitmap = g->d_bitmap; P.parent = d_out;
     P.cold_tb = g->d_cold_tb; P.chunk_tab = g->d_tab; P.pool = g->d_pool;
     P.chunk_consumed = g->d_consumed; P.chunk_next = g->d_next; P.block_cold = g->d_block_cold;
     P.ctl = g->d_ctl;
@@ -307,6 +318,7 @@ static int launch_one(dfs_graph* g, int32_t root, int32_t* d_out, const dfs_opti
     P.pub_batch = o.pub_batch > 0 ? (uint32_t)o.pub_batch : 4u;
     P.speculate = o.speculate;
     P.steal_half = o.steal_half;
+    P.probe_mode = o.probe_mode;
     P.timeline = g->d_timeline;
     P.timeline_len = g->timeline_len;
     P.timeline_dt_ns = g->timeline_dt_ns;
@@ -429,6 +441,10 @@ static int run_many(dfs_graph* g, const int32_t* roots_host, int32_t k, int32_t*
         stats->idle_ns = (int64_t)counters[kCntIdleNs];
         stats->inter_scans = (int64_t)counters[kCntInterScans];
         stats->spills = (int64_t)counters[kCntSpills];
+        stats->cyc_window = (int64_t)counters[kCntTWin];
+        stats->cyc_probe = (int64_t)counters[kCntTProbe];
+        stats->cyc_claim = (int64_t)counters[kCntTClaim];
+        stats->cyc_tail = (int64_t)counters[kCntTTail];
     }
     return DFS_OK;
 }

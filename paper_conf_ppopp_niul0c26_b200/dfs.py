@@ -46,7 +46,8 @@ class _Options(ctypes.Structure):
                 ("inter_any", ctypes.c_int32), ("spill_idle", ctypes.c_int32),
                 ("backoff_max_ns", ctypes.c_int32), ("window", ctypes.c_int32),
                 ("pub_batch", ctypes.c_int32), ("speculate", ctypes.c_int32),
-                ("steal_half", ctypes.c_int32), ("reserved", ctypes.c_int32 * 3)]
+                ("steal_half", ctypes.c_int32), ("probe_mode", ctypes.c_int32),
+                ("reserved", ctypes.c_int32 * 2)]
 
 
 class _Stats(ctypes.Structure):
@@ -58,7 +59,9 @@ class _Stats(ctypes.Structure):
                 ("intra_steals", ctypes.c_int64), ("inter_steals", ctypes.c_int64),
                 ("steal_attempts", ctypes.c_int64), ("chunks_allocated", ctypes.c_int64),
                 ("windows", ctypes.c_int64), ("idle_ns", ctypes.c_int64),
-                ("inter_scans", ctypes.c_int64), ("spills", ctypes.c_int64)]
+                ("inter_scans", ctypes.c_int64), ("spills", ctypes.c_int64),
+                ("cyc_window", ctypes.c_int64), ("cyc_probe", ctypes.c_int64),
+                ("cyc_claim", ctypes.c_int64), ("cyc_tail", ctypes.c_int64)]
 
 
 @dataclass
@@ -83,6 +86,7 @@ class Options:
     pub_batch: Optional[int] = None
     speculate: Optional[int] = None
     steal_half: Optional[bool] = None
+    probe_mode: Optional[int] = None
 
     def to_c(self) -> _Options:
         o = _Options()
@@ -114,6 +118,10 @@ class Stats:
     idle_ns: int
     inter_scans: int
     spills: int
+    cyc_window: int
+    cyc_probe: int
+    cyc_claim: int
+    cyc_tail: int
 
 
 _lib = None

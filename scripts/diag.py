@@ -90,6 +90,12 @@ VARIANTS = {
     "h1c2": dict(hot_cutoff=1, cold_cutoff=2),
     "h4c4": dict(hot_cutoff=4, cold_cutoff=4),
     "h1c1nohalf": dict(hot_cutoff=1, cold_cutoff=1, steal_half=False),
+    "det_p1": dict(deterministic=True, probe_mode=1),
+    "det_p2": dict(deterministic=True, probe_mode=2),
+    "det_p1nospec": dict(deterministic=True, probe_mode=1, speculate=0),
+    "p1": dict(probe_mode=1),
+    "p2": dict(probe_mode=2),
+    "p1nospec": dict(probe_mode=1, speculate=0),
 }
 
 
@@ -150,7 +156,9 @@ def main():
                        refills=st.refills, intra=st.intra_steals, inter=st.inter_steals,
                        attempts=st.steal_attempts, scans=st.inter_scans, spills=st.spills, chunks=st.chunks_allocated,
                        us_per_claim_per_warp=round(st.traversal_ms * 1e3 * warps * util / max(1, st.claims), 3),
-                       windows_per_claim=round(st.windows / max(1, st.claims), 3))
+                       windows_per_claim=round(st.windows / max(1, st.claims), 3),
+                       cyc_per_window=[round(x / max(1, st.windows), 1) for x in
+                                       (st.cyc_window, st.cyc_probe, st.cyc_claim, st.cyc_tail)])
             if a.timeline:
                 G.run(int(r), out=out, options=o)      # sampled run
                 tl = G.timeline(TL, a.timeline * 1000, fetch=True)
