@@ -47,7 +47,8 @@ def parse():
     ap.add_argument("--steps", type=int, default=10)
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--config", default="road24m",
-                    choices=["road24m", "grid256", "rmat24", "path100m", "caterpillar"])
+                    choices=["road24m", "grid256", "rmat24", "path100m", "caterpillar", "batch1024"])
+    ap.add_argument("--batch-roots", type=int, default=1024)
     ap.add_argument("--impl", default="b200", choices=["b200", "reference"])
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu-baseline", action="store_true")
@@ -163,6 +164,8 @@ def main():
 
     if a.impl == "reference":
         return reference_arm(a, world, rank)
+    if a.config == "batch1024":
+        return batch_arm(a, world, rank, local)
 
     import torch
     import torch.distributed as dist
@@ -292,6 +295,69 @@ def main():
     if not a.no_e2e:
         rec["e2e"] = e2e_leg(a, g, my_roots, m_r, dfsmod)
     print(json.dumps(rec), flush=True)
+    G.close()
+    if world > 1:
+        dist.destroy_process_group()
+
+
+def batch_arm(a, world, rank, local):
+    """C5 (BASELINE.json configs[4]): 1,024 seeded roots on the replicated road graph, partitioned
+    contiguously across ranks (strong scaling); one NCCL all_gather of per-root summaries."""
+    import torch
+    import torch.distributed as dist
+
+    import graphgen
+    from paper_conf_ppopp_niul0c26_b200 import Graph
+    from paper_conf_ppopp_niul0c26_b200 import batch
+
+    torch.cuda.set_device(local)
+    if world > 1:
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    dev = torch.device("cuda", local)
+    t0 = time.time()
+    g = graphgen.road(4900, 4900)
+    roots = graphgen.random_roots(g, a.batch_roots, seed=0xC5)
+    log(f"[rank {rank}] batch graph n={g.n} m={g.m} built in {time.time() - t0:.1f}s; {len(roots)} roots")
+    G = Graph(g.row_ptr, g.col_idx)
+    lo, hi = batch.partition(len(roots), world, rank)
+    out_rows = torch.empty((min(16, max(1, hi - lo)), g.n), dtype=torch.int32, device=dev)
+    for s_ in range(a.warmup):                       # warm-up traversals (untimed)
+        G.run(int(roots[(lo + s_) % len(roots)]), out=out_rows[0])
+    launches0 = G.launch_count()
+    clocks = ClockSampler(local)
+    clocks.start()
+    if world > 1:
+        dist.barrier()
+    torch.cuda.synchronize()
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    e0.record()
+    res = batch.run_batch(batch.gpu_runner(G, out_rows), roots, world=world, rank=rank, device=dev)
+    e1.record()
+    torch.cuda.synchronize()
+    if world > 1:
+        dist.barrier()
+    clk = clocks.stop()
+    region_ms = e0.elapsed_time(e1)
+    if world > 1:
+        t = torch.tensor([region_ms], dtype=torch.float64, device=dev)
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        region_ms = float(t.item())
+    launches = G.launch_count() - launches0
+    if rank == 0:
+        k = len(roots)
+        rec = {"metric": METRIC, "value": round(res.gteps(), 6), "unit": "GTEPS", "n_gpus": world,
+               "steps": k, "warmup": a.warmup, "ms_per_step": round(res.max_ms / max(1, hi - lo), 4),
+               "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "int32",
+               "data": "synthetic",
+               "config": {"workload": "batch1024", "desc": "C5: road-maze 4900x4900, 1024 seeded roots "
+                          "partitioned contiguously across ranks, NCCL all_gather of per-root summaries",
+                          "n": g.n, "m": g.m, "roots": k, "parallelism": f"replicas x{world}",
+                          "l2": f"inputs larger than L2 ({((g.n + 1) * 4 + g.m * 8 + g.n * 4) / 1e6:.0f} MB)"},
+               "dfs_per_s": round(res.dfs_per_s(), 3),
+               "dfs_per_s_region": round(k / (region_ms * 1e-3), 3),
+               "region_ms": round(region_ms, 3), "gpu_launches": int(launches), "clocks": clk,
+               "exchange": "all_gather_into_tensor of (k x 5) float64 summaries"}
+        print(json.dumps(rec), flush=True)
     G.close()
     if world > 1:
         dist.destroy_process_group()

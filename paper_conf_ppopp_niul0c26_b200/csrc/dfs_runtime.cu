@@ -388,7 +388,7 @@ static int run_many(dfs_graph* g, const int32_t* roots_host, int32_t k, int32_t*
         rc = launch_one(g, roots_host[q], d_out, o, blocks, warps, stats != nullptr);
         if (rc != DFS_OK) return fail(rc);
         cudaEventRecord(g->ev1, g->stream);
-        if (stats && o.collect_stats) {
+        if (stats) {
             cudaMemsetAsync(g->d_count2, 0, 2 * sizeof(unsigned long long), g->stream);
             dfs_count_kernel<<<g->sms * 4, 256, 0, g->stream>>>(g->d_bitmap, g->d_rp, (uint32_t)g->n, g->d_count2);
             g->launches++;
@@ -414,7 +414,7 @@ static int run_many(dfs_graph* g, const int32_t* roots_host, int32_t k, int32_t*
             total_ms += ms;
             trav_ms += kms;
             for (int c = 0; c < kNumCounters; ++c) counters[c] += h.counters[c];
-            if (o.collect_stats) {
+            {
                 unsigned long long c2[2];
                 cudaMemcpyAsync(c2, g->d_count2, sizeof(c2), cudaMemcpyDeviceToHost, g->stream);
                 cudaStreamSynchronize(g->stream);

@@ -232,12 +232,11 @@ class Graph:
 
     @staticmethod
     def _opts(options: Optional[Options], stats: bool):
-        if options is None and not stats:
+        # stats=True returns dfs_stats (times, visited counts); the scheduler counters are only
+        # compiled in when options.collect_stats is set
+        if options is None:
             return None
-        o = (options or Options()).to_c()
-        if stats:
-            o.collect_stats = 1
-        return o
+        return options.to_c()
 
     # -- API ----------------------------------------------------------------------------
     def run(self, root: int, out=None, options: Optional[Options] = None, stats: bool = False):

@@ -139,7 +139,7 @@ def main():
     if a.timeline:
         G.timeline(TL, a.timeline * 1000)
     for vn in a.variants.split(","):
-        o = Options(**VARIANTS[vn])
+        o = Options(collect_stats=True, **VARIANTS[vn])
         for r in roots:
             best = None
             for _ in range(a.reps):

@@ -218,11 +218,14 @@ def test_errors():
 def test_stats_counters():
     g = graphgen.road(512, 512, seed=3)
     with Graph(g.row_ptr, g.col_idx) as G:
-        p, st = G.run(0, stats=True)
+        p, st = G.run(0, stats=True, options=Options(collect_stats=True))
         r = _valid(g, 0, p)
         assert st.n_visited == r.n_visited and st.m_visited == r.m_visited
         assert st.claims == r.n_visited - 1
-        assert st.kernel_ms > 0
+        assert st.kernel_ms > 0 and 0 < st.traversal_ms <= st.kernel_ms
+        p2, st2 = G.run(7, stats=True)                 # counts without the counter build
+        r2 = _valid(g, 7, p2)
+        assert st2.n_visited == r2.n_visited and st2.m_visited == r2.m_visited and st2.claims == 0
 
 
 def test_stream_and_repeat_consistency():
