@@ -256,6 +256,7 @@ __global__ void __launch_bounds__(32 * WMAX, 1) dfs_persistent_kernel(const KPar
     static_assert(VEC == 1 || VEC == 4, "VEC is 1 or 4");
     constexpr uint32_t kBatch = H / 2;              // flush batch (reading S10)
     constexpr uint32_t kWin = 32u * VEC;            // positions per window
+    constexpr int kHeadLanes = 8;                   // lanes fetched before a window's end is known
     extern __shared__ __align__(16) unsigned char smem_raw[];
     SmemCtl& S = *reinterpret_cast<SmemCtl*>(smem_raw);
     constexpr int kCtlBytes = (sizeof(SmemCtl) + 15) & ~15;
@@ -311,11 +312,14 @@ __global__ void __launch_bounds__(32 * WMAX, 1) dfs_persistent_kernel(const KPar
     // window loader: lane holds positions base + VEC*lane + e, e < VEC.  Each entry is
     // {v, row_ptr[v]}, so the child's window address is known as soon as its id is: one
     // dependent load per DFS level instead of two (col_idx then row_ptr).
-    auto load_window = [&](uint32_t base, int* nb, uint32_t* rs) {
+    // Only lanes < `lanes` load (a window whose end is not yet known is fetched for its first
+    // kHeadLanes lanes; the rest is loaded once the end shows it is needed).
+    auto load_window = [&](uint32_t base, uint32_t limit, int lanes, int* nb, uint32_t* rs, int lane_lo = 0) {
         const uint32_t q = base + (uint32_t)VEC * lane;
+        const bool ld = lane >= lane_lo && lane < lanes && q < limit;
         if constexpr (VEC == 4) {
             uint4 x0 = make_uint4(kFull, 0u, kFull, 0u), x1 = x0;
-            if (q < P.m) {                                                   // adj padded
+            if (ld) {                                                        // adj padded
                 x0 = __ldg(reinterpret_cast<const uint4*>(P.adj + q));
                 x1 = __ldg(reinterpret_cast<const uint4*>(P.adj + q + 2));
             }
@@ -323,10 +327,12 @@ __global__ void __launch_bounds__(32 * WMAX, 1) dfs_persistent_kernel(const KPar
             nb[2] = (int)x1.x; rs[2] = x1.y; nb[3] = (int)x1.z; rs[3] = x1.w;
         } else {
             uint2 x = make_uint2(kFull, 0u);
-            if (q < P.m) x = __ldg(P.adj + q);
+            if (ld) x = __ldg(P.adj + q);
             nb[0] = (int)x.x; rs[0] = x.y;
         }
     };
+    // lanes of the current window that hold data (the rest are loaded on demand)
+    int win_lanes = 32;
 
     // ---------------------------------------------------------------- owner stack operations
     // publish the private entries [pub, my_head) to thieves (CTA-scope release)
@@ -522,9 +528,29 @@ __global__ void __launch_bounds__(32 * WMAX, 1) dfs_persistent_kernel(const KPar
             // Window = positions [a, a + kWin), a = i rounded down to a multiple of VEC; lane k
             // holds positions a+VEC*k .. a+VEC*k+VEC-1.  Positions outside [i, end) are masked.
             if (!have_win) {
-                const uint32_t e2 = need_end ? __ldg(P.rp + u + 1) : end;
-                load_window(i & ~(uint32_t)(VEC - 1), nbv, rsv);
-                end = e2; need_end = false;
+                if (need_end) {                                   // popped entry: end unknown
+                    const uint32_t e2 = __ldg(P.rp + u + 1);
+                    load_window(i & ~(uint32_t)(VEC - 1), P.m, kHeadLanes, nbv, rsv);
+                    win_lanes = kHeadLanes;
+                    end = e2; need_end = false;
+                } else {
+                    load_window(i & ~(uint32_t)(VEC - 1), end, 32, nbv, rsv);
+                    win_lanes = 32;
+                }
+            }
+            {
+                // complete a head-only window when the list is longer than its loaded lanes
+                const uint32_t a0 = i & ~(uint32_t)(VEC - 1);
+                if (win_lanes < 32 && end > a0 + (uint32_t)VEC * (uint32_t)win_lanes) {
+                    int tnb[VEC];
+                    uint32_t trs[VEC];
+                    load_window(a0, end, 32, tnb, trs, win_lanes);
+                    if (lane >= win_lanes) {
+#pragma unroll
+                        for (int f = 0; f < VEC; ++f) { nbv[f] = tnb[f]; rsv[f] = trs[f]; }
+                    }
+                    win_lanes = 32;
+                }
             }
             if (STATS && lane == 0) ++cnt[kCntWindows];
             long long tc0 = 0, tc1 = 0;
@@ -536,7 +562,7 @@ __global__ void __launch_bounds__(32 * WMAX, 1) dfs_persistent_kernel(const KPar
             int nxt[VEC];
             uint32_t nxr[VEC];
             const bool have_nxt = a + kWin < end;
-            if (have_nxt) load_window(a + kWin, nxt, nxr);
+            if (have_nxt) load_window(a + kWin, end, 32, nxt, nxr);
             // speculative claim (fresh child only): the first position whose neighbour is not the
             // parent we came from is, if unvisited, exactly Alg 1's next tree edge.  Its claim,
             // its end offset and its first window are all issued in parallel with the probes.
@@ -563,7 +589,7 @@ __global__ void __launch_bounds__(32 * WMAX, 1) dfs_persistent_kernel(const KPar
                     s_rs = __shfl_sync(kFull, pick_rs, sk);
                     if (lane == 0) s_old = atomicOr(P.bitmap + (sv >> 5), 1u << (sv & 31));
                     s_re = __ldg(P.rp + sv + 1);
-                    load_window(s_rs & ~(uint32_t)(VEC - 1), cnb, cnr);
+                    load_window(s_rs & ~(uint32_t)(VEC - 1), P.m, kHeadLanes, cnb, cnr);
                 }
             }
             // probe the visited bits of every position in the window
@@ -605,6 +631,7 @@ __global__ void __launch_bounds__(32 * WMAX, 1) dfs_persistent_kernel(const KPar
                 }
                 par = u;
                 u = v; i = vrs; end = vre; have_win = true; need_end = false; spec_ok = true;
+                win_lanes = kHeadLanes;
 #pragma unroll
                 for (int f = 0; f < VEC; ++f) { nbv[f] = cnb[f]; rsv[f] = cnr[f]; }
                 descended = true;
@@ -638,7 +665,7 @@ __global__ void __launch_bounds__(32 * WMAX, 1) dfs_persistent_kernel(const KPar
                 if (lane == 0) old = atomicOr(P.bitmap + (v >> 5), bit);          // claim
                 // the child's end offset and first window load overlap the claim
                 const uint32_t vre = __ldg(P.rp + v + 1);
-                load_window(vrs & ~(uint32_t)(VEC - 1), cnb, cnr);
+                load_window(vrs & ~(uint32_t)(VEC - 1), P.m, kHeadLanes, cnb, cnr);
                 old = __shfl_sync(kFull, old, 0);
                 if (!(old & bit)) {
                     if (!descend(k, e, v, vrs, vre)) goto exit_loop;
@@ -660,6 +687,7 @@ __global__ void __launch_bounds__(32 * WMAX, 1) dfs_persistent_kernel(const KPar
 #pragma unroll
                     for (int f = 0; f < VEC; ++f) { nbv[f] = nxt[f]; rsv[f] = nxr[f]; }
                     have_win = true;
+                    win_lanes = 32;
                 } else {
                     have_win = false;                             // i >= end: Alg 1 l.14: pop
                     has_top = pop(u, i);
