@@ -49,6 +49,8 @@ def parse():
     ap.add_argument("--config", default="road24m",
                     choices=["road24m", "grid256", "rmat24", "path100m", "caterpillar", "batch1024"])
     ap.add_argument("--batch-roots", type=int, default=1024)
+    ap.add_argument("--concurrency", type=int, default=0,
+                    help="batch1024: traversals in flight per GPU (0 = auto)")
     ap.add_argument("--impl", default="b200", choices=["b200", "reference"])
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu-baseline", action="store_true")
@@ -320,7 +322,8 @@ def batch_arm(a, world, rank, local):
     log(f"[rank {rank}] batch graph n={g.n} m={g.m} built in {time.time() - t0:.1f}s; {len(roots)} roots")
     G = Graph(g.row_ptr, g.col_idx)
     lo, hi = batch.partition(len(roots), world, rank)
-    out_rows = torch.empty((min(16, max(1, hi - lo)), g.n), dtype=torch.int32, device=dev)
+    conc = a.concurrency if a.concurrency > 0 else 4
+    out_rows = torch.empty((max(conc, min(16, max(1, hi - lo))), g.n), dtype=torch.int32, device=dev)
     for s_ in range(a.warmup):                       # warm-up traversals (untimed)
         G.run(int(roots[(lo + s_) % len(roots)]), out=out_rows[0])
     launches0 = G.launch_count()
@@ -331,7 +334,7 @@ def batch_arm(a, world, rank, local):
     torch.cuda.synchronize()
     e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
     e0.record()
-    res = batch.run_batch(batch.gpu_runner(G, out_rows), roots, world=world, rank=rank, device=dev)
+    res = batch.run_batch_chunked(G, out_rows, roots, world=world, rank=rank, device=dev, concurrency=conc)
     e1.record()
     torch.cuda.synchronize()
     if world > 1:
@@ -356,7 +359,8 @@ def batch_arm(a, world, rank, local):
                "dfs_per_s": round(res.dfs_per_s(), 3),
                "dfs_per_s_region": round(k / (region_ms * 1e-3), 3),
                "region_ms": round(region_ms, 3), "gpu_launches": int(launches), "clocks": clk,
-               "exchange": "all_gather_into_tensor of (k x 5) float64 summaries"}
+               "exchange": "all_gather_into_tensor of (k x 5) float64 summaries",
+               "concurrency": conc}
         print(json.dumps(rec), flush=True)
     G.close()
     if world > 1:

@@ -111,7 +111,12 @@ typedef struct dfs_options {
     int32_t probe_mode;      /* visited probes: 0 = L2 (ld.global.cg, default), 1 = L1-cached,
                                 2 = ld.relaxed.gpu.  A stale probe can only say "unvisited" for a
                                 claimed vertex; the atomic claim decides, so all are exact         */
-    int32_t reserved[2];
+    int32_t concurrency;     /* batches: number of traversals run concurrently on the GPU, each on
+                                its own stream and a 1/concurrency share of the SMs (SURVEY
+                                §8(f)-2); 0 = auto (4, capped by the number of roots; a single
+                                dfs_run is always 1).  Slots beyond the first allocate their
+                                scratch on first use.                                              */
+    int32_t reserved[1];
 } dfs_options;
 
 typedef struct dfs_stats {
@@ -129,6 +134,9 @@ typedef struct dfs_stats {
     /* SM-cycle breakdown of the expansion step summed over windows (collect_stats; diagnostics):
        wait for the window data, wait for the probes, wait for the speculative claim, rest */
     int64_t cyc_window, cyc_probe, cyc_claim, cyc_tail;
+    /* optional, caller-owned host array of 2*num_roots int64 (NULL = not wanted): per-root
+       (n_visited, m_visited) of a batch, in root order */
+    int64_t *root_counts;
 } dfs_stats;
 
 void dfs_options_default(dfs_options *opt);

@@ -127,3 +127,26 @@ def gpu_runner(G, out_rows, collect: Optional[list] = None):
             collect.append(st)
         return st.n_visited, st.m_visited, st.kernel_ms
     return run
+
+
+def run_batch_chunked(G, out_rows, roots, world: int = 1, rank: int = 0, group=None, device=None,
+                      concurrency: int = 1) -> BatchResult:
+    """GPU batch: this rank's slice goes to ``dfs_run_batch_ex`` in chunks of
+    ``out_rows.shape[0]`` roots with ``concurrency`` traversals in flight (§8(f)-2).  Per-root
+    (n_visited, m_visited) come from the library's per-root counts; a chunk's device time (CUDA
+    events) is attributed evenly to its roots.  Then the summaries are exchanged (run_batch)."""
+    from .dfs import Options
+    k = len(roots)
+    lo, hi = partition(k, world, rank)
+    mine = [int(r) for r in roots[lo:hi]]
+    rows = out_rows.shape[0]
+    results = []
+    for c0 in range(0, len(mine), rows):
+        chunk = mine[c0:c0 + rows]
+        _, st = G.run_batch(chunk, out=out_rows[:len(chunk)], options=Options(concurrency=concurrency),
+                            stats=True)
+        share = st.kernel_ms / len(chunk)
+        for q in range(len(chunk)):
+            results.append((int(st.root_counts[q, 0]), int(st.root_counts[q, 1]), share))
+    it = iter(results)
+    return run_batch(lambda root, q: next(it), roots, world=world, rank=rank, group=group, device=device)

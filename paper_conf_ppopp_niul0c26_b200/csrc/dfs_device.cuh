@@ -989,8 +989,10 @@ __global__ void dfs_reset_kernel(uint32_t* bitmap, uint32_t nwords, unsigned lon
     }
 }
 
-__global__ void dfs_finalize_kernel(const uint32_t* __restrict__ bitmap, int32_t* parent, uint32_t n) {
+__global__ void dfs_finalize_kernel(const uint32_t* __restrict__ bitmap, int32_t* parent, uint32_t n,
+                                    const Ctl* ctl, int* status_acc) {
     const size_t stride = (size_t)gridDim.x * blockDim.x;
+    if (blockIdx.x == 0 && threadIdx.x == 0 && ctl->status != 0) atomicMin(status_acc, ctl->status);
     for (size_t v = blockIdx.x * (size_t)blockDim.x + threadIdx.x; v < n; v += stride) {
         const uint32_t word = __ldg(bitmap + (v >> 5));
         if (!((word >> (v & 31)) & 1u)) parent[v] = -2;            // DFS_UNREACHED (reading S2)

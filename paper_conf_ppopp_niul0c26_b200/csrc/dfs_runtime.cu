@@ -1,9 +1,11 @@
 // dfs_runtime.cu — host runtime + C ABI (include/dfs.h) of the B200 unordered-DFS library.
 //
-// Owns graph residency (step a1: copy, validate, narrow row_ptr to uint32), the per-handle
-// scratch (visited bitmap, per-warp ColdSeg words, chunk table, chunk pool, control block),
-// and the per-traversal launch sequence: reset (a2) -> persistent traversal (a3-a8) ->
-// finalize (a9).  "P:a-b" = /root/reference/PAPER.md lines.
+// Owns graph residency (step a1: copy, validate, narrow row_ptr to uint32, build the
+// edge-annotated adjacency {v, row_ptr[v]}), per-traversal scratch "slots" (visited bitmap,
+// per-warp ColdSeg words, chunk table, chunk pool, control block) and the launch sequence
+// reset (a2) -> persistent traversal (a3-a8) -> finalize (a9).  A batch (a10) may run K
+// traversals concurrently on K slots / streams, each on a 1/K share of the SMs (SURVEY
+// §8(f)-2).  "P:a-b" = /root/reference/PAPER.md lines.
 #include <cuda_runtime.h>
 
 #include <algorithm>
@@ -22,6 +24,7 @@ using namespace b200dfs;
 namespace {
 
 constexpr int kRing = 256;                   // HotRing entries per warp (P:367 uses 128)
+constexpr int kMaxSlots = 8;                 // concurrent traversals per handle (batches)
 thread_local int g_last_error = DFS_OK;
 
 int fail(int code) { g_last_error = code; return code; }
@@ -46,6 +49,27 @@ size_t smem_bytes(int warps) {
     return ((sizeof(SmemCtl) + 15) & ~size_t(15)) + (size_t)warps * kRing * sizeof(unsigned long long);
 }
 
+// per-traversal scratch set
+struct Slot {
+    bool ready = false;
+    uint32_t* bitmap = nullptr;
+    int32_t* parent = nullptr;              // lazily allocated for host outputs
+    unsigned long long* cold_tb = nullptr;
+    uint32_t* tab = nullptr;
+    unsigned long long* pool = nullptr;
+    uint32_t* consumed = nullptr;
+    uint32_t* next = nullptr;
+    int* block_cold = nullptr;
+    Ctl* ctl = nullptr;
+    unsigned long long* count2 = nullptr;   // visited count, TEPS numerator (summed over a batch)
+    int* status = nullptr;                  // worst status over the slot's traversals in a batch
+    size_t tab_words = 0;
+    uint32_t n_chunks = 0;
+    bool tab_dirty = false;
+    cudaStream_t stream = nullptr;          // own stream (slots >= 1 of a concurrent batch)
+    cudaEvent_t ev0 = nullptr, ev1 = nullptr, evk0 = nullptr, evk1 = nullptr;
+};
+
 }  // namespace
 
 struct dfs_graph {
@@ -54,43 +78,73 @@ struct dfs_graph {
     int64_t n = 0, m = 0;
     int sms = 0;
     int max_blocks = 0;          // co-resident 32-warp blocks (allocation bound)
+    int tab_log2 = 0;
     uint32_t* d_rp = nullptr;
     uint2* d_adj = nullptr;      // {col_idx[j], row_ptr[col_idx[j]]} per CSR entry (+8 padding)
-    uint32_t* d_bitmap = nullptr;
-    int32_t* d_parent = nullptr; // lazily allocated for host outputs
-    unsigned long long* d_cold_tb = nullptr;
-    uint32_t* d_tab = nullptr;
-    unsigned long long* d_pool = nullptr;
-    uint32_t* d_consumed = nullptr;
-    uint32_t* d_next = nullptr;
-    int* d_block_cold = nullptr;
-    Ctl* d_ctl = nullptr;
-    unsigned long long* d_count2 = nullptr;
-    int tab_log2 = 0;
-    uint32_t n_chunks = 0;
-    size_t tab_words = 0;
-    bool tab_dirty = false;
+    Slot slots[kMaxSlots];
     int64_t launches = 0;
-    cudaEvent_t ev0 = nullptr, ev1 = nullptr, evk0 = nullptr, evk1 = nullptr;
     unsigned int* d_timeline = nullptr;   // diagnostics (dfs_debug_timeline)
     unsigned int timeline_len = 0, timeline_dt_ns = 0;
+    unsigned long long* d_counts = nullptr;   // per-root (n_visited, m_visited) of a stats call
+    int32_t counts_cap = 0;
 };
+
+static void free_slot(Slot& s) {
+    cudaFree(s.bitmap); cudaFree(s.parent); cudaFree(s.cold_tb); cudaFree(s.tab); cudaFree(s.pool);
+    cudaFree(s.consumed); cudaFree(s.next); cudaFree(s.block_cold); cudaFree(s.ctl); cudaFree(s.count2);
+    cudaFree(s.status);
+    if (s.stream) cudaStreamDestroy(s.stream);
+    if (s.ev0) cudaEventDestroy(s.ev0);
+    if (s.ev1) cudaEventDestroy(s.ev1);
+    if (s.evk0) cudaEventDestroy(s.evk0);
+    if (s.evk1) cudaEventDestroy(s.evk1);
+    s = Slot();
+}
 
 static void free_graph(dfs_graph* g) {
     if (!g) return;
     int cur = 0;
     cudaGetDevice(&cur);
     cudaSetDevice(g->device);
-    cudaFree(g->d_rp); cudaFree(g->d_adj); cudaFree(g->d_bitmap); cudaFree(g->d_parent);
-    cudaFree(g->d_cold_tb); cudaFree(g->d_tab); cudaFree(g->d_pool); cudaFree(g->d_consumed);
-    cudaFree(g->d_next); cudaFree(g->d_block_cold); cudaFree(g->d_ctl); cudaFree(g->d_count2);
-    cudaFree(g->d_timeline);
-    if (g->ev0) cudaEventDestroy(g->ev0);
-    if (g->ev1) cudaEventDestroy(g->ev1);
-    if (g->evk0) cudaEventDestroy(g->evk0);
-    if (g->evk1) cudaEventDestroy(g->evk1);
+    cudaFree(g->d_rp); cudaFree(g->d_adj); cudaFree(g->d_timeline); cudaFree(g->d_counts);
+    for (int k = 0; k < kMaxSlots; ++k) free_slot(g->slots[k]);
     cudaSetDevice(cur);
     delete g;
+}
+
+// allocate scratch slot k (sized for every warp of the device, so any block split fits)
+static int ensure_slot(dfs_graph* g, int k) {
+    Slot& s = g->slots[k];
+    if (s.ready) return DFS_OK;
+    const int64_t n = g->n;
+    const int64_t n_warps = (int64_t)g->max_blocks * kMaxWarps;
+    s.tab_words = (size_t)n_warps << g->tab_log2;
+    // pool: sum of live spans <= n, plus <= 4 partially used chunks per warp (reading S9)
+    s.n_chunks = (uint32_t)(n / kChunk + 4 * n_warps + 16);
+    const size_t nwords = (size_t)((n + 31) / 32);
+    bool ok = true;
+    auto A = [&](void** p, size_t bytes) { if (ok && cudaMalloc(p, bytes ? bytes : 16) != cudaSuccess) ok = false; };
+    A((void**)&s.bitmap, nwords * sizeof(uint32_t));
+    A((void**)&s.cold_tb, (size_t)n_warps * sizeof(unsigned long long));
+    A((void**)&s.tab, s.tab_words * sizeof(uint32_t));
+    A((void**)&s.pool, (size_t)s.n_chunks * kChunk * sizeof(unsigned long long));
+    A((void**)&s.consumed, (size_t)s.n_chunks * sizeof(uint32_t));
+    A((void**)&s.next, (size_t)s.n_chunks * sizeof(uint32_t));
+    A((void**)&s.block_cold, (size_t)g->max_blocks * sizeof(int));
+    A((void**)&s.ctl, sizeof(Ctl));
+    A((void**)&s.count2, 2 * sizeof(unsigned long long));
+    A((void**)&s.status, sizeof(int));
+    if (!ok) { cudaGetLastError(); free_slot(s); return DFS_ENOMEM; }
+    if (cudaEventCreate(&s.ev0) != cudaSuccess || cudaEventCreate(&s.ev1) != cudaSuccess ||
+        cudaEventCreate(&s.evk0) != cudaSuccess || cudaEventCreate(&s.evk1) != cudaSuccess ||
+        (k > 0 && cudaStreamCreateWithFlags(&s.stream, cudaStreamNonBlocking) != cudaSuccess)) {
+        cudaGetLastError(); free_slot(s); return DFS_ECUDA;
+    }
+    if (cudaMemset(s.tab, 0xFF, s.tab_words * sizeof(uint32_t)) != cudaSuccess) {   // all chunk slots empty
+        cudaGetLastError(); free_slot(s); return DFS_ECUDA;
+    }
+    s.ready = true;
+    return DFS_OK;
 }
 
 extern "C" {
@@ -118,6 +172,7 @@ void dfs_options_default(dfs_options* o) {
     o->speculate = 2;
     o->steal_half = 1;
     o->probe_mode = 0;
+    o->concurrency = 0;
 }
 
 int dfs_last_error(void) { return g_last_error; }
@@ -151,8 +206,7 @@ dfs_graph* dfs_graph_create(const int64_t* row_ptr, const int32_t* col_idx, int6
     const size_t sm32 = smem_bytes(32);
     bool attr_ok = true;
     for (int kf = 0; kf < 8; ++kf) {
-        const void* f = kernel_table()[kf];
-        if (f && cudaFuncSetAttribute(f, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm32) != cudaSuccess)
+        if (cudaFuncSetAttribute(kernel_table()[kf], cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm32) != cudaSuccess)
             attr_ok = false;
     }
     if (!attr_ok) { cudaGetLastError(); delete g; fail(DFS_ECUDA); return nullptr; }
@@ -162,35 +216,17 @@ dfs_graph* dfs_graph_create(const int64_t* row_ptr, const int32_t* col_idx, int6
         cudaGetLastError(); per_sm = 1;
     }
     g->max_blocks = g->sms * per_sm;
-
-    const int64_t n_warps = (int64_t)g->max_blocks * kMaxWarps;
     // chunk table: 2^tab_log2 >= (max live span + 2 chunks + flush batch) / chunk  (reading S9)
-    int64_t need = (n + 2 * (int64_t)kChunk + kRing) / kChunk + 2;
+    const int64_t need = (n + 2 * (int64_t)kChunk + kRing) / kChunk + 2;
     g->tab_log2 = 2;
     while (((int64_t)1 << g->tab_log2) < need) ++g->tab_log2;
-    g->tab_words = (size_t)n_warps << g->tab_log2;
-    // pool: sum of live spans <= n, plus <= 4 partially used chunks per warp
-    g->n_chunks = (uint32_t)(n / kChunk + 4 * n_warps + 16);
 
-    const size_t nwords = (size_t)((n + 31) / 32);
-    bool ok = true;
-    auto A = [&](void** p, size_t bytes) { if (ok && cudaMalloc(p, bytes ? bytes : 16) != cudaSuccess) ok = false; };
-    A((void**)&g->d_rp, (size_t)(n + 1) * sizeof(uint32_t));
-    A((void**)&g->d_adj, (size_t)(m + 8) * sizeof(uint2));       // padded for 128-bit window loads
-    A((void**)&g->d_bitmap, nwords * sizeof(uint32_t));
-    A((void**)&g->d_cold_tb, (size_t)n_warps * sizeof(unsigned long long));
-    A((void**)&g->d_tab, g->tab_words * sizeof(uint32_t));
-    A((void**)&g->d_pool, (size_t)g->n_chunks * kChunk * sizeof(unsigned long long));
-    A((void**)&g->d_consumed, (size_t)g->n_chunks * sizeof(uint32_t));
-    A((void**)&g->d_next, (size_t)g->n_chunks * sizeof(uint32_t));
-    A((void**)&g->d_block_cold, (size_t)g->max_blocks * sizeof(int));
-    A((void**)&g->d_ctl, sizeof(Ctl));
-    A((void**)&g->d_count2, 2 * sizeof(unsigned long long));
-    if (!ok) { cudaGetLastError(); free_graph(g); fail(DFS_ENOMEM); return nullptr; }
-    if (cudaEventCreate(&g->ev0) != cudaSuccess || cudaEventCreate(&g->ev1) != cudaSuccess ||
-        cudaEventCreate(&g->evk0) != cudaSuccess || cudaEventCreate(&g->evk1) != cudaSuccess) {
-        cudaGetLastError(); free_graph(g); fail(DFS_ECUDA); return nullptr;
+    if (cudaMalloc(&g->d_rp, (size_t)(n + 1) * sizeof(uint32_t)) != cudaSuccess ||
+        cudaMalloc(&g->d_adj, (size_t)(m + 8) * sizeof(uint2)) != cudaSuccess) {   // padded for 128-bit loads
+        cudaGetLastError(); free_graph(g); fail(DFS_ENOMEM); return nullptr;
     }
+    const int rc = ensure_slot(g, 0);
+    if (rc != DFS_OK) { free_graph(g); fail(rc); return nullptr; }
 
     // ---- copy + validate + narrow (step a1) ----
     int* d_bad = nullptr;
@@ -231,7 +267,6 @@ dfs_graph* dfs_graph_create(const int64_t* row_ptr, const int32_t* col_idx, int6
     cudaFree(d_col);
     if (cudaGetLastError() != cudaSuccess) { free_graph(g); fail(DFS_ECUDA); return nullptr; }
     if (bad || hbad) { free_graph(g); fail(DFS_EINVAL); return nullptr; }
-    cudaMemset(g->d_tab, 0xFF, g->tab_words * sizeof(uint32_t));   // all chunk slots empty
     cudaMemset(g->d_adj + m, 0xFF, 8 * sizeof(uint2));              // padding (never a valid position)
     if (cudaDeviceSynchronize() != cudaSuccess) { cudaGetLastError(); free_graph(g); fail(DFS_ECUDA); return nullptr; }
     return g;
@@ -287,27 +322,26 @@ int dfs_debug_timeline(dfs_graph* g, uint32_t len, uint32_t dt_ns, uint32_t* out
 }  // extern "C"
 
 // ------------------------------------------------------------------------------------------
-// one traversal on the handle's stream (no synchronisation)
+// one traversal on slot `sl`, stream-ordered on `s` (no synchronisation)
 // ------------------------------------------------------------------------------------------
-static int launch_one(dfs_graph* g, int32_t root, int32_t* d_out, const dfs_options& o, int blocks,
-                      int warps, bool timed) {
-    cudaStream_t s = g->stream;
+static int launch_one(dfs_graph* g, Slot& sl, cudaStream_t s, int32_t root, int32_t* d_out,
+                      const dfs_options& o, int blocks, int warps, bool timed, bool cooperative) {
     const uint32_t nwords = (uint32_t)((g->n + 31) / 32);
-    const int rblocks = (int)std::min<int64_t>((std::max<int64_t>(nwords, g->tab_dirty ? (int64_t)g->tab_words : 0) + 255) / 256 + 1,
+    const int rblocks = (int)std::min<int64_t>((std::max<int64_t>(nwords, sl.tab_dirty ? (int64_t)sl.tab_words : 0) + 255) / 256 + 1,
                                                (int64_t)g->sms * 8);
-    dfs_reset_kernel<<<rblocks, 256, 0, s>>>(g->d_bitmap, nwords, g->d_cold_tb, (uint32_t)(blocks * warps),
-                                            g->d_block_cold, (uint32_t)blocks, g->d_ctl, d_out, root,
-                                            g->d_tab, g->tab_dirty ? g->tab_words : 0);
+    dfs_reset_kernel<<<rblocks, 256, 0, s>>>(sl.bitmap, nwords, sl.cold_tb, (uint32_t)(blocks * warps),
+                                            sl.block_cold, (uint32_t)blocks, sl.ctl, d_out, root,
+                                            sl.tab, sl.tab_dirty ? sl.tab_words : 0);
     g->launches++;
-    g->tab_dirty = false;
+    sl.tab_dirty = false;
 
     KParams P;
-    P.rp = g->d_rp; P.adj = g->d_adj; P.bitmap = g->d_bitmap; P.parent = d_out;
-    P.cold_tb = g->d_cold_tb; P.chunk_tab = g->d_tab; P.pool = g->d_pool;
-    P.chunk_consumed = g->d_consumed; P.chunk_next = g->d_next; P.block_cold = g->d_block_cold;
-    P.ctl = g->d_ctl;
+    P.rp = g->d_rp; P.adj = g->d_adj; P.bitmap = sl.bitmap; P.parent = d_out;
+    P.cold_tb = sl.cold_tb; P.chunk_tab = sl.tab; P.pool = sl.pool;
+    P.chunk_consumed = sl.consumed; P.chunk_next = sl.next; P.block_cold = sl.block_cold;
+    P.ctl = sl.ctl;
     P.n = (uint32_t)g->n; P.m = (uint32_t)g->m; P.root = root; P.tab_log2 = g->tab_log2;
-    P.n_chunks = g->n_chunks;
+    P.n_chunks = sl.n_chunks;
     P.hot_cutoff = o.hot_cutoff; P.cold_cutoff = o.cold_cutoff;
     P.intra = o.intra_steal; P.inter = o.inter_steal; P.policy = o.victim_policy;
     P.collect_stats = o.collect_stats;
@@ -315,30 +349,38 @@ static int launch_one(dfs_graph* g, int32_t root, int32_t* d_out, const dfs_opti
     P.spill_idle = o.spill_idle > 0 ? o.spill_idle : 32;
     P.inter_any = o.inter_any;
     P.backoff_max_ns = o.backoff_max_ns > 0 ? (unsigned)o.backoff_max_ns : 2048u;
-    P.pub_batch = o.pub_batch > 0 ? (uint32_t)o.pub_batch : 4u;
+    P.pub_batch = o.pub_batch > 0 ? (uint32_t)o.pub_batch : 1u;
     P.speculate = o.speculate;
     P.steal_half = o.steal_half;
     P.probe_mode = o.probe_mode;
-    P.timeline = g->d_timeline;
-    P.timeline_len = g->timeline_len;
-    P.timeline_dt_ns = g->timeline_dt_ns;
+    const bool tl = g->d_timeline && &sl == &g->slots[0];
+    P.timeline = tl ? g->d_timeline : nullptr;
+    P.timeline_len = tl ? g->timeline_len : 0;
+    P.timeline_dt_ns = tl ? g->timeline_dt_ns : 1;
     P.timeout_ns = (unsigned long long)o.timeout_ms * 1000000ull;
     P.seed = o.seed;
     void* args[] = {(void*)&P};
-    if (timed) cudaEventRecord(g->evk0, s);
     const void* kfn = kernel_table()[(o.window == 128 ? 4 : 0) + (warps <= 16 ? 2 : 0) + (o.collect_stats ? 1 : 0)];
-    cudaError_t e = cudaLaunchCooperativeKernel(kfn, dim3(blocks),
-                                                dim3(32 * warps), args, smem_bytes(warps), s);
+    if (timed) cudaEventRecord(sl.evk0, s);
+    cudaError_t e;
+    if (cooperative) {
+        e = cudaLaunchCooperativeKernel(kfn, dim3(blocks), dim3(32 * warps), args, smem_bytes(warps), s);
+    } else {
+        // concurrent batch slots: co-residency is not required for progress — a block that starts
+        // late finds the traversal done or steals the remaining work
+        e = cudaLaunchKernel(kfn, dim3(blocks), dim3(32 * warps), args, smem_bytes(warps), s);
+    }
     if (e != cudaSuccess) { cudaGetLastError(); return DFS_ECUDA; }
-    if (timed) cudaEventRecord(g->evk1, s);
+    if (timed) cudaEventRecord(sl.evk1, s);
     g->launches++;
     const int fblocks = (int)std::min<int64_t>((g->n + 255) / 256, (int64_t)g->sms * 16);
-    dfs_finalize_kernel<<<fblocks, 256, 0, s>>>(g->d_bitmap, d_out, (uint32_t)g->n);
+    dfs_finalize_kernel<<<fblocks, 256, 0, s>>>(sl.bitmap, d_out, (uint32_t)g->n, sl.ctl, sl.status);
     g->launches++;
     return DFS_OK;
 }
 
-static int resolve_options(const dfs_graph* g, const dfs_options* in, dfs_options& o, int& blocks, int& warps) {
+static int resolve_options(const dfs_graph* g, const dfs_options* in, int num_roots, dfs_options& o,
+                           int& blocks, int& warps, int& conc) {
     dfs_options_default(&o);
     if (in) o = *in;
     if (o.hot_cutoff == 0) o.hot_cutoff = 1;
@@ -351,10 +393,15 @@ static int resolve_options(const dfs_graph* g, const dfs_options* in, dfs_option
     if (o.victim_policy != 0 && o.victim_policy != 1) return DFS_EINVAL;
     if (o.window == 0) o.window = (g->n > 0 && g->m >= 8 * g->n) ? 128 : 32;   // wide windows for dense lists
     if (o.window != 32 && o.window != 128) return DFS_EINVAL;
+    if (o.concurrency < 0 || o.concurrency > kMaxSlots) return DFS_EINVAL;
     warps = o.warps_per_block <= 0 ? 32 : o.warps_per_block;
     if (warps > 32) return DFS_EINVAL;
-    blocks = o.blocks <= 0 ? g->max_blocks : o.blocks;
-    if (blocks > g->max_blocks) return DFS_EINVAL;
+    conc = o.concurrency == 0 ? 4 : o.concurrency;       // auto: 4 in flight (B200 sweep)
+    if (o.deterministic) conc = 1;
+    if (conc > num_roots) conc = std::max(1, num_roots);
+    const int share = std::max(1, g->max_blocks / conc);
+    blocks = o.blocks <= 0 ? share : o.blocks;
+    if (blocks > g->max_blocks || (conc > 1 && blocks * conc > g->max_blocks)) return DFS_EINVAL;
     if (o.deterministic) { blocks = 1; warps = 1; o.intra_steal = 0; o.inter_steal = 0; }
     return DFS_OK;
 }
@@ -365,16 +412,67 @@ static int check_device(const dfs_graph* g) {
     return cur == g->device ? DFS_OK : DFS_EDEVICE;
 }
 
-static int run_many(dfs_graph* g, const int32_t* roots_host, int32_t k, int32_t* out, bool out_dev,
-                    const dfs_options* opt, dfs_stats* stats) {
-    dfs_options o;
-    int blocks = 0, warps = 0;
-    int rc = resolve_options(g, opt, o, blocks, warps);
-    if (rc != DFS_OK) return fail(rc);
-    for (int32_t q = 0; q < k; ++q)
-        if (roots_host[q] < 0 || roots_host[q] >= g->n) return fail(DFS_EINVAL);
-    if (!out_dev && !g->d_parent) {
-        if (cudaMalloc(&g->d_parent, (size_t)g->n * sizeof(int32_t)) != cudaSuccess) {
+static void fill_stats(dfs_stats* stats, int blocks, int warps, float total_ms, float trav_ms, int64_t nv,
+                       int64_t mv, const unsigned long long* counters) {
+    int64_t* keep = stats->root_counts;
+    std::memset(stats, 0, sizeof(*stats));
+    stats->root_counts = keep;
+    stats->kernel_ms = total_ms;
+    stats->traversal_ms = trav_ms;
+    stats->blocks = blocks; stats->warps_per_block = warps;
+    stats->n_visited = nv; stats->m_visited = mv;
+    stats->claims = (int64_t)counters[kCntClaims];
+    stats->failed_claims = (int64_t)counters[kCntFailedClaims];
+    stats->flushes = (int64_t)counters[kCntFlushes];
+    stats->refills = (int64_t)counters[kCntRefills];
+    stats->intra_steals = (int64_t)counters[kCntIntraSteals];
+    stats->inter_steals = (int64_t)counters[kCntInterSteals];
+    stats->steal_attempts = (int64_t)counters[kCntStealAttempts];
+    stats->chunks_allocated = (int64_t)counters[kCntChunks];
+    stats->windows = (int64_t)counters[kCntWindows];
+    stats->idle_ns = (int64_t)counters[kCntIdleNs];
+    stats->inter_scans = (int64_t)counters[kCntInterScans];
+    stats->spills = (int64_t)counters[kCntSpills];
+    stats->cyc_window = (int64_t)counters[kCntTWin];
+    stats->cyc_probe = (int64_t)counters[kCntTProbe];
+    stats->cyc_claim = (int64_t)counters[kCntTClaim];
+    stats->cyc_tail = (int64_t)counters[kCntTTail];
+}
+
+// per-root count buffer (2 x u64 per root) for stats calls
+static int ensure_counts(dfs_graph* g, int32_t k) {
+    if (g->counts_cap >= k) return DFS_OK;
+    cudaFree(g->d_counts);
+    g->d_counts = nullptr; g->counts_cap = 0;
+    if (cudaMalloc(&g->d_counts, (size_t)k * 2 * sizeof(unsigned long long)) != cudaSuccess) {
+        cudaGetLastError();
+        return DFS_ENOMEM;
+    }
+    g->counts_cap = k;
+    return DFS_OK;
+}
+
+// copy the per-root counts out (and total them)
+static int finish_counts(dfs_graph* g, int32_t k, dfs_stats* stats, int64_t& nv, int64_t& mv) {
+    std::vector<unsigned long long> h((size_t)k * 2);
+    if (cudaMemcpy(h.data(), g->d_counts, h.size() * sizeof(unsigned long long), cudaMemcpyDeviceToHost) != cudaSuccess) {
+        cudaGetLastError();
+        return DFS_ECUDA;
+    }
+    nv = mv = 0;
+    for (int32_t q = 0; q < k; ++q) {
+        nv += (int64_t)h[2 * q]; mv += (int64_t)h[2 * q + 1];
+        if (stats->root_counts) { stats->root_counts[2 * q] = (int64_t)h[2 * q]; stats->root_counts[2 * q + 1] = (int64_t)h[2 * q + 1]; }
+    }
+    return DFS_OK;
+}
+
+// sequential path: one slot, cooperative launch, per-traversal status check and stats
+static int run_sequential(dfs_graph* g, const int32_t* roots, int32_t k, int32_t* out, bool out_dev,
+                          const dfs_options& o, int blocks, int warps, dfs_stats* stats) {
+    Slot& sl = g->slots[0];
+    if (!out_dev && !sl.parent) {
+        if (cudaMalloc(&sl.parent, (size_t)g->n * sizeof(int32_t)) != cudaSuccess) {
             cudaGetLastError();
             return fail(DFS_ENOMEM);
         }
@@ -382,71 +480,145 @@ static int run_many(dfs_graph* g, const int32_t* roots_host, int32_t k, int32_t*
     unsigned long long counters[kNumCounters] = {0};
     float total_ms = 0.f, trav_ms = 0.f;
     int64_t nv = 0, mv = 0;
-    for (int32_t q = 0; q < k; ++q) {
-        int32_t* d_out = out_dev ? out + (size_t)q * g->n : g->d_parent;
-        cudaEventRecord(g->ev0, g->stream);
-        rc = launch_one(g, roots_host[q], d_out, o, blocks, warps, stats != nullptr);
+    cudaStream_t s = g->stream;
+    if (stats) {
+        const int rc = ensure_counts(g, k);
         if (rc != DFS_OK) return fail(rc);
-        cudaEventRecord(g->ev1, g->stream);
+        cudaMemsetAsync(g->d_counts, 0, (size_t)k * 2 * sizeof(unsigned long long), s);
+    }
+    for (int32_t q = 0; q < k; ++q) {
+        int32_t* d_out = out_dev ? out + (size_t)q * g->n : sl.parent;
+        cudaMemsetAsync(sl.status, 0, sizeof(int), s);
+        cudaEventRecord(sl.ev0, s);
+        int rc = launch_one(g, sl, s, roots[q], d_out, o, blocks, warps, stats != nullptr, true);
+        if (rc != DFS_OK) return fail(rc);
+        cudaEventRecord(sl.ev1, s);
         if (stats) {
-            cudaMemsetAsync(g->d_count2, 0, 2 * sizeof(unsigned long long), g->stream);
-            dfs_count_kernel<<<g->sms * 4, 256, 0, g->stream>>>(g->d_bitmap, g->d_rp, (uint32_t)g->n, g->d_count2);
+            dfs_count_kernel<<<g->sms * 4, 256, 0, s>>>(sl.bitmap, g->d_rp, (uint32_t)g->n, g->d_counts + 2 * q);
             g->launches++;
         }
         Ctl h;
-        if (cudaMemcpyAsync(&h, g->d_ctl, sizeof(Ctl), cudaMemcpyDeviceToHost, g->stream) != cudaSuccess ||
-            cudaStreamSynchronize(g->stream) != cudaSuccess) {
+        if (cudaMemcpyAsync(&h, sl.ctl, sizeof(Ctl), cudaMemcpyDeviceToHost, s) != cudaSuccess ||
+            cudaStreamSynchronize(s) != cudaSuccess) {
             cudaGetLastError();
             return fail(DFS_ECUDA);
         }
-        if (h.status != 0) { g->tab_dirty = true; return fail(h.status); }
+        if (h.status != 0) { sl.tab_dirty = true; return fail(h.status); }
         if (!out_dev) {
-            if (cudaMemcpyAsync(out + (size_t)q * g->n, g->d_parent, (size_t)g->n * sizeof(int32_t),
-                                cudaMemcpyDeviceToHost, g->stream) != cudaSuccess) {
+            if (cudaMemcpyAsync(out + (size_t)q * g->n, sl.parent, (size_t)g->n * sizeof(int32_t),
+                                cudaMemcpyDeviceToHost, s) != cudaSuccess) {
                 cudaGetLastError();
                 return fail(DFS_ECUDA);
             }
         }
         if (stats) {
             float ms = 0.f, kms = 0.f;
-            cudaEventElapsedTime(&ms, g->ev0, g->ev1);
-            cudaEventElapsedTime(&kms, g->evk0, g->evk1);
+            cudaEventElapsedTime(&ms, sl.ev0, sl.ev1);
+            cudaEventElapsedTime(&kms, sl.evk0, sl.evk1);
             total_ms += ms;
             trav_ms += kms;
             for (int c = 0; c < kNumCounters; ++c) counters[c] += h.counters[c];
-            {
-                unsigned long long c2[2];
-                cudaMemcpyAsync(c2, g->d_count2, sizeof(c2), cudaMemcpyDeviceToHost, g->stream);
-                cudaStreamSynchronize(g->stream);
-                nv += (int64_t)c2[0]; mv += (int64_t)c2[1];
+        }
+    }
+    if (cudaStreamSynchronize(s) != cudaSuccess) { cudaGetLastError(); return fail(DFS_ECUDA); }
+    if (stats) {
+        const int rc = finish_counts(g, k, stats, nv, mv);
+        if (rc != DFS_OK) return fail(rc);
+        fill_stats(stats, blocks, warps, total_ms, trav_ms, nv, mv, counters);
+    }
+    return DFS_OK;
+}
+
+// concurrent path (§8(f)-2): `conc` slots, each on its own stream and a 1/conc share of the
+// SMs, take roots round-robin; no host synchronisation until the whole batch is issued
+static int run_concurrent(dfs_graph* g, const int32_t* roots, int32_t k, int32_t* out, bool out_dev,
+                          const dfs_options& o, int blocks, int warps, int conc, dfs_stats* stats) {
+    for (int c = 0; c < conc; ++c) {
+        int rc = ensure_slot(g, c);
+        if (rc != DFS_OK) return fail(rc);
+        Slot& sl = g->slots[c];
+        if (!out_dev && !sl.parent) {
+            if (cudaMalloc(&sl.parent, (size_t)g->n * sizeof(int32_t)) != cudaSuccess) {
+                cudaGetLastError();
+                return fail(DFS_ENOMEM);
             }
         }
     }
-    if (cudaStreamSynchronize(g->stream) != cudaSuccess) { cudaGetLastError(); return fail(DFS_ECUDA); }
+    // fork: every slot stream waits for the handle's stream; slot 0 gets its own stream too
+    cudaStream_t base = g->stream;
     if (stats) {
-        std::memset(stats, 0, sizeof(*stats));
-        stats->kernel_ms = total_ms;
-        stats->traversal_ms = trav_ms;
-        stats->blocks = blocks; stats->warps_per_block = warps;
-        stats->n_visited = nv; stats->m_visited = mv;
-        stats->claims = (int64_t)counters[kCntClaims];
-        stats->failed_claims = (int64_t)counters[kCntFailedClaims];
-        stats->flushes = (int64_t)counters[kCntFlushes];
-        stats->refills = (int64_t)counters[kCntRefills];
-        stats->intra_steals = (int64_t)counters[kCntIntraSteals];
-        stats->inter_steals = (int64_t)counters[kCntInterSteals];
-        stats->steal_attempts = (int64_t)counters[kCntStealAttempts];
-        stats->chunks_allocated = (int64_t)counters[kCntChunks];
-        stats->windows = (int64_t)counters[kCntWindows];
-        stats->idle_ns = (int64_t)counters[kCntIdleNs];
-        stats->inter_scans = (int64_t)counters[kCntInterScans];
-        stats->spills = (int64_t)counters[kCntSpills];
-        stats->cyc_window = (int64_t)counters[kCntTWin];
-        stats->cyc_probe = (int64_t)counters[kCntTProbe];
-        stats->cyc_claim = (int64_t)counters[kCntTClaim];
-        stats->cyc_tail = (int64_t)counters[kCntTTail];
+        const int rc = ensure_counts(g, k);
+        if (rc != DFS_OK) return fail(rc);
+        cudaMemsetAsync(g->d_counts, 0, (size_t)k * 2 * sizeof(unsigned long long), base);
+    }
+    if (!g->slots[0].stream && cudaStreamCreateWithFlags(&g->slots[0].stream, cudaStreamNonBlocking) != cudaSuccess) {
+        cudaGetLastError();
+        return fail(DFS_ECUDA);
+    }
+    Slot& s0 = g->slots[0];
+    cudaEventRecord(s0.ev0, base);
+    for (int c = 0; c < conc; ++c) {
+        Slot& sl = g->slots[c];
+        cudaStreamWaitEvent(sl.stream, s0.ev0, 0);
+        cudaMemsetAsync(sl.status, 0, sizeof(int), sl.stream);
+        cudaMemsetAsync(sl.count2, 0, 2 * sizeof(unsigned long long), sl.stream);
+    }
+    for (int32_t q = 0; q < k; ++q) {
+        Slot& sl = g->slots[q % conc];
+        int32_t* d_out = out_dev ? out + (size_t)q * g->n : sl.parent;
+        int rc = launch_one(g, sl, sl.stream, roots[q], d_out, o, blocks, warps, false, false);
+        if (rc != DFS_OK) return fail(rc);
+        if (stats) {
+            dfs_count_kernel<<<g->sms * 4, 256, 0, sl.stream>>>(sl.bitmap, g->d_rp, (uint32_t)g->n, g->d_counts + 2 * q);
+            g->launches++;
+        }
+        if (!out_dev) {
+            if (cudaMemcpyAsync(out + (size_t)q * g->n, sl.parent, (size_t)g->n * sizeof(int32_t),
+                                cudaMemcpyDeviceToHost, sl.stream) != cudaSuccess) {
+                cudaGetLastError();
+                return fail(DFS_ECUDA);
+            }
+        }
+    }
+    // join
+    for (int c = 0; c < conc; ++c) {
+        Slot& sl = g->slots[c];
+        cudaEventRecord(sl.ev1, sl.stream);
+        cudaStreamWaitEvent(base, sl.ev1, 0);
+    }
+    cudaEventRecord(s0.evk1, base);
+    if (cudaStreamSynchronize(base) != cudaSuccess) { cudaGetLastError(); return fail(DFS_ECUDA); }
+    int worst = 0;
+    int64_t nv = 0, mv = 0;
+    for (int c = 0; c < conc; ++c) {
+        Slot& sl = g->slots[c];
+        int st = 0;
+        cudaMemcpy(&st, sl.status, sizeof(int), cudaMemcpyDeviceToHost);
+        if (st != 0) { sl.tab_dirty = true; worst = std::min(worst, st); }
+    }
+    if (cudaGetLastError() != cudaSuccess) return fail(DFS_ECUDA);
+    if (worst != 0) return fail(worst);
+    if (stats) {
+        const int rc = finish_counts(g, k, stats, nv, mv);
+        if (rc != DFS_OK) return fail(rc);
+        float ms = 0.f;
+        cudaEventElapsedTime(&ms, s0.ev0, s0.evk1);
+        unsigned long long counters[kNumCounters] = {0};
+        fill_stats(stats, blocks, warps, ms, ms, nv, mv, counters);
     }
     return DFS_OK;
+}
+
+static int run_many(dfs_graph* g, const int32_t* roots_host, int32_t k, int32_t* out, bool out_dev,
+                    const dfs_options* opt, dfs_stats* stats) {
+    dfs_options o;
+    int blocks = 0, warps = 0, conc = 1;
+    int rc = resolve_options(g, opt, k, o, blocks, warps, conc);
+    if (rc != DFS_OK) return fail(rc);
+    for (int32_t q = 0; q < k; ++q)
+        if (roots_host[q] < 0 || roots_host[q] >= g->n) return fail(DFS_EINVAL);
+    if (conc <= 1) return run_sequential(g, roots_host, k, out, out_dev, o, blocks, warps, stats);
+    return run_concurrent(g, roots_host, k, out, out_dev, o, blocks, warps, conc, stats);
 }
 
 extern "C" {

@@ -47,7 +47,7 @@ class _Options(ctypes.Structure):
                 ("backoff_max_ns", ctypes.c_int32), ("window", ctypes.c_int32),
                 ("pub_batch", ctypes.c_int32), ("speculate", ctypes.c_int32),
                 ("steal_half", ctypes.c_int32), ("probe_mode", ctypes.c_int32),
-                ("reserved", ctypes.c_int32 * 2)]
+                ("concurrency", ctypes.c_int32), ("reserved", ctypes.c_int32 * 1)]
 
 
 class _Stats(ctypes.Structure):
@@ -61,7 +61,8 @@ class _Stats(ctypes.Structure):
                 ("windows", ctypes.c_int64), ("idle_ns", ctypes.c_int64),
                 ("inter_scans", ctypes.c_int64), ("spills", ctypes.c_int64),
                 ("cyc_window", ctypes.c_int64), ("cyc_probe", ctypes.c_int64),
-                ("cyc_claim", ctypes.c_int64), ("cyc_tail", ctypes.c_int64)]
+                ("cyc_claim", ctypes.c_int64), ("cyc_tail", ctypes.c_int64),
+                ("root_counts", ctypes.c_void_p)]
 
 
 @dataclass
@@ -87,6 +88,7 @@ class Options:
     speculate: Optional[int] = None
     steal_half: Optional[bool] = None
     probe_mode: Optional[int] = None
+    concurrency: Optional[int] = None
 
     def to_c(self) -> _Options:
         o = _Options()
@@ -122,6 +124,7 @@ class Stats:
     cyc_probe: int
     cyc_claim: int
     cyc_tail: int
+    root_counts: Optional[np.ndarray] = None
 
 
 _lib = None
@@ -168,6 +171,11 @@ def load_library():
         lib.dfs_strerror.restype = ctypes.c_char_p
         _lib = lib
     return _lib
+
+
+def _stats(st, counts=None) -> "Stats":
+    d = {f[0]: getattr(st, f[0]) for f in _Stats._fields_ if f[0] != "root_counts"}
+    return Stats(root_counts=counts, **d)
 
 
 def _strerror(code: int) -> str:
@@ -255,7 +263,7 @@ class Graph:
         if rc != 0:
             raise DfsError(rc, "dfs_run_ex")
         if stats:
-            return out, Stats(**{f[0]: getattr(st, f[0]) for f in _Stats._fields_})
+            return out, _stats(st)
         return out
 
     def run_batch(self, roots, out=None, options: Optional[Options] = None, stats: bool = False):
@@ -270,6 +278,9 @@ class Graph:
         self._stream()
         o = self._opts(options, stats)
         st = _Stats() if stats else None
+        counts = np.zeros(2 * k, dtype=np.int64) if stats else None
+        if stats:
+            st.root_counts = counts.ctypes.data
         rr = r.contiguous()
         rc = self._lib.dfs_run_batch_ex(self._h, rr.data_ptr(), k, out.data_ptr(),
                                         ctypes.byref(o) if o is not None else None,
@@ -277,7 +288,7 @@ class Graph:
         if rc != 0:
             raise DfsError(rc, "dfs_run_batch_ex")
         if stats:
-            return out, Stats(**{f[0]: getattr(st, f[0]) for f in _Stats._fields_})
+            return out, _stats(st, counts.reshape(k, 2))
         return out
 
     def timeline(self, len_: int = 0, dt_ns: int = 10_000, fetch: bool = False):

@@ -240,3 +240,28 @@ def test_stream_and_repeat_consistency():
         for p, v in zip(ps, vis):
             assert np.array_equal(v, vis[0])
             _valid(g, r, p)
+
+
+@pytest.mark.parametrize("conc", [2, 3, 4])
+def test_concurrent_batch(conc):
+    """§8(f)-2: K traversals at once on K slots / streams / SM shares; every row valid."""
+    g = graphgen.road(400, 300, seed=9)
+    roots = graphgen.random_roots(g, 7, seed=conc)
+    with Graph(g.row_ptr, g.col_idx) as G:
+        out, st = G.run_batch(roots, options=Options(concurrency=conc), stats=True)
+        tot_v = 0
+        for q, r in enumerate(roots):
+            res = _valid(g, int(r), out[q])
+            tot_v += res.n_visited
+            assert tuple(st.root_counts[q]) == (res.n_visited, res.m_visited)
+        assert st.n_visited == tot_v
+        hb = torch.empty((len(roots), g.n), dtype=torch.int32)
+        G.run_batch(roots, out=hb, options=Options(concurrency=conc, hot_cutoff=4, window=128))
+        for q, r in enumerate(roots):
+            _valid(g, int(r), hb[q].numpy())
+        # deterministic ignores concurrency and stays bit-exact
+        d = G.run_batch(roots[:3], options=Options(concurrency=conc, deterministic=True))
+        for q, r in enumerate(roots[:3]):
+            _exact(g, int(r), d[q])
+        with pytest.raises(DfsError):
+            G.run_batch(roots, options=Options(concurrency=conc, blocks=148))   # blocks*conc > SMs
