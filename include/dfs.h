@@ -116,7 +116,9 @@ typedef struct dfs_options {
                                 §8(f)-2); 0 = auto (4, capped by the number of roots; a single
                                 dfs_run is always 1).  Slots beyond the first allocate their
                                 scratch on first use.                                              */
-    int32_t reserved[1];
+    int32_t prefetch;        /* 1: L2-prefetch every probed candidate's first adjacency window */
+    int32_t ring_cap;        /* usable HotRing entries (0 = all 256); 2 makes every push spill: the
+                                "one-level stack" of the paper's v1 (Fig 8)            */
 } dfs_options;
 
 typedef struct dfs_stats {
@@ -134,9 +136,14 @@ typedef struct dfs_stats {
     /* SM-cycle breakdown of the expansion step summed over windows (collect_stats; diagnostics):
        wait for the window data, wait for the probes, wait for the speculative claim, rest */
     int64_t cyc_window, cyc_probe, cyc_claim, cyc_tail;
+    int64_t cyc_outside;     /* cycles between consecutive expansion steps of a busy warp (pops,
+                                flushes, spills, periodic checks)                                  */
     /* optional, caller-owned host array of 2*num_roots int64 (NULL = not wanted): per-root
        (n_visited, m_visited) of a batch, in root order */
     int64_t *root_counts;
+    /* optional, caller-owned host array of `blocks` int64 (NULL = not wanted; single traversals):
+       claims (tree vertices discovered) per block — the task distribution of Fig 9 */
+    int64_t *block_claims;
 } dfs_stats;
 
 void dfs_options_default(dfs_options *opt);

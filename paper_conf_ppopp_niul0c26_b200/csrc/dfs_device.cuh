@@ -55,13 +55,13 @@ struct Ctl {
     int status;                        // 0 or a negative dfs_status
     unsigned int pool_bump;            // bump allocator over the chunk pool
     unsigned long long free_head;      // tagged free-stack head: (tag << 32) | chunk id
-    unsigned long long counters[16];   // stats (collect_stats)
+    unsigned long long counters[24];   // stats (collect_stats)
 };
 
 enum CounterIdx {
     kCntClaims = 0, kCntFailedClaims, kCntFlushes, kCntRefills, kCntIntraSteals, kCntInterSteals,
     kCntStealAttempts, kCntChunks, kCntWindows, kCntIdleNs, kCntInterScans, kCntSpills,
-    kCntTWin, kCntTProbe, kCntTClaim, kCntTTail, kNumCounters
+    kCntTWin, kCntTProbe, kCntTClaim, kCntTTail, kCntTOut, kCntOutIters, kNumCounters
 };
 
 struct KParams {
@@ -96,6 +96,9 @@ struct KParams {
     int speculate;                           // speculative claim of the child's first neighbour
     int steal_half;                          // steal max(h_s, rest/2) (resp. c_s) entries
     int probe_mode;                          // 0: L2 (.cg) probes; 1: L1-cached probes; 2: .relaxed.gpu
+    int prefetch;                            // L2-prefetch every candidate's first window
+    uint32_t ring_cap;                       // usable HotRing entries (<= H); 2 ~ one-level stack (v1)
+    unsigned long long* block_claims;        // optional: claims per block (Fig 9 task counts)
 };
 
 // ------------------------------------------------------------------------------------------
@@ -193,8 +196,7 @@ struct SmemCtl {
     unsigned int warp_mask;                // 1 = warp active
     volatile int done;                     // block-local copy of ctl->done
     uint32_t inter_token;                  // one idle warp per block scans other blocks at a time
-    unsigned long long cnt[kMaxWarps][16]; // per-warp stats counters (collect_stats)
-    static_assert(kNumCounters <= 16, "counter slots");
+    unsigned long long cnt[kMaxWarps][kNumCounters]; // per-warp stats counters (collect_stats)
 };
 
 __device__ __forceinline__ void smem_lock(uint32_t* l) {
@@ -256,7 +258,7 @@ __global__ void __launch_bounds__(32 * WMAX, 1) dfs_persistent_kernel(const KPar
     static_assert(VEC == 1 || VEC == 4, "VEC is 1 or 4");
     constexpr uint32_t kBatch = H / 2;              // flush batch (reading S10)
     constexpr uint32_t kWin = 32u * VEC;            // positions per window
-    constexpr int kHeadLanes = 8;                   // lanes fetched before a window's end is known
+    constexpr int kHeadLanes = VEC == 1 ? 8 : 16;   // lanes fetched before a window's end is known
     extern __shared__ __align__(16) unsigned char smem_raw[];
     SmemCtl& S = *reinterpret_cast<SmemCtl*>(smem_raw);
     constexpr int kCtlBytes = (sizeof(SmemCtl) + 15) & ~15;
@@ -277,7 +279,7 @@ __global__ void __launch_bounds__(32 * WMAX, 1) dfs_persistent_kernel(const KPar
     }
     if (threadIdx.x == 0) { S.warp_mask = (blockIdx.x == 0) ? 1u : 0u; S.done = 0; S.inter_token = 0; }
     unsigned long long* const cnt = S.cnt[w];     // lane 0 updates its warp's counters
-    if (STATS && lane < 16) cnt[lane] = 0;
+    if (STATS && lane < kNumCounters) cnt[lane] = 0;
     __syncthreads();
 
     // ---- per-warp state (warp-uniform registers) ----
@@ -301,7 +303,9 @@ __global__ void __launch_bounds__(32 * WMAX, 1) dfs_persistent_kernel(const KPar
     if (rng == 0) rng = 1;
     const unsigned long long t_start = globaltimer();
     unsigned long long t_idle0 = 0;
+    long long tc_prev = 0;                       // STATS: end of the previous expansion step
     uint32_t iter = 0;
+    unsigned long long my_claims = 0;            // for P.block_claims (Fig 9 task distribution)
 
     if (blockIdx.x == 0 && w == 0) {
         // Alg 1 l.1-3: root claimed by the reset kernel; <root, row_ptr[root]> is our top
@@ -419,9 +423,9 @@ __global__ void __launch_bounds__(32 * WMAX, 1) dfs_persistent_kernel(const KPar
     // push <v, idx> at head (Fig 2(c)); flushes first when full
     auto push = [&](uint32_t v, uint32_t idx) -> bool {
         int full = 0;
-        if (lane == 0) full = ((my_head - S.tailf[w]) & 0xFFFFu) >= (uint32_t)H;
+        if (lane == 0) full = ((my_head - S.tailf[w]) & 0xFFFFu) >= P.ring_cap;
         if (__shfl_sync(kFull, full, 0)) {
-            if (!flush(kBatch, 0u)) return false;
+            if (!flush(P.ring_cap >= 2u ? P.ring_cap / 2u : 1u, 0u)) return false;
         }
         if (lane == 0) ring[my_head & (H - 1)] = pack_entry(v, idx);
         ++my_head;
@@ -554,7 +558,11 @@ __global__ void __launch_bounds__(32 * WMAX, 1) dfs_persistent_kernel(const KPar
             }
             if (STATS && lane == 0) ++cnt[kCntWindows];
             long long tc0 = 0, tc1 = 0;
-            if (STATS) { tc0 = clock_after(0u); tc1 = clock_after((uint32_t)nbv[0] ^ end); }
+            if (STATS) {
+                tc0 = clock_after(0u);
+                if (lane == 0 && tc_prev) { cnt[kCntTOut] += tc0 - tc_prev; ++cnt[kCntOutIters]; }
+                tc1 = clock_after((uint32_t)nbv[0] ^ end);
+            }
             const uint32_t a = i & ~(uint32_t)(VEC - 1);
             const uint32_t q0 = a + (uint32_t)VEC * lane;
             // long list (hubs): load the next window now so it is in flight while this window's
@@ -604,6 +612,9 @@ __global__ void __launch_bounds__(32 * WMAX, 1) dfs_persistent_kernel(const KPar
                     const uint32_t* wp = P.bitmap + ((uint32_t)x >> 5);
                     const uint32_t word = P.probe_mode == 1 ? *wp
                                         : P.probe_mode == 2 ? ld_relaxed_u32(wp) : __ldcg(wp);
+                    // a candidate's adjacency window will be loaded if it is claimed (by this
+                    // warp now or by whoever reaches it later): start moving it into L2 now
+                    if (P.prefetch) asm volatile("prefetch.global.L2 [%0];" ::"l"(P.adj + rsv[e]));
                     if (!((word >> (x & 31)) & 1u)) m4 |= 1u << e;
                 }
             }
@@ -617,6 +628,7 @@ __global__ void __launch_bounds__(32 * WMAX, 1) dfs_persistent_kernel(const KPar
             // candidate, or past the window.
             auto descend = [&](int k, int e, uint32_t v, uint32_t vrs, uint32_t vre) -> bool {
                 if (STATS && lane == 0) ++cnt[kCntClaims];
+                ++my_claims;
                 if (lane == 0) P.parent[v] = (int32_t)u;                            // Alg 1 l.10
                 const uint32_t mine = (lane == k) ? (m4 & ~((2u << e) - 1u)) : (lane > k ? m4 : 0u);
                 const uint32_t later = __ballot_sync(kFull, mine != 0);
@@ -679,6 +691,7 @@ __global__ void __launch_bounds__(32 * WMAX, 1) dfs_persistent_kernel(const KPar
                 const long long tc4 = clock_after((uint32_t)nbv[0] ^ i);
                 cnt[kCntTWin] += tc1 - tc0; cnt[kCntTProbe] += tc2 - tc1;
                 cnt[kCntTClaim] += tc3 - tc2; cnt[kCntTTail] += tc4 - tc3;
+                tc_prev = tc4;
             }
             if (!descended) {
                 i = a + kWin;
@@ -743,6 +756,7 @@ __global__ void __launch_bounds__(32 * WMAX, 1) dfs_persistent_kernel(const KPar
         }
         bool got_work = false;
         uint32_t backoff = 32;
+        tc_prev = 0;
         t_idle0 = STATS ? globaltimer() : 0ull;
         while (!got_work) {
             if (__shfl_sync(kFull, S.done, 0)) goto exit_loop;
@@ -954,7 +968,8 @@ exit_loop:
             if (ld_relaxed_u32(slot) != kEmptySlot) st_relaxed_u32(slot, kEmptySlot);
         }
     }
-    if (STATS) {
+    if (P.block_claims && lane == 0 && my_claims) atomicAdd(&P.block_claims[blockIdx.x], my_claims);
+    if (STATS && (P.collect_stats != 2 || gw == 0)) {     // 2: the root warp's counters only
 #pragma unroll
         for (int k = 0; k < kNumCounters; ++k)
             if (lane == 0 && cnt[k]) atomicAdd(&P.ctl->counters[k], cnt[k]);
@@ -985,7 +1000,7 @@ __global__ void dfs_reset_kernel(uint32_t* bitmap, uint32_t nwords, unsigned lon
         ctl->status = 0;
         ctl->pool_bump = 0u;
         ctl->free_head = (unsigned long long)kEmptySlot;
-        for (int k = 0; k < 16; ++k) ctl->counters[k] = 0ull;
+        for (int k = 0; k < 24; ++k) ctl->counters[k] = 0ull;
     }
 }
 

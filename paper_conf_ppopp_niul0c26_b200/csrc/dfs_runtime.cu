@@ -63,6 +63,7 @@ struct Slot {
     Ctl* ctl = nullptr;
     unsigned long long* count2 = nullptr;   // visited count, TEPS numerator (summed over a batch)
     int* status = nullptr;                  // worst status over the slot's traversals in a batch
+    unsigned long long* block_claims = nullptr;   // per-block claim counts (stats), else null
     size_t tab_words = 0;
     uint32_t n_chunks = 0;
     bool tab_dirty = false;
@@ -92,7 +93,7 @@ struct dfs_graph {
 static void free_slot(Slot& s) {
     cudaFree(s.bitmap); cudaFree(s.parent); cudaFree(s.cold_tb); cudaFree(s.tab); cudaFree(s.pool);
     cudaFree(s.consumed); cudaFree(s.next); cudaFree(s.block_cold); cudaFree(s.ctl); cudaFree(s.count2);
-    cudaFree(s.status);
+    cudaFree(s.status); cudaFree(s.block_claims);
     if (s.stream) cudaStreamDestroy(s.stream);
     if (s.ev0) cudaEventDestroy(s.ev0);
     if (s.ev1) cudaEventDestroy(s.ev1);
@@ -173,6 +174,8 @@ void dfs_options_default(dfs_options* o) {
     o->steal_half = 1;
     o->probe_mode = 0;
     o->concurrency = 0;
+    o->prefetch = 0;
+    o->ring_cap = 0;
 }
 
 int dfs_last_error(void) { return g_last_error; }
@@ -353,6 +356,9 @@ static int launch_one(dfs_graph* g, Slot& sl, cudaStream_t s, int32_t root, int3
     P.speculate = o.speculate;
     P.steal_half = o.steal_half;
     P.probe_mode = o.probe_mode;
+    P.prefetch = o.prefetch;
+    P.ring_cap = (o.ring_cap > 0 && o.ring_cap < kRing) ? (uint32_t)o.ring_cap : (uint32_t)kRing;
+    P.block_claims = sl.block_claims;
     const bool tl = g->d_timeline && &sl == &g->slots[0];
     P.timeline = tl ? g->d_timeline : nullptr;
     P.timeline_len = tl ? g->timeline_len : 0;
@@ -437,6 +443,7 @@ static void fill_stats(dfs_stats* stats, int blocks, int warps, float total_ms, 
     stats->cyc_probe = (int64_t)counters[kCntTProbe];
     stats->cyc_claim = (int64_t)counters[kCntTClaim];
     stats->cyc_tail = (int64_t)counters[kCntTTail];
+    stats->cyc_outside = (int64_t)counters[kCntTOut];
 }
 
 // per-root count buffer (2 x u64 per root) for stats calls
@@ -486,6 +493,17 @@ static int run_sequential(dfs_graph* g, const int32_t* roots, int32_t k, int32_t
         if (rc != DFS_OK) return fail(rc);
         cudaMemsetAsync(g->d_counts, 0, (size_t)k * 2 * sizeof(unsigned long long), s);
     }
+    const bool want_blocks = stats && stats->block_claims;
+    if (want_blocks) {
+        if (!sl.block_claims && cudaMalloc(&sl.block_claims, (size_t)g->max_blocks * sizeof(unsigned long long)) != cudaSuccess) {
+            cudaGetLastError();
+            return fail(DFS_ENOMEM);
+        }
+        cudaMemsetAsync(sl.block_claims, 0, (size_t)g->max_blocks * sizeof(unsigned long long), s);
+    } else if (sl.block_claims) {
+        cudaFree(sl.block_claims);           // launch_one passes it to the kernel when non-null
+        sl.block_claims = nullptr;
+    }
     for (int32_t q = 0; q < k; ++q) {
         int32_t* d_out = out_dev ? out + (size_t)q * g->n : sl.parent;
         cudaMemsetAsync(sl.status, 0, sizeof(int), s);
@@ -524,7 +542,14 @@ static int run_sequential(dfs_graph* g, const int32_t* roots, int32_t k, int32_t
     if (stats) {
         const int rc = finish_counts(g, k, stats, nv, mv);
         if (rc != DFS_OK) return fail(rc);
+        int64_t* bc = stats->block_claims;
         fill_stats(stats, blocks, warps, total_ms, trav_ms, nv, mv, counters);
+        stats->block_claims = bc;
+        if (bc) {
+            std::vector<unsigned long long> h((size_t)blocks);
+            cudaMemcpy(h.data(), sl.block_claims, h.size() * sizeof(unsigned long long), cudaMemcpyDeviceToHost);
+            for (int b = 0; b < blocks; ++b) bc[b] = (int64_t)h[(size_t)b];
+        }
     }
     return DFS_OK;
 }
@@ -537,6 +562,7 @@ static int run_concurrent(dfs_graph* g, const int32_t* roots, int32_t k, int32_t
         int rc = ensure_slot(g, c);
         if (rc != DFS_OK) return fail(rc);
         Slot& sl = g->slots[c];
+        if (sl.block_claims) { cudaFree(sl.block_claims); sl.block_claims = nullptr; }
         if (!out_dev && !sl.parent) {
             if (cudaMalloc(&sl.parent, (size_t)g->n * sizeof(int32_t)) != cudaSuccess) {
                 cudaGetLastError();

@@ -47,7 +47,8 @@ class _Options(ctypes.Structure):
                 ("backoff_max_ns", ctypes.c_int32), ("window", ctypes.c_int32),
                 ("pub_batch", ctypes.c_int32), ("speculate", ctypes.c_int32),
                 ("steal_half", ctypes.c_int32), ("probe_mode", ctypes.c_int32),
-                ("concurrency", ctypes.c_int32), ("reserved", ctypes.c_int32 * 1)]
+                ("concurrency", ctypes.c_int32), ("prefetch", ctypes.c_int32),
+                ("ring_cap", ctypes.c_int32)]
 
 
 class _Stats(ctypes.Structure):
@@ -62,7 +63,8 @@ class _Stats(ctypes.Structure):
                 ("inter_scans", ctypes.c_int64), ("spills", ctypes.c_int64),
                 ("cyc_window", ctypes.c_int64), ("cyc_probe", ctypes.c_int64),
                 ("cyc_claim", ctypes.c_int64), ("cyc_tail", ctypes.c_int64),
-                ("root_counts", ctypes.c_void_p)]
+                ("cyc_outside", ctypes.c_int64), ("root_counts", ctypes.c_void_p),
+                ("block_claims", ctypes.c_void_p)]
 
 
 @dataclass
@@ -89,6 +91,8 @@ class Options:
     steal_half: Optional[bool] = None
     probe_mode: Optional[int] = None
     concurrency: Optional[int] = None
+    prefetch: Optional[bool] = None
+    ring_cap: Optional[int] = None
 
     def to_c(self) -> _Options:
         o = _Options()
@@ -124,7 +128,9 @@ class Stats:
     cyc_probe: int
     cyc_claim: int
     cyc_tail: int
+    cyc_outside: int
     root_counts: Optional[np.ndarray] = None
+    block_claims: Optional[np.ndarray] = None
 
 
 _lib = None
@@ -173,9 +179,11 @@ def load_library():
     return _lib
 
 
-def _stats(st, counts=None) -> "Stats":
-    d = {f[0]: getattr(st, f[0]) for f in _Stats._fields_ if f[0] != "root_counts"}
-    return Stats(root_counts=counts, **d)
+def _stats(st, counts=None, blocks=None) -> "Stats":
+    d = {f[0]: getattr(st, f[0]) for f in _Stats._fields_ if f[0] not in ("root_counts", "block_claims")}
+    if blocks is not None:
+        blocks = blocks[:st.blocks].copy()
+    return Stats(root_counts=counts, block_claims=blocks, **d)
 
 
 def _strerror(code: int) -> str:
@@ -247,7 +255,8 @@ class Graph:
         return options.to_c()
 
     # -- API ----------------------------------------------------------------------------
-    def run(self, root: int, out=None, options: Optional[Options] = None, stats: bool = False):
+    def run(self, root: int, out=None, options: Optional[Options] = None, stats: bool = False,
+            block_claims: bool = False):
         """One unordered DFS from ``root`` (``dfs_run_ex``).  Returns the int32 parent tensor
         (``out`` if given; host or device) and, with ``stats=True``, a :class:`Stats`."""
         import torch
@@ -257,13 +266,17 @@ class Graph:
         self._stream()
         o = self._opts(options, stats)
         st = _Stats() if stats else None
+        bc = None
+        if stats and block_claims:
+            bc = np.zeros(1024, dtype=np.int64)
+            st.block_claims = bc.ctypes.data
         rc = self._lib.dfs_run_ex(self._h, int(root), out.data_ptr(),
                                   ctypes.byref(o) if o is not None else None,
                                   ctypes.byref(st) if st is not None else None)
         if rc != 0:
             raise DfsError(rc, "dfs_run_ex")
         if stats:
-            return out, _stats(st)
+            return out, _stats(st, blocks=bc)
         return out
 
     def run_batch(self, roots, out=None, options: Optional[Options] = None, stats: bool = False):

@@ -96,6 +96,16 @@ VARIANTS = {
     "p1": dict(probe_mode=1),
     "p2": dict(probe_mode=2),
     "p1nospec": dict(probe_mode=1, speculate=0),
+    "pf": dict(prefetch=True),
+    "pfp1": dict(prefetch=True, probe_mode=1),
+    "nospill": dict(spill=False),
+    "b37": dict(blocks=37),
+    "b16": dict(blocks=16),
+    "h4c4": dict(hot_cutoff=4, cold_cutoff=4),
+    "pb8": dict(pub_batch=8),
+    "w0": dict(collect_stats=2),
+    "w0nospill": dict(collect_stats=2, spill=False),
+    "w0det": dict(collect_stats=2, deterministic=True),
 }
 
 
@@ -139,7 +149,9 @@ def main():
     if a.timeline:
         G.timeline(TL, a.timeline * 1000)
     for vn in a.variants.split(","):
-        o = Options(collect_stats=True, **VARIANTS[vn])
+        kw = dict(VARIANTS[vn])
+        kw.setdefault("collect_stats", True)
+        o = Options(**kw)
         for r in roots:
             best = None
             for _ in range(a.reps):
@@ -150,6 +162,7 @@ def main():
             warps = st.blocks * st.warps_per_block
             util = 1.0 - st.idle_ns / max(1.0, warps * st.traversal_ms * 1e6)
             rec = dict(graph=a.graph, variant=vn, root=int(r), ms=round(st.traversal_ms, 3),
+                       cyc_total=[st.cyc_window, st.cyc_probe, st.cyc_claim, st.cyc_tail, st.cyc_outside],
                        total_ms=round(st.kernel_ms, 3), gteps=round(st.m_visited / st.traversal_ms / 1e6, 4),
                        n_visited=st.n_visited, util=round(util, 4), claims=st.claims,
                        failed=st.failed_claims, windows=st.windows, flushes=st.flushes,
@@ -158,7 +171,7 @@ def main():
                        us_per_claim_per_warp=round(st.traversal_ms * 1e3 * warps * util / max(1, st.claims), 3),
                        windows_per_claim=round(st.windows / max(1, st.claims), 3),
                        cyc_per_window=[round(x / max(1, st.windows), 1) for x in
-                                       (st.cyc_window, st.cyc_probe, st.cyc_claim, st.cyc_tail)])
+                                       (st.cyc_window, st.cyc_probe, st.cyc_claim, st.cyc_tail, st.cyc_outside)])
             if a.timeline:
                 G.run(int(r), out=out, options=o)      # sampled run
                 tl = G.timeline(TL, a.timeline * 1000, fetch=True)

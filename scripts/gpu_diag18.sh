@@ -1,0 +1,12 @@
+cd $GRAFT_REPO_ROOT
+mkdir -p gpurun_out
+timeout 600 python scripts/diag.py --graph cat:262144 --roots 1 --reps 1 --variants default,det32 > gpurun_out/diag18_cat.jsonl 2> gpurun_out/diag18.err
+timeout 600 python scripts/diag.py --graph road:4900 --roots 2 --reps 1 --variants default > gpurun_out/diag18_road.jsonl 2>> gpurun_out/diag18.err
+timeout 300 python scripts/diag.py --graph rmat:22 --roots 2 --reps 2 --variants default > gpurun_out/diag18_rmat.jsonl 2>> gpurun_out/diag18.err
+python - <<'PY'
+import json
+for f in ['gpurun_out/diag18_cat.jsonl','gpurun_out/diag18_road.jsonl','gpurun_out/diag18_rmat.jsonl']:
+    for l in open(f):
+        d=json.loads(l); print(d['graph'],d['variant'],d['root'],d['ms'],d['gteps'],'util',d['util'],'us/claim',d['us_per_claim_per_warp'],'w/c',d['windows_per_claim'],'cyc',d['cyc_per_window'])
+PY
+tail -2 gpurun_out/diag18.err

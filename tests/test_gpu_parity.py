@@ -265,3 +265,17 @@ def test_concurrent_batch(conc):
             _exact(g, int(r), d[q])
         with pytest.raises(DfsError):
             G.run_batch(roots, options=Options(concurrency=conc, blocks=148))   # blocks*conc > SMs
+
+
+def test_one_level_stack_and_block_claims():
+    """ring_cap=2 (v1 one-level stack: every push spills) stays valid; block claims sum to the
+    claims (Fig 9 task counts)."""
+    g = graphgen.road(300, 200, seed=12)
+    with Graph(g.row_ptr, g.col_idx) as G:
+        for opts in (dict(ring_cap=2), dict(ring_cap=3, blocks=1, inter_steal=False),
+                     dict(ring_cap=2, deterministic=True)):
+            p, st = G.run(0, options=Options(**opts), stats=True, block_claims=True)
+            r = _valid(g, 0, p)
+            assert int(st.block_claims.sum()) == r.n_visited - 1
+            if opts.get("deterministic"):
+                _exact(g, 0, p)
