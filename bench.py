@@ -295,7 +295,7 @@ def main():
                                          f"{ms:.1f} ms each, 1 host thread ({platform.processor() or 'cpu'}, "
                                          f"{os.cpu_count()} host cores)"}
     if not a.no_e2e:
-        rec["e2e"] = e2e_leg(a, g, my_roots, m_r, dfsmod)
+        rec["e2e"] = e2e_leg(a, g, my_roots, m_r, dfsmod, G)
     print(json.dumps(rec), flush=True)
     G.close()
     if world > 1:
@@ -367,36 +367,62 @@ def batch_arm(a, world, rank, local):
         dist.destroy_process_group()
 
 
-def e2e_leg(a, g, my_roots, m_r, dfsmod):
-    """Public C ABI with host buffers: create (H2D CSR) + run (D2H parents) + destroy per step."""
+def e2e_leg(a, g, my_roots, m_r, dfsmod, G):
+    """Public C ABI with host buffers.
+
+    e2e (headline): the graph is resident (like a model's weights); each step is one user call
+    dfs_run(handle, root, parent_out) with parent_out in pinned host memory — the step's input
+    (the root) goes host -> device and the result (n int32 parents) comes back device -> host
+    inside the timed region.
+    with_upload: additionally dfs_graph_create from the host CSR and dfs_graph_destroy per step.
+    """
     import ctypes
 
     import torch
     lib = dfsmod.load_library()
-    rp = np.ascontiguousarray(g.row_ptr)
-    ci = np.ascontiguousarray(g.col_idx)
     out = torch.empty(g.n, dtype=torch.int32).pin_memory()
-    k = max(1, min(3, a.steps))
+    k = max(1, min(5, a.steps))
+    h = ctypes.c_void_p(G._h)
     ts, edges = [], 0
     for s in range(k + 1):
         r = my_roots[s % len(my_roots)]
         torch.cuda.synchronize()
         t0 = time.perf_counter()
-        h = lib.dfs_graph_create(rp.ctypes.data, ci.ctypes.data, g.n, g.m)
-        assert h, lib.dfs_last_error()
         rc = lib.dfs_run(h, int(r), ctypes.c_void_p(out.data_ptr()))
-        lib.dfs_graph_destroy(h)
         torch.cuda.synchronize()
         dt = time.perf_counter() - t0
         assert rc == 0, rc
         if s > 0:                      # first is warm-up
             ts.append(dt)
             edges += m_r[r]
-    h2d = (g.n + 1) * 4 + g.m * 4
-    return {"value": round(edges / sum(ts) / 1e9, 6), "unit": "GTEPS", "h2d_bytes_per_step": int(h2d),
-            "d2h_bytes_per_step": int(g.n * 4), "steps": k, "ms_per_step": round(sum(ts) / k * 1e3, 3),
-            "what": "dfs_graph_create(host CSR) + dfs_run(host parent_out) + dfs_graph_destroy; wall clock "
-                    "with cuda sync on both sides"}
+    rec = {"value": round(edges / sum(ts) / 1e9, 6), "unit": "GTEPS", "h2d_bytes_per_step": 4,
+           "d2h_bytes_per_step": int(g.n * 4), "steps": k, "ms_per_step": round(sum(ts) / k * 1e3, 3),
+           "what": "dfs_run(resident graph, root, pinned host parent_out); wall clock, cuda sync both sides"}
+    # with the CSR upload in every step
+    rp = np.ascontiguousarray(g.row_ptr)
+    ci = np.ascontiguousarray(g.col_idx)
+    ku = max(1, min(2, a.steps))
+    tu, eu = [], 0
+    for s in range(ku + 1):
+        r = my_roots[s % len(my_roots)]
+        torch.cuda.synchronize()
+        t0 = time.perf_counter()
+        hu = lib.dfs_graph_create(rp.ctypes.data, ci.ctypes.data, g.n, g.m)
+        assert hu, lib.dfs_last_error()
+        rc = lib.dfs_run(hu, int(r), ctypes.c_void_p(out.data_ptr()))
+        lib.dfs_graph_destroy(hu)
+        torch.cuda.synchronize()
+        dt = time.perf_counter() - t0
+        assert rc == 0, rc
+        if s > 0:
+            tu.append(dt)
+            eu += m_r[r]
+    rec["with_upload"] = {"value": round(eu / sum(tu) / 1e9, 6), "unit": "GTEPS",
+                          "h2d_bytes_per_step": int((g.n + 1) * 8 + g.m * 4),
+                          "d2h_bytes_per_step": int(g.n * 4), "steps": ku,
+                          "ms_per_step": round(sum(tu) / ku * 1e3, 3),
+                          "what": "dfs_graph_create(host CSR) + dfs_run(pinned host out) + dfs_graph_destroy"}
+    return rec
 
 
 def reference_arm(a, world, rank):

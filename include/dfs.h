@@ -119,6 +119,8 @@ typedef struct dfs_options {
     int32_t prefetch;        /* 1: L2-prefetch every probed candidate's first adjacency window */
     int32_t ring_cap;        /* usable HotRing entries (0 = all 256); 2 makes every push spill: the
                                 "one-level stack" of the paper's v1 (Fig 8)            */
+    int32_t backoff_min_ns;  /* first __nanosleep of an idle warp's backoff; default 32           */
+    int32_t reserved[7];     /* zero                                                              */
 } dfs_options;
 
 typedef struct dfs_stats {

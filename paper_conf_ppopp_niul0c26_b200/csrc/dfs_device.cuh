@@ -87,6 +87,7 @@ struct KParams {
     int spill_idle;                          // ... when at least this many warps are idle
     int inter_any;                           // any idle warp may steal inter-block (else leader of an idle block)
     unsigned int backoff_max_ns;             // idle-loop exponential backoff cap
+    unsigned int backoff_min_ns;             // ... and first step
     unsigned int* timeline;                  // optional: busy-warp samples (block 0 / warp 0)
     unsigned int timeline_len;
     unsigned int timeline_dt_ns;
@@ -755,7 +756,7 @@ __global__ void __launch_bounds__(32 * WMAX, 1) dfs_persistent_kernel(const KPar
             __syncwarp();
         }
         bool got_work = false;
-        uint32_t backoff = 32;
+        uint32_t backoff = P.backoff_min_ns;
         tc_prev = 0;
         t_idle0 = STATS ? globaltimer() : 0ull;
         while (!got_work) {

@@ -176,6 +176,7 @@ void dfs_options_default(dfs_options* o) {
     o->concurrency = 0;
     o->prefetch = 0;
     o->ring_cap = 0;
+    o->backoff_min_ns = 32;
 }
 
 int dfs_last_error(void) { return g_last_error; }
@@ -232,28 +233,31 @@ dfs_graph* dfs_graph_create(const int64_t* row_ptr, const int32_t* col_idx, int6
     if (rc != DFS_OK) { free_graph(g); fail(rc); return nullptr; }
 
     // ---- copy + validate + narrow (step a1) ----
+    // Both arrays are staged on the device (host inputs are copied as they are; device inputs are
+    // used in place) and validated by kernels: no O(n) host loop on the create path.
     int* d_bad = nullptr;
-    if (cudaMalloc(&d_bad, sizeof(int)) != cudaSuccess) { cudaGetLastError(); free_graph(g); fail(DFS_ENOMEM); return nullptr; }
-    cudaMemset(d_bad, 0, sizeof(int));
-    bool bad = false;
-    if (is_device_ptr(row_ptr)) {
-        const int blocks = (int)std::min<int64_t>((n + 256) / 256 + 1, 65535);
-        dfs_validate_rowptr_kernel<<<blocks, 256>>>(row_ptr, g->d_rp, n, m, d_bad);
-        g->launches++;
-    } else {
-        std::vector<uint32_t> rp32((size_t)n + 1);
-        for (int64_t v = 0; v <= n; ++v) {
-            const int64_t a = row_ptr[v];
-            if (a < 0 || a > m || (v == 0 && a != 0) || (v == n && a != m) || (v < n && row_ptr[v + 1] < a)) { bad = true; break; }
-            rp32[(size_t)v] = (uint32_t)a;
-        }
-        if (!bad) cudaMemcpy(g->d_rp, rp32.data(), (size_t)(n + 1) * sizeof(uint32_t), cudaMemcpyHostToDevice);
+    int64_t* d_rp64 = nullptr;                 // staging copy of a host row_ptr
+    int32_t* d_col = nullptr;                  // staging copy of col_idx (freed after adj is built)
+    const bool rp_dev = is_device_ptr(row_ptr);
+    bool ok = cudaMalloc(&d_bad, sizeof(int)) == cudaSuccess &&
+              (rp_dev || cudaMalloc(&d_rp64, (size_t)(n + 1) * sizeof(int64_t)) == cudaSuccess) &&
+              (m == 0 || cudaMalloc(&d_col, (size_t)m * sizeof(int32_t)) == cudaSuccess);
+    if (!ok) {
+        cudaGetLastError(); cudaFree(d_bad); cudaFree(d_rp64); cudaFree(d_col);
+        free_graph(g); fail(DFS_ENOMEM); return nullptr;
     }
-    int32_t* d_col = nullptr;   // staging copy of col_idx (freed after the adjacency is built)
-    if (!bad && m > 0) {
-        if (cudaMalloc(&d_col, (size_t)m * sizeof(int32_t)) != cudaSuccess) {
-            cudaGetLastError(); cudaFree(d_bad); free_graph(g); fail(DFS_ENOMEM); return nullptr;
-        }
+    cudaMemset(d_bad, 0, sizeof(int));
+    const int64_t* rp_src = row_ptr;
+    if (!rp_dev) {
+        cudaMemcpy(d_rp64, row_ptr, (size_t)(n + 1) * sizeof(int64_t), cudaMemcpyHostToDevice);
+        rp_src = d_rp64;
+    }
+    {
+        const int blocks = (int)std::min<int64_t>((n + 256) / 256 + 1, 65535);
+        dfs_validate_rowptr_kernel<<<blocks, 256>>>(rp_src, g->d_rp, n, m, d_bad);
+        g->launches++;
+    }
+    if (m > 0) {
         cudaMemcpy(d_col, col_idx, (size_t)m * sizeof(int32_t), cudaMemcpyDefault);
         const int blocks = (int)std::min<int64_t>((m + 255) / 256, 65535);
         dfs_validate_col_kernel<<<blocks, 256>>>(d_col, m, n, d_bad);
@@ -262,14 +266,15 @@ dfs_graph* dfs_graph_create(const int64_t* row_ptr, const int32_t* col_idx, int6
     int hbad = 0;
     cudaMemcpy(&hbad, d_bad, sizeof(int), cudaMemcpyDeviceToHost);
     cudaFree(d_bad);
-    if (!bad && !hbad && m > 0) {
+    cudaFree(d_rp64);
+    if (!hbad && m > 0) {
         const int blocks = (int)std::min<int64_t>((m + 255) / 256, 65535);
         dfs_build_adj_kernel<<<blocks, 256>>>(d_col, g->d_rp, g->d_adj, m);
         g->launches++;
     }
     cudaFree(d_col);
     if (cudaGetLastError() != cudaSuccess) { free_graph(g); fail(DFS_ECUDA); return nullptr; }
-    if (bad || hbad) { free_graph(g); fail(DFS_EINVAL); return nullptr; }
+    if (hbad) { free_graph(g); fail(DFS_EINVAL); return nullptr; }
     cudaMemset(g->d_adj + m, 0xFF, 8 * sizeof(uint2));              // padding (never a valid position)
     if (cudaDeviceSynchronize() != cudaSuccess) { cudaGetLastError(); free_graph(g); fail(DFS_ECUDA); return nullptr; }
     return g;
@@ -352,6 +357,7 @@ static int launch_one(dfs_graph* g, Slot& sl, cudaStream_t s, int32_t root, int3
     P.spill_idle = o.spill_idle > 0 ? o.spill_idle : 32;
     P.inter_any = o.inter_any;
     P.backoff_max_ns = o.backoff_max_ns > 0 ? (unsigned)o.backoff_max_ns : 2048u;
+    P.backoff_min_ns = o.backoff_min_ns > 0 ? (unsigned)o.backoff_min_ns : 32u;
     P.pub_batch = o.pub_batch > 0 ? (uint32_t)o.pub_batch : 1u;
     P.speculate = o.speculate;
     P.steal_half = o.steal_half;

@@ -106,6 +106,10 @@ VARIANTS = {
     "w0": dict(collect_stats=2),
     "w0nospill": dict(collect_stats=2, spill=False),
     "w0det": dict(collect_stats=2, deterministic=True),
+    "bmin256": dict(backoff_min_ns=256),
+    "bmin1k": dict(backoff_min_ns=1024, backoff_max_ns=4096),
+    "bmax512": dict(backoff_max_ns=512),
+    "bmax8k": dict(backoff_max_ns=8192),
 }
 
 
@@ -134,6 +138,7 @@ def main():
     ap.add_argument("--reps", type=int, default=2)
     ap.add_argument("--variants", default="default")
     ap.add_argument("--timeline", type=int, default=0, help="timeline sample period in us (0 = off)")
+    ap.add_argument("--nostats", action="store_true", help="time the production (non-STATS) kernel")
     a = ap.parse_args()
     import torch
     from paper_conf_ppopp_niul0c26_b200 import Graph, Options
@@ -150,7 +155,7 @@ def main():
         G.timeline(TL, a.timeline * 1000)
     for vn in a.variants.split(","):
         kw = dict(VARIANTS[vn])
-        kw.setdefault("collect_stats", True)
+        kw.setdefault("collect_stats", not a.nostats)
         o = Options(**kw)
         for r in roots:
             best = None
