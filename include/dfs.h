@@ -108,19 +108,15 @@ typedef struct dfs_options {
     int32_t steal_half;      /* 1 (default): a thief takes max(h_s, rest/2) <= 32 HotRing entries
                                 (resp. max(c_s, rest/2) <= 64 ColdSeg entries); 0: exactly h_s/c_s
                                 as in Alg 3/4                                                       */
-    int32_t probe_mode;      /* visited probes: 0 = L2 (ld.global.cg, default), 1 = L1-cached,
-                                2 = ld.relaxed.gpu.  A stale probe can only say "unvisited" for a
-                                claimed vertex; the atomic claim decides, so all are exact         */
     int32_t concurrency;     /* batches: number of traversals run concurrently on the GPU, each on
                                 its own stream and a 1/concurrency share of the SMs (SURVEY
                                 §8(f)-2); 0 = auto (4, capped by the number of roots; a single
                                 dfs_run is always 1).  Slots beyond the first allocate their
                                 scratch on first use.                                              */
-    int32_t prefetch;        /* 1: L2-prefetch every probed candidate's first adjacency window */
     int32_t ring_cap;        /* usable HotRing entries (0 = all 256); 2 makes every push spill: the
                                 "one-level stack" of the paper's v1 (Fig 8)            */
     int32_t backoff_min_ns;  /* first __nanosleep of an idle warp's backoff; default 32           */
-    int32_t reserved[7];     /* zero                                                              */
+    int32_t reserved[9];     /* zero                                                              */
 } dfs_options;
 
 typedef struct dfs_stats {

@@ -96,8 +96,6 @@ struct KParams {
     uint32_t pub_batch;                      // publish the HotRing head every pub_batch pushes
     int speculate;                           // speculative claim of the child's first neighbour
     int steal_half;                          // steal max(h_s, rest/2) (resp. c_s) entries
-    int probe_mode;                          // 0: L2 (.cg) probes; 1: L1-cached probes; 2: .relaxed.gpu
-    int prefetch;                            // L2-prefetch every candidate's first window
     uint32_t ring_cap;                       // usable HotRing entries (<= H); 2 ~ one-level stack (v1)
     unsigned long long* block_claims;        // optional: claims per block (Fig 9 task counts)
 };
@@ -529,183 +527,324 @@ __global__ void __launch_bounds__(32 * WMAX, 1) dfs_persistent_kernel(const KPar
     // ---------------------------------------------------------------- main loop (Alg 2)
     for (;;) {
         if (has_top) {
-            // ===== warp-level expansion step (Alg 1 l.5-12 over one window) =====
-            // Window = positions [a, a + kWin), a = i rounded down to a multiple of VEC; lane k
-            // holds positions a+VEC*k .. a+VEC*k+VEC-1.  Positions outside [i, end) are masked.
-            if (!have_win) {
-                if (need_end) {                                   // popped entry: end unknown
-                    const uint32_t e2 = __ldg(P.rp + u + 1);
-                    load_window(i & ~(uint32_t)(VEC - 1), P.m, kHeadLanes, nbv, rsv);
-                    win_lanes = kHeadLanes;
+            if constexpr (VEC == 1) {
+                // ===== warp-level expansion step, 32-position window (Alg 1 l.5-12) =====
+                // lane k holds position i+k: neighbour nbv[0] and its row offset rsv[0]
+                if (!have_win) {
+                    const uint32_t q = i + lane;
+                    uint2 x = make_uint2(kFull, 0u);
+                    uint32_t e2 = end;
+                    if (need_end) {                                   // popped entry: end unknown
+                        e2 = __ldg(P.rp + u + 1);
+                        if (lane < kHeadLanes && q < P.m) x = __ldg(P.adj + q);
+                        win_lanes = kHeadLanes;
+                    } else {
+                        if (q < end) x = __ldg(P.adj + q);
+                        win_lanes = 32;
+                    }
+                    nbv[0] = (int)x.x; rsv[0] = x.y;
                     end = e2; need_end = false;
-                } else {
-                    load_window(i & ~(uint32_t)(VEC - 1), end, 32, nbv, rsv);
-                    win_lanes = 32;
                 }
-            }
-            {
-                // complete a head-only window when the list is longer than its loaded lanes
-                const uint32_t a0 = i & ~(uint32_t)(VEC - 1);
-                if (win_lanes < 32 && end > a0 + (uint32_t)VEC * (uint32_t)win_lanes) {
-                    int tnb[VEC];
-                    uint32_t trs[VEC];
-                    load_window(a0, end, 32, tnb, trs, win_lanes);
-                    if (lane >= win_lanes) {
-#pragma unroll
-                        for (int f = 0; f < VEC; ++f) { nbv[f] = tnb[f]; rsv[f] = trs[f]; }
+                if (win_lanes < 32 && end > i + (uint32_t)win_lanes) {   // complete a head-only window
+                    const uint32_t q = i + lane;
+                    if (lane >= win_lanes && q < end) {
+                        const uint2 x = __ldg(P.adj + q);
+                        nbv[0] = (int)x.x; rsv[0] = x.y;
                     }
                     win_lanes = 32;
                 }
-            }
-            if (STATS && lane == 0) ++cnt[kCntWindows];
-            long long tc0 = 0, tc1 = 0;
-            if (STATS) {
-                tc0 = clock_after(0u);
-                if (lane == 0 && tc_prev) { cnt[kCntTOut] += tc0 - tc_prev; ++cnt[kCntOutIters]; }
-                tc1 = clock_after((uint32_t)nbv[0] ^ end);
-            }
-            const uint32_t a = i & ~(uint32_t)(VEC - 1);
-            const uint32_t q0 = a + (uint32_t)VEC * lane;
-            // long list (hubs): load the next window now so it is in flight while this window's
-            // probes resolve (a sequential scan then costs one probe round trip per window)
-            int nxt[VEC];
-            uint32_t nxr[VEC];
-            const bool have_nxt = a + kWin < end;
-            if (have_nxt) load_window(a + kWin, end, 32, nxt, nxr);
-            // speculative claim (fresh child only): the first position whose neighbour is not the
-            // parent we came from is, if unvisited, exactly Alg 1's next tree edge.  Its claim,
-            // its end offset and its first window are all issued in parallel with the probes.
-            int sk = -1, se = 0;
-            uint32_t sv = 0, s_old = 0, s_rs = 0, s_re = 0;
-            int cnb[VEC];
-            uint32_t cnr[VEC];
-            if ((P.speculate == 1 || (P.speculate == 2 && VEC == 1)) && spec_ok) {
-                uint32_t vm = 0;
-#pragma unroll
+                if (STATS && lane == 0) ++cnt[kCntWindows];
+                long long tc0 = 0, tc1 = 0;
+                if (STATS) {
+                    tc0 = clock_after(0u);
+                    if (lane == 0 && tc_prev) { cnt[kCntTOut] += tc0 - tc_prev; ++cnt[kCntOutIters]; }
+                    tc1 = clock_after((uint32_t)nbv[0] ^ end);
+                }
+                const uint32_t q = i + lane;
+                const bool valid = q < end;
+                const int x = nbv[0];
+                // long list: the next window is in flight while this one is probed
+                const bool have_nxt = i + 32u < end;
+                int nxt0 = -1;
+                uint32_t nxr0 = 0;
+                if (have_nxt && q + 32u < end) {
+                    const uint2 y = __ldg(P.adj + q + 32u);
+                    nxt0 = (int)y.x; nxr0 = y.y;
+                }
+                // speculative claim of a fresh child's first non-parent neighbour: claim, end
+                // offset and first window are issued before the probes resolve
+                int sk = -1;
+                uint32_t sv = 0, s_old = 0, s_rs = 0, s_re = 0, cnr0 = 0;
+                int cnb0 = -1;
+                if (P.speculate != 0 && spec_ok) {
+                    const uint32_t vb = __ballot_sync(kFull, valid && (uint32_t)x != par);
+                    if (vb) {
+                        sk = __ffs(vb) - 1;
+                        sv = (uint32_t)__shfl_sync(kFull, x, sk);
+                        s_rs = __shfl_sync(kFull, rsv[0], sk);
+                        if (lane == 0) s_old = atomicOr(P.bitmap + (sv >> 5), 1u << (sv & 31));
+                        s_re = __ldg(P.rp + sv + 1);
+                        const uint32_t cq = s_rs + lane;
+                        if (lane < kHeadLanes && cq < P.m) {
+                            const uint2 y = __ldg(P.adj + cq);
+                            cnb0 = (int)y.x; cnr0 = y.y;
+                        }
+                    }
+                }
+                // probe the visited bit of every position in the window
+                uint32_t word = kFull;
+                if (valid) word = __ldcg(P.bitmap + ((uint32_t)x >> 5));
+                uint32_t unv = __ballot_sync(kFull, valid && !((word >> (x & 31)) & 1u));
+                long long tc2 = 0, tc3 = 0;
+                if (STATS) { tc2 = clock_after(unv); tc3 = tc2; }
+                bool descended = false;
+                // descend into the child claimed at position i+j: push <u, next candidate> unless
+                // u is exhausted (positions whose probe saw a claimed target stay claimed), then
+                // the child becomes the register top with its first window already loaded
+                auto descend1 = [&](int j, uint32_t v, uint32_t vrs, uint32_t vre, int cnb, uint32_t cnr) -> bool {
+                    if (STATS && lane == 0) ++cnt[kCntClaims];
+                    ++my_claims;
+                    const uint32_t later = unv & ~((2u << j) - 1u);
+                    const uint32_t ni = later ? i + (uint32_t)(__ffs(later) - 1) : i + 32u;
+                    if (ni < end) {
+                        if (!push(u, ni)) return false;
+                    }
+                    if (lane == 0) P.parent[v] = (int32_t)u;                        // Alg 1 l.10
+                    par = u;
+                    u = v; i = vrs; end = vre; have_win = true; need_end = false; spec_ok = true;
+                    win_lanes = kHeadLanes;
+                    nbv[0] = cnb; rsv[0] = cnr;
+                    descended = true;
+                    return true;
+                };
+                if (sk >= 0) {
+                    unv &= ~(1u << sk);                               // p0 is claimed either way
+                    s_old = __shfl_sync(kFull, s_old, 0);
+                    if (STATS) tc3 = clock_after(s_old);
+                    if (!(s_old & (1u << (sv & 31)))) {
+                        if (!descend1(sk, sv, s_rs, s_re, cnb0, cnr0)) goto exit_loop;
+                    } else if (STATS && lane == 0) {
+                        ++cnt[kCntFailedClaims];
+                    }
+                }
+                while (!descended && unv) {
+                    const int j = __ffs(unv) - 1;                     // first unvisited in CSR order
+                    const uint32_t v = (uint32_t)__shfl_sync(kFull, x, j);
+                    const uint32_t vrs = __shfl_sync(kFull, rsv[0], j);
+                    const uint32_t bit = 1u << (v & 31);
+                    uint32_t old = 0;
+                    if (lane == 0) old = atomicOr(P.bitmap + (v >> 5), bit);      // claim
+                    const uint32_t vre = __ldg(P.rp + v + 1);
+                    int cnb = -1;
+                    uint32_t cnr = 0;
+                    const uint32_t cq = vrs + lane;
+                    if (lane < kHeadLanes && cq < P.m) {
+                        const uint2 y = __ldg(P.adj + cq);
+                        cnb = (int)y.x; cnr = y.y;
+                    }
+                    old = __shfl_sync(kFull, old, 0);
+                    if (!(old & bit)) {
+                        if (!descend1(j, v, vrs, vre, cnb, cnr)) goto exit_loop;
+                        break;
+                    }
+                    if (STATS && lane == 0) ++cnt[kCntFailedClaims];
+                    unv &= unv - 1;                                   // lost the race: next one
+                }
+                if (STATS && lane == 0) {
+                    const long long tc4 = clock_after((uint32_t)nbv[0] ^ i);
+                    cnt[kCntTWin] += tc1 - tc0; cnt[kCntTProbe] += tc2 - tc1;
+                    cnt[kCntTClaim] += tc3 - tc2; cnt[kCntTTail] += tc4 - tc3;
+                    tc_prev = tc4;
+                }
+                if (!descended) {
+                    i += 32u;
+                    spec_ok = false;
+                    if (have_nxt) {                                   // next window already loaded
+                        nbv[0] = nxt0; rsv[0] = nxr0;
+                        have_win = true;
+                        win_lanes = 32;
+                    } else {
+                        have_win = false;                             // i >= end: Alg 1 l.14: pop
+                        has_top = pop(u, i);
+                        need_end = true;
+                    }
+                }
+            } else {
+                // ===== warp-level expansion step (Alg 1 l.5-12 over one window) =====
+                // Window = positions [a, a + kWin), a = i rounded down to a multiple of VEC; lane k
+                // holds positions a+VEC*k .. a+VEC*k+VEC-1.  Positions outside [i, end) are masked.
+                if (!have_win) {
+                    if (need_end) {                                   // popped entry: end unknown
+                        const uint32_t e2 = __ldg(P.rp + u + 1);
+                        load_window(i & ~(uint32_t)(VEC - 1), P.m, kHeadLanes, nbv, rsv);
+                        win_lanes = kHeadLanes;
+                        end = e2; need_end = false;
+                    } else {
+                        load_window(i & ~(uint32_t)(VEC - 1), end, 32, nbv, rsv);
+                        win_lanes = 32;
+                    }
+                }
+                {
+                    // complete a head-only window when the list is longer than its loaded lanes
+                    const uint32_t a0 = i & ~(uint32_t)(VEC - 1);
+                    if (win_lanes < 32 && end > a0 + (uint32_t)VEC * (uint32_t)win_lanes) {
+                        int tnb[VEC];
+                        uint32_t trs[VEC];
+                        load_window(a0, end, 32, tnb, trs, win_lanes);
+                        if (lane >= win_lanes) {
+    #pragma unroll
+                            for (int f = 0; f < VEC; ++f) { nbv[f] = tnb[f]; rsv[f] = trs[f]; }
+                        }
+                        win_lanes = 32;
+                    }
+                }
+                if (STATS && lane == 0) ++cnt[kCntWindows];
+                long long tc0 = 0, tc1 = 0;
+                if (STATS) {
+                    tc0 = clock_after(0u);
+                    if (lane == 0 && tc_prev) { cnt[kCntTOut] += tc0 - tc_prev; ++cnt[kCntOutIters]; }
+                    tc1 = clock_after((uint32_t)nbv[0] ^ end);
+                }
+                const uint32_t a = i & ~(uint32_t)(VEC - 1);
+                const uint32_t q0 = a + (uint32_t)VEC * lane;
+                // long list (hubs): load the next window now so it is in flight while this window's
+                // probes resolve (a sequential scan then costs one probe round trip per window)
+                int nxt[VEC];
+                uint32_t nxr[VEC];
+                const bool have_nxt = a + kWin < end;
+                if (have_nxt) load_window(a + kWin, end, 32, nxt, nxr);
+                // speculative claim (fresh child only): the first position whose neighbour is not the
+                // parent we came from is, if unvisited, exactly Alg 1's next tree edge.  Its claim,
+                // its end offset and its first window are all issued in parallel with the probes.
+                int sk = -1, se = 0;
+                uint32_t sv = 0, s_old = 0, s_rs = 0, s_re = 0;
+                int cnb[VEC];
+                uint32_t cnr[VEC];
+                if (P.speculate == 1 && spec_ok) {
+                    uint32_t vm = 0;
+    #pragma unroll
+                    for (int e = 0; e < VEC; ++e) {
+                        const uint32_t p = q0 + e;
+                        if (p >= i && p < end && (uint32_t)nbv[e] != par) vm |= 1u << e;
+                    }
+                    const uint32_t vb = __ballot_sync(kFull, vm != 0);
+                    if (vb) {
+                        sk = __ffs(vb) - 1;
+                        se = __ffs(__shfl_sync(kFull, vm, sk)) - 1;
+                        int pick = nbv[0];
+                        uint32_t pick_rs = rsv[0];
+    #pragma unroll
+                        for (int f = 1; f < VEC; ++f) if (se == f) { pick = nbv[f]; pick_rs = rsv[f]; }
+                        sv = (uint32_t)__shfl_sync(kFull, pick, sk);
+                        s_rs = __shfl_sync(kFull, pick_rs, sk);
+                        if (lane == 0) s_old = atomicOr(P.bitmap + (sv >> 5), 1u << (sv & 31));
+                        s_re = __ldg(P.rp + sv + 1);
+                        load_window(s_rs & ~(uint32_t)(VEC - 1), P.m, kHeadLanes, cnb, cnr);
+                    }
+                }
+                // probe the visited bits of every position in the window
+                uint32_t m4 = 0;
+    #pragma unroll
                 for (int e = 0; e < VEC; ++e) {
                     const uint32_t p = q0 + e;
-                    if (p >= i && p < end && (uint32_t)nbv[e] != par) vm |= 1u << e;
+                    const int x = nbv[e];
+                    if (p >= i && p < end) {
+                        // a probe that reads "visited" is always right (bits are only ever set), so a
+                        // possibly-stale cached copy is a valid filter: the atomic claim decides
+                        const uint32_t word = __ldcg(P.bitmap + ((uint32_t)x >> 5));
+                        if (!((word >> (x & 31)) & 1u)) m4 |= 1u << e;
+                    }
                 }
-                const uint32_t vb = __ballot_sync(kFull, vm != 0);
-                if (vb) {
-                    sk = __ffs(vb) - 1;
-                    se = __ffs(__shfl_sync(kFull, vm, sk)) - 1;
-                    int pick = nbv[0];
-                    uint32_t pick_rs = rsv[0];
-#pragma unroll
-                    for (int f = 1; f < VEC; ++f) if (se == f) { pick = nbv[f]; pick_rs = rsv[f]; }
-                    sv = (uint32_t)__shfl_sync(kFull, pick, sk);
-                    s_rs = __shfl_sync(kFull, pick_rs, sk);
-                    if (lane == 0) s_old = atomicOr(P.bitmap + (sv >> 5), 1u << (sv & 31));
-                    s_re = __ldg(P.rp + sv + 1);
-                    load_window(s_rs & ~(uint32_t)(VEC - 1), P.m, kHeadLanes, cnb, cnr);
+                bool descended = false;
+                long long tc2 = 0;
+                if (STATS) tc2 = clock_after(m4);
+                // descend into child v found at window slot (k, e): push <u, next candidate> (Alg 1
+                // l.8 + l.11) unless u is exhausted, then make v the register top.  Positions after
+                // (k, e) whose probe saw a claimed target stay claimed (claims are monotone), so
+                // scanning them again cannot change anything: resume at the next still-unvisited
+                // candidate, or past the window.
+                auto descend = [&](int k, int e, uint32_t v, uint32_t vrs, uint32_t vre) -> bool {
+                    if (STATS && lane == 0) ++cnt[kCntClaims];
+                    ++my_claims;
+                    const uint32_t mine = (lane == k) ? (m4 & ~((2u << e) - 1u)) : (lane > k ? m4 : 0u);
+                    const uint32_t later = __ballot_sync(kFull, mine != 0);
+                    uint32_t ni = a + kWin;
+                    if (later) {
+                        const int k2 = __ffs(later) - 1;
+                        const uint32_t m2 = __shfl_sync(kFull, mine, k2);
+                        ni = a + (uint32_t)VEC * (uint32_t)k2 + (uint32_t)(__ffs(m2) - 1);
+                    }
+                    if (ni < end) {
+                        if (!push(u, ni)) return false;
+                    }
+                    // the parent store is issued after the push so the push's CTA-scope release does
+                    // not wait for it
+                    if (lane == 0) P.parent[v] = (int32_t)u;                            // Alg 1 l.10
+                    par = u;
+                    u = v; i = vrs; end = vre; have_win = true; need_end = false; spec_ok = true;
+                    win_lanes = kHeadLanes;
+    #pragma unroll
+                    for (int f = 0; f < VEC; ++f) { nbv[f] = cnb[f]; rsv[f] = cnr[f]; }
+                    descended = true;
+                    return true;
+                };
+                long long tc3 = tc2;
+                if (sk >= 0) {
+                    if (lane == sk) m4 &= ~(1u << se);               // p0 is claimed either way
+                    s_old = __shfl_sync(kFull, s_old, 0);
+                    if (STATS) tc3 = clock_after(s_old);
+                    if (!(s_old & (1u << (sv & 31)))) {              // speculative claim won
+                        if (!descend(sk, se, sv, s_rs, s_re)) goto exit_loop;
+                    } else if (STATS && lane == 0) {
+                        ++cnt[kCntFailedClaims];
+                    }
                 }
-            }
-            // probe the visited bits of every position in the window
-            uint32_t m4 = 0;
-#pragma unroll
-            for (int e = 0; e < VEC; ++e) {
-                const uint32_t p = q0 + e;
-                const int x = nbv[e];
-                if (p >= i && p < end) {
-                    // a probe that reads "visited" is always right (bits are only ever set), so a
-                    // possibly-stale cached copy is a valid filter: the atomic claim decides
-                    const uint32_t* wp = P.bitmap + ((uint32_t)x >> 5);
-                    const uint32_t word = P.probe_mode == 1 ? *wp
-                                        : P.probe_mode == 2 ? ld_relaxed_u32(wp) : __ldcg(wp);
-                    // a candidate's adjacency window will be loaded if it is claimed (by this
-                    // warp now or by whoever reaches it later): start moving it into L2 now
-                    if (P.prefetch) asm volatile("prefetch.global.L2 [%0];" ::"l"(P.adj + rsv[e]));
-                    if (!((word >> (x & 31)) & 1u)) m4 |= 1u << e;
+                uint32_t any = descended ? 0u : __ballot_sync(kFull, m4 != 0);
+                while (any) {
+                    const int k = __ffs(any) - 1;                      // first lane with a candidate
+                    const uint32_t mk = __shfl_sync(kFull, m4, k);
+                    const int e = __ffs(mk) - 1;                       // first candidate in CSR order
+                    int mine_nb = nbv[0];
+                    uint32_t mine_rs = rsv[0];
+    #pragma unroll
+                    for (int f = 1; f < VEC; ++f)
+                        if (e == f) { mine_nb = nbv[f]; mine_rs = rsv[f]; }
+                    const uint32_t v = (uint32_t)__shfl_sync(kFull, mine_nb, k);
+                    const uint32_t vrs = __shfl_sync(kFull, mine_rs, k);
+                    const uint32_t bit = 1u << (v & 31);
+                    uint32_t old = 0;
+                    if (lane == 0) old = atomicOr(P.bitmap + (v >> 5), bit);          // claim
+                    // the child's end offset and first window load overlap the claim
+                    const uint32_t vre = __ldg(P.rp + v + 1);
+                    load_window(vrs & ~(uint32_t)(VEC - 1), P.m, kHeadLanes, cnb, cnr);
+                    old = __shfl_sync(kFull, old, 0);
+                    if (!(old & bit)) {
+                        if (!descend(k, e, v, vrs, vre)) goto exit_loop;
+                        break;
+                    }
+                    if (STATS && lane == 0) ++cnt[kCntFailedClaims];
+                    if (lane == k) m4 &= ~(1u << e);                  // lost the race: next candidate
+                    any = __ballot_sync(kFull, m4 != 0);
                 }
-            }
-            bool descended = false;
-            long long tc2 = 0;
-            if (STATS) tc2 = clock_after(m4);
-            // descend into child v found at window slot (k, e): push <u, next candidate> (Alg 1
-            // l.8 + l.11) unless u is exhausted, then make v the register top.  Positions after
-            // (k, e) whose probe saw a claimed target stay claimed (claims are monotone), so
-            // scanning them again cannot change anything: resume at the next still-unvisited
-            // candidate, or past the window.
-            auto descend = [&](int k, int e, uint32_t v, uint32_t vrs, uint32_t vre) -> bool {
-                if (STATS && lane == 0) ++cnt[kCntClaims];
-                ++my_claims;
-                if (lane == 0) P.parent[v] = (int32_t)u;                            // Alg 1 l.10
-                const uint32_t mine = (lane == k) ? (m4 & ~((2u << e) - 1u)) : (lane > k ? m4 : 0u);
-                const uint32_t later = __ballot_sync(kFull, mine != 0);
-                uint32_t ni = a + kWin;
-                if (later) {
-                    const int k2 = __ffs(later) - 1;
-                    const uint32_t m2 = __shfl_sync(kFull, mine, k2);
-                    ni = a + (uint32_t)VEC * (uint32_t)k2 + (uint32_t)(__ffs(m2) - 1);
+                if (STATS && lane == 0) {
+                    const long long tc4 = clock_after((uint32_t)nbv[0] ^ i);
+                    cnt[kCntTWin] += tc1 - tc0; cnt[kCntTProbe] += tc2 - tc1;
+                    cnt[kCntTClaim] += tc3 - tc2; cnt[kCntTTail] += tc4 - tc3;
+                    tc_prev = tc4;
                 }
-                if (ni < end) {
-                    if (!push(u, ni)) return false;
-                }
-                par = u;
-                u = v; i = vrs; end = vre; have_win = true; need_end = false; spec_ok = true;
-                win_lanes = kHeadLanes;
-#pragma unroll
-                for (int f = 0; f < VEC; ++f) { nbv[f] = cnb[f]; rsv[f] = cnr[f]; }
-                descended = true;
-                return true;
-            };
-            long long tc3 = tc2;
-            if (sk >= 0) {
-                if (lane == sk) m4 &= ~(1u << se);               // p0 is claimed either way
-                s_old = __shfl_sync(kFull, s_old, 0);
-                if (STATS) tc3 = clock_after(s_old);
-                if (!(s_old & (1u << (sv & 31)))) {              // speculative claim won
-                    if (!descend(sk, se, sv, s_rs, s_re)) goto exit_loop;
-                } else if (STATS && lane == 0) {
-                    ++cnt[kCntFailedClaims];
-                }
-            }
-            uint32_t any = descended ? 0u : __ballot_sync(kFull, m4 != 0);
-            while (any) {
-                const int k = __ffs(any) - 1;                      // first lane with a candidate
-                const uint32_t mk = __shfl_sync(kFull, m4, k);
-                const int e = __ffs(mk) - 1;                       // first candidate in CSR order
-                int mine_nb = nbv[0];
-                uint32_t mine_rs = rsv[0];
-#pragma unroll
-                for (int f = 1; f < VEC; ++f)
-                    if (e == f) { mine_nb = nbv[f]; mine_rs = rsv[f]; }
-                const uint32_t v = (uint32_t)__shfl_sync(kFull, mine_nb, k);
-                const uint32_t vrs = __shfl_sync(kFull, mine_rs, k);
-                const uint32_t bit = 1u << (v & 31);
-                uint32_t old = 0;
-                if (lane == 0) old = atomicOr(P.bitmap + (v >> 5), bit);          // claim
-                // the child's end offset and first window load overlap the claim
-                const uint32_t vre = __ldg(P.rp + v + 1);
-                load_window(vrs & ~(uint32_t)(VEC - 1), P.m, kHeadLanes, cnb, cnr);
-                old = __shfl_sync(kFull, old, 0);
-                if (!(old & bit)) {
-                    if (!descend(k, e, v, vrs, vre)) goto exit_loop;
-                    break;
-                }
-                if (STATS && lane == 0) ++cnt[kCntFailedClaims];
-                if (lane == k) m4 &= ~(1u << e);                  // lost the race: next candidate
-                any = __ballot_sync(kFull, m4 != 0);
-            }
-            if (STATS && lane == 0) {
-                const long long tc4 = clock_after((uint32_t)nbv[0] ^ i);
-                cnt[kCntTWin] += tc1 - tc0; cnt[kCntTProbe] += tc2 - tc1;
-                cnt[kCntTClaim] += tc3 - tc2; cnt[kCntTTail] += tc4 - tc3;
-                tc_prev = tc4;
-            }
-            if (!descended) {
-                i = a + kWin;
-                spec_ok = false;
-                if (have_nxt) {                                   // next window already loaded
-#pragma unroll
-                    for (int f = 0; f < VEC; ++f) { nbv[f] = nxt[f]; rsv[f] = nxr[f]; }
-                    have_win = true;
-                    win_lanes = 32;
-                } else {
-                    have_win = false;                             // i >= end: Alg 1 l.14: pop
-                    has_top = pop(u, i);
-                    need_end = true;
+                if (!descended) {
+                    i = a + kWin;
+                    spec_ok = false;
+                    if (have_nxt) {                                   // next window already loaded
+    #pragma unroll
+                        for (int f = 0; f < VEC; ++f) { nbv[f] = nxt[f]; rsv[f] = nxr[f]; }
+                        have_win = true;
+                        win_lanes = 32;
+                    } else {
+                        have_win = false;                             // i >= end: Alg 1 l.14: pop
+                        has_top = pop(u, i);
+                        need_end = true;
+                    }
                 }
             }
             ++iter;

@@ -172,9 +172,7 @@ void dfs_options_default(dfs_options* o) {
     o->pub_batch = 1;
     o->speculate = 2;
     o->steal_half = 1;
-    o->probe_mode = 0;
     o->concurrency = 0;
-    o->prefetch = 0;
     o->ring_cap = 0;
     o->backoff_min_ns = 32;
 }
@@ -361,8 +359,6 @@ static int launch_one(dfs_graph* g, Slot& sl, cudaStream_t s, int32_t root, int3
     P.pub_batch = o.pub_batch > 0 ? (uint32_t)o.pub_batch : 1u;
     P.speculate = o.speculate;
     P.steal_half = o.steal_half;
-    P.probe_mode = o.probe_mode;
-    P.prefetch = o.prefetch;
     P.ring_cap = (o.ring_cap > 0 && o.ring_cap < kRing) ? (uint32_t)o.ring_cap : (uint32_t)kRing;
     P.block_claims = sl.block_claims;
     const bool tl = g->d_timeline && &sl == &g->slots[0];

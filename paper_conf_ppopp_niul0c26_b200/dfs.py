@@ -46,10 +46,9 @@ class _Options(ctypes.Structure):
                 ("inter_any", ctypes.c_int32), ("spill_idle", ctypes.c_int32),
                 ("backoff_max_ns", ctypes.c_int32), ("window", ctypes.c_int32),
                 ("pub_batch", ctypes.c_int32), ("speculate", ctypes.c_int32),
-                ("steal_half", ctypes.c_int32), ("probe_mode", ctypes.c_int32),
-                ("concurrency", ctypes.c_int32), ("prefetch", ctypes.c_int32),
+                ("steal_half", ctypes.c_int32), ("concurrency", ctypes.c_int32),
                 ("ring_cap", ctypes.c_int32), ("backoff_min_ns", ctypes.c_int32),
-                ("reserved", ctypes.c_int32 * 7)]
+                ("reserved", ctypes.c_int32 * 9)]
 
 
 class _Stats(ctypes.Structure):
@@ -90,9 +89,7 @@ class Options:
     pub_batch: Optional[int] = None
     speculate: Optional[int] = None
     steal_half: Optional[bool] = None
-    probe_mode: Optional[int] = None
     concurrency: Optional[int] = None
-    prefetch: Optional[bool] = None
     ring_cap: Optional[int] = None
     backoff_min_ns: Optional[int] = None
 

@@ -90,14 +90,6 @@ VARIANTS = {
     "h1c2": dict(hot_cutoff=1, cold_cutoff=2),
     "h4c4": dict(hot_cutoff=4, cold_cutoff=4),
     "h1c1nohalf": dict(hot_cutoff=1, cold_cutoff=1, steal_half=False),
-    "det_p1": dict(deterministic=True, probe_mode=1),
-    "det_p2": dict(deterministic=True, probe_mode=2),
-    "det_p1nospec": dict(deterministic=True, probe_mode=1, speculate=0),
-    "p1": dict(probe_mode=1),
-    "p2": dict(probe_mode=2),
-    "p1nospec": dict(probe_mode=1, speculate=0),
-    "pf": dict(prefetch=True),
-    "pfp1": dict(prefetch=True, probe_mode=1),
     "nospill": dict(spill=False),
     "b37": dict(blocks=37),
     "b16": dict(blocks=16),

@@ -64,8 +64,8 @@ def test_deterministic_bit_exact(name, build, root):
     if root is None:
         root = int(graphgen.random_roots(g, 1, seed=1)[0])
     with Graph(g.row_ptr, g.col_idx) as G:
-        for win, pm in ((32, 0), (128, 0), (32, 1), (128, 2)):
-            p = G.run(root, options=Options(deterministic=True, window=win, probe_mode=pm))
+        for win, sp in ((32, 2), (128, 2), (32, 0), (128, 1)):
+            p = G.run(root, options=Options(deterministic=True, window=win, speculate=sp))
             torch.cuda.synchronize()
             _exact(g, root, p)
 
@@ -131,8 +131,8 @@ def test_parallel_directed_with_self_loops_and_duplicates():
     dict(hot_cutoff=3, cold_cutoff=5, steal_half=False),
     dict(hot_cutoff=1, cold_cutoff=1, warps_per_block=2, blocks=3, spill_idle=1, pub_batch=3),
     dict(speculate=1, window=128, steal_half=False),
-    dict(probe_mode=1),
-    dict(probe_mode=2, window=128),
+    dict(speculate=0),
+    dict(speculate=1, window=128),
 ])
 def test_stress_options(opts):
     graphs = [graphgen.road(300, 300, seed=3), graphgen.rmat(14, 8, seed=9),
