@@ -178,10 +178,11 @@ int dfs_graph_info(const dfs_graph *g, int64_t *n, int64_t *m, int32_t *device);
  * finalize, ...): the bench's "gpu_launches" count. */
 int64_t dfs_launch_count(const dfs_graph *g);
 
-/* Diagnostics: busy-warp timeline.  dfs_debug_timeline(g, len, dt_ns, NULL) enables sampling of
- * the global busy-warp counter every dt_ns (block 0 / warp 0) into a device buffer of len
- * samples (sample = busy + 1; 0 = no sample) for subsequent runs; calling it again with the same
- * len and a host buffer `out` copies the last run's samples out and clears them; len = 0 disables. */
+/* Diagnostics: busy-warp timeline.  dfs_debug_timeline(g, len, dt_ns, NULL) enables sampling
+ * every dt_ns (block 0 / warp 0) into a device buffer of len entries for subsequent runs: entry
+ * k < len/2 = busy warps + 1 (0 = no sample), entry len/2 + k = claims reported so far (busy warps
+ * report every 32 windows); calling it again with the same len and a host buffer `out` copies the
+ * last run's samples out and clears them; len = 0 disables. */
 int dfs_debug_timeline(dfs_graph *g, uint32_t len, uint32_t dt_ns, uint32_t *out);
 
 void dfs_graph_destroy(dfs_graph *g);

@@ -56,6 +56,7 @@ struct Ctl {
     unsigned int pool_bump;            // bump allocator over the chunk pool
     unsigned long long free_head;      // tagged free-stack head: (tag << 32) | chunk id
     unsigned long long counters[24];   // stats (collect_stats)
+    unsigned long long claims_progress;// timeline diagnostics: claims reported so far
 };
 
 enum CounterIdx {
@@ -305,6 +306,7 @@ __global__ void __launch_bounds__(32 * WMAX, 1) dfs_persistent_kernel(const KPar
     long long tc_prev = 0;                       // STATS: end of the previous expansion step
     uint32_t iter = 0;
     unsigned long long my_claims = 0;            // for P.block_claims (Fig 9 task distribution)
+    unsigned long long tl_reported = 0;          // timeline diagnostics
 
     if (blockIdx.x == 0 && w == 0) {
         // Alg 1 l.1-3: root claimed by the reset kernel; <root, row_ptr[root]> is our top
@@ -517,8 +519,10 @@ __global__ void __launch_bounds__(32 * WMAX, 1) dfs_persistent_kernel(const KPar
         if (P.timeline && blockIdx.x == 0 && w == 0 && lane == 0) {
             const unsigned long long now = globaltimer() - t_start;
             const unsigned int slot = (unsigned int)(now / P.timeline_dt_ns);
-            if (slot >= tl_next && slot < P.timeline_len) {
+            if (slot >= tl_next && slot < P.timeline_len / 2) {
                 P.timeline[slot] = *(volatile unsigned int*)&P.ctl->busy + 1u;   // 0 = no sample
+                P.timeline[P.timeline_len / 2 + slot] =
+                    (unsigned int)*(volatile unsigned long long*)&P.ctl->claims_progress;
                 tl_next = slot + 1;
             }
         }
@@ -848,7 +852,13 @@ __global__ void __launch_bounds__(32 * WMAX, 1) dfs_persistent_kernel(const KPar
                 }
             }
             ++iter;
-            if ((iter & 31u) == 0) sample();
+            if ((iter & 31u) == 0) {
+                if (P.timeline && lane == 0) {                    // diagnostics: claim progress
+                    atomicAdd(&P.ctl->claims_progress, my_claims - tl_reported);
+                    tl_reported = my_claims;
+                }
+                sample();
+            }
             if (P.spill && (iter & 31u) == 0) {
                 // demand-driven spill: many warps idle and a deep HotRing -> make the oldest half
                 // of it visible to other blocks (Alg 4 steals ColdSeg bottoms only)
@@ -1140,6 +1150,7 @@ __global__ void dfs_reset_kernel(uint32_t* bitmap, uint32_t nwords, unsigned lon
         ctl->status = 0;
         ctl->pool_bump = 0u;
         ctl->free_head = (unsigned long long)kEmptySlot;
+        ctl->claims_progress = 0ull;
         for (int k = 0; k < 24; ++k) ctl->counters[k] = 0ull;
     }
 }

@@ -305,7 +305,7 @@ class Graph:
 
     def timeline(self, len_: int = 0, dt_ns: int = 10_000, fetch: bool = False):
         """Diagnostics (dfs_debug_timeline): enable with len_ > 0; fetch=True returns the last
-        run's busy-warp samples as a numpy array (-1 = no sample)."""
+        run's (busy-warp samples (-1 = no sample), claims-so-far samples) as numpy arrays."""
         if not fetch:
             rc = self._lib.dfs_debug_timeline(self._h, len_, dt_ns, None)
             if rc != 0:
@@ -315,7 +315,8 @@ class Graph:
         rc = self._lib.dfs_debug_timeline(self._h, len_, dt_ns, buf.ctypes.data)
         if rc != 0:
             raise DfsError(rc, "dfs_debug_timeline")
-        return buf.astype(np.int64) - 1
+        h = len_ // 2
+        return buf[:h].astype(np.int64) - 1, buf[h:].astype(np.int64)
 
     def launch_count(self) -> int:
         return int(self._lib.dfs_launch_count(self._h))

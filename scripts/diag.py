@@ -171,9 +171,12 @@ def main():
                                        (st.cyc_window, st.cyc_probe, st.cyc_claim, st.cyc_tail, st.cyc_outside)])
             if a.timeline:
                 G.run(int(r), out=out, options=o)      # sampled run
-                tl = G.timeline(TL, a.timeline * 1000, fetch=True)
+                tl, prog = G.timeline(TL, a.timeline * 1000, fetch=True)
                 k = int(np.nonzero(tl >= 0)[0].max()) + 1 if np.any(tl >= 0) else 0
                 tl = tl[:k]
+                prog = prog[:k]
+                if k >= 20:
+                    rec["claims_by_5pct"] = [int(c[c > 0].max()) if np.any(c > 0) else 0 for c in np.array_split(prog, 20)]
                 valid = tl[tl >= 0]
                 dec = [int(np.mean(c[c >= 0])) if np.any(c >= 0) else -1 for c in np.array_split(tl, 20)] if k >= 20 else []
                 rec["timeline_us"] = a.timeline
