@@ -67,7 +67,7 @@ enum CounterIdx {
 
 struct KParams {
     const uint32_t* __restrict__ rp;         // n+1 (narrowed row_ptr; m < 2^32)
-    const uint2* __restrict__ adj;           // m (+8 padding): {neighbour v, row_ptr[v]} per CSR entry
+    const int32_t* __restrict__ col;         // m (+8 padding)
     uint32_t* bitmap;                        // ceil(n/32) visited words
     int32_t* parent;                         // n output
     unsigned long long* cold_tb;             // n_warps: (top << 32) | bottom
@@ -259,6 +259,7 @@ __global__ void __launch_bounds__(32 * WMAX, 1) dfs_persistent_kernel(const KPar
     constexpr uint32_t kBatch = H / 2;              // flush batch (reading S10)
     constexpr uint32_t kWin = 32u * VEC;            // positions per window
     constexpr int kHeadLanes = VEC == 1 ? 8 : 16;   // lanes fetched before a window's end is known
+    constexpr int kPfLanes = 8 / VEC;               // lanes covering the first 8 positions
     extern __shared__ __align__(16) unsigned char smem_raw[];
     SmemCtl& S = *reinterpret_cast<SmemCtl*>(smem_raw);
     constexpr int kCtlBytes = (sizeof(SmemCtl) + 15) & ~15;
@@ -287,10 +288,9 @@ __global__ void __launch_bounds__(32 * WMAX, 1) dfs_persistent_kernel(const KPar
     bool have_win = false;       // nbv holds the window starting at i
     bool need_end = false;       // end must be re-read from row_ptr
     uint32_t u = 0, i = 0, end = 0;
-    int nbv[VEC];                // this lane's neighbours in the current window ...
-    uint32_t rsv[VEC];           // ... and their row_ptr values (edge-annotated adjacency)
+    int nbv[VEC];                // this lane's neighbours in the current window
 #pragma unroll
-    for (int e = 0; e < VEC; ++e) { nbv[e] = -1; rsv[e] = 0; }
+    for (int e = 0; e < VEC; ++e) nbv[e] = -1;
     uint32_t my_head = 0;        // owner's true HotRing head (16-bit wrap)
     uint32_t pub = 0;            // head value published in S.ht (entries in [pub, my_head) are
                                  // private: pushed/popped without synchronisation)
@@ -314,26 +314,17 @@ __global__ void __launch_bounds__(32 * WMAX, 1) dfs_persistent_kernel(const KPar
         u = (uint32_t)P.root; i = __ldg(P.rp + u); end = __ldg(P.rp + u + 1);
     }
 
-    // window loader: lane holds positions base + VEC*lane + e, e < VEC.  Each entry is
-    // {v, row_ptr[v]}, so the child's window address is known as soon as its id is: one
-    // dependent load per DFS level instead of two (col_idx then row_ptr).
-    // Only lanes < `lanes` load (a window whose end is not yet known is fetched for its first
-    // kHeadLanes lanes; the rest is loaded once the end shows it is needed).
-    auto load_window = [&](uint32_t base, uint32_t limit, int lanes, int* nb, uint32_t* rs, int lane_lo = 0) {
+    // window loader: lane holds positions base + VEC*lane + e, e < VEC (col_idx entries; one
+    // 128-bit load per lane when VEC = 4).  Lanes outside [lane_lo, lanes) or past `limit` skip.
+    auto load_window = [&](uint32_t base, uint32_t limit, int lanes, int* nb, int lane_lo = 0) {
         const uint32_t q = base + (uint32_t)VEC * lane;
         const bool ld = lane >= lane_lo && lane < lanes && q < limit;
         if constexpr (VEC == 4) {
-            uint4 x0 = make_uint4(kFull, 0u, kFull, 0u), x1 = x0;
-            if (ld) {                                                        // adj padded
-                x0 = __ldg(reinterpret_cast<const uint4*>(P.adj + q));
-                x1 = __ldg(reinterpret_cast<const uint4*>(P.adj + q + 2));
-            }
-            nb[0] = (int)x0.x; rs[0] = x0.y; nb[1] = (int)x0.z; rs[1] = x0.w;
-            nb[2] = (int)x1.x; rs[2] = x1.y; nb[3] = (int)x1.z; rs[3] = x1.w;
+            int4 x = make_int4(-1, -1, -1, -1);
+            if (ld) x = __ldg(reinterpret_cast<const int4*>(P.col + q));    // col padded
+            nb[0] = x.x; nb[1] = x.y; nb[2] = x.z; nb[3] = x.w;
         } else {
-            uint2 x = make_uint2(kFull, 0u);
-            if (ld) x = __ldg(P.adj + q);
-            nb[0] = (int)x.x; rs[0] = x.y;
+            nb[0] = ld ? __ldg(P.col + q) : -1;
         }
     };
     // lanes of the current window that hold data (the rest are loaded on demand)
@@ -531,324 +522,190 @@ __global__ void __launch_bounds__(32 * WMAX, 1) dfs_persistent_kernel(const KPar
     // ---------------------------------------------------------------- main loop (Alg 2)
     for (;;) {
         if (has_top) {
-            if constexpr (VEC == 1) {
-                // ===== warp-level expansion step, 32-position window (Alg 1 l.5-12) =====
-                // lane k holds position i+k: neighbour nbv[0] and its row offset rsv[0]
-                if (!have_win) {
-                    const uint32_t q = i + lane;
-                    uint2 x = make_uint2(kFull, 0u);
-                    uint32_t e2 = end;
-                    if (need_end) {                                   // popped entry: end unknown
-                        e2 = __ldg(P.rp + u + 1);
-                        if (lane < kHeadLanes && q < P.m) x = __ldg(P.adj + q);
-                        win_lanes = kHeadLanes;
-                    } else {
-                        if (q < end) x = __ldg(P.adj + q);
-                        win_lanes = 32;
-                    }
-                    nbv[0] = (int)x.x; rsv[0] = x.y;
+            // ===== warp-level expansion step (Alg 1 l.5-12 over one window) =====
+            // Window = positions [a, a + kWin), a = i rounded down to a multiple of VEC; lane k
+            // holds positions a+VEC*k .. a+VEC*k+VEC-1 (col_idx entries).  Positions outside
+            // [i, end) are masked.  A popped entry's window is fetched together with its end
+            // offset for the first kHeadLanes lanes, and completed only if the list is longer.
+            if (!have_win) {
+                const uint32_t a0 = i & ~(uint32_t)(VEC - 1);
+                if (need_end) {                                   // popped entry: end unknown
+                    const uint32_t e2 = __ldg(P.rp + u + 1);
+                    load_window(a0, P.m, kHeadLanes, nbv);
+                    win_lanes = kHeadLanes;
                     end = e2; need_end = false;
+                } else {
+                    load_window(a0, end, 32, nbv);
+                    win_lanes = 32;
                 }
-                if (win_lanes < 32 && end > i + (uint32_t)win_lanes) {   // complete a head-only window
-                    const uint32_t q = i + lane;
-                    if (lane >= win_lanes && q < end) {
-                        const uint2 x = __ldg(P.adj + q);
-                        nbv[0] = (int)x.x; rsv[0] = x.y;
+            }
+            {
+                const uint32_t a0 = i & ~(uint32_t)(VEC - 1);
+                if (win_lanes < 32 && end > a0 + (uint32_t)VEC * (uint32_t)win_lanes) {
+                    int tnb[VEC];
+                    load_window(a0, end, 32, tnb, win_lanes);
+                    if (lane >= win_lanes) {
+#pragma unroll
+                        for (int f = 0; f < VEC; ++f) nbv[f] = tnb[f];
                     }
                     win_lanes = 32;
                 }
-                if (STATS && lane == 0) ++cnt[kCntWindows];
-                long long tc0 = 0, tc1 = 0;
-                if (STATS) {
-                    tc0 = clock_after(0u);
-                    if (lane == 0 && tc_prev) { cnt[kCntTOut] += tc0 - tc_prev; ++cnt[kCntOutIters]; }
-                    tc1 = clock_after((uint32_t)nbv[0] ^ end);
-                }
-                const uint32_t q = i + lane;
-                const bool valid = q < end;
-                const int x = nbv[0];
-                // long list: the next window is in flight while this one is probed
-                const bool have_nxt = i + 32u < end;
-                int nxt0 = -1;
-                uint32_t nxr0 = 0;
-                if (have_nxt && q + 32u < end) {
-                    const uint2 y = __ldg(P.adj + q + 32u);
-                    nxt0 = (int)y.x; nxr0 = y.y;
-                }
-                // speculative claim of a fresh child's first non-parent neighbour: claim, end
-                // offset and first window are issued before the probes resolve
-                int sk = -1;
-                uint32_t sv = 0, s_old = 0, s_rs = 0, s_re = 0, cnr0 = 0;
-                int cnb0 = -1;
-                if (P.speculate != 0 && spec_ok) {
-                    const uint32_t vb = __ballot_sync(kFull, valid && (uint32_t)x != par);
-                    if (vb) {
-                        sk = __ffs(vb) - 1;
-                        sv = (uint32_t)__shfl_sync(kFull, x, sk);
-                        s_rs = __shfl_sync(kFull, rsv[0], sk);
-                        if (lane == 0) s_old = atomicOr(P.bitmap + (sv >> 5), 1u << (sv & 31));
-                        s_re = __ldg(P.rp + sv + 1);
-                        const uint32_t cq = s_rs + lane;
-                        if (lane < kHeadLanes && cq < P.m) {
-                            const uint2 y = __ldg(P.adj + cq);
-                            cnb0 = (int)y.x; cnr0 = y.y;
-                        }
-                    }
-                }
-                // probe the visited bit of every position in the window
-                uint32_t word = kFull;
-                if (valid) word = __ldcg(P.bitmap + ((uint32_t)x >> 5));
-                uint32_t unv = __ballot_sync(kFull, valid && !((word >> (x & 31)) & 1u));
-                long long tc2 = 0, tc3 = 0;
-                if (STATS) { tc2 = clock_after(unv); tc3 = tc2; }
-                bool descended = false;
-                // descend into the child claimed at position i+j: push <u, next candidate> unless
-                // u is exhausted (positions whose probe saw a claimed target stay claimed), then
-                // the child becomes the register top with its first window already loaded
-                auto descend1 = [&](int j, uint32_t v, uint32_t vrs, uint32_t vre, int cnb, uint32_t cnr) -> bool {
-                    if (STATS && lane == 0) ++cnt[kCntClaims];
-                    ++my_claims;
-                    const uint32_t later = unv & ~((2u << j) - 1u);
-                    const uint32_t ni = later ? i + (uint32_t)(__ffs(later) - 1) : i + 32u;
-                    if (ni < end) {
-                        if (!push(u, ni)) return false;
-                    }
-                    if (lane == 0) P.parent[v] = (int32_t)u;                        // Alg 1 l.10
-                    par = u;
-                    u = v; i = vrs; end = vre; have_win = true; need_end = false; spec_ok = true;
-                    win_lanes = kHeadLanes;
-                    nbv[0] = cnb; rsv[0] = cnr;
-                    descended = true;
-                    return true;
-                };
-                if (sk >= 0) {
-                    unv &= ~(1u << sk);                               // p0 is claimed either way
-                    s_old = __shfl_sync(kFull, s_old, 0);
-                    if (STATS) tc3 = clock_after(s_old);
-                    if (!(s_old & (1u << (sv & 31)))) {
-                        if (!descend1(sk, sv, s_rs, s_re, cnb0, cnr0)) goto exit_loop;
-                    } else if (STATS && lane == 0) {
-                        ++cnt[kCntFailedClaims];
-                    }
-                }
-                while (!descended && unv) {
-                    const int j = __ffs(unv) - 1;                     // first unvisited in CSR order
-                    const uint32_t v = (uint32_t)__shfl_sync(kFull, x, j);
-                    const uint32_t vrs = __shfl_sync(kFull, rsv[0], j);
-                    const uint32_t bit = 1u << (v & 31);
-                    uint32_t old = 0;
-                    if (lane == 0) old = atomicOr(P.bitmap + (v >> 5), bit);      // claim
-                    const uint32_t vre = __ldg(P.rp + v + 1);
-                    int cnb = -1;
-                    uint32_t cnr = 0;
-                    const uint32_t cq = vrs + lane;
-                    if (lane < kHeadLanes && cq < P.m) {
-                        const uint2 y = __ldg(P.adj + cq);
-                        cnb = (int)y.x; cnr = y.y;
-                    }
-                    old = __shfl_sync(kFull, old, 0);
-                    if (!(old & bit)) {
-                        if (!descend1(j, v, vrs, vre, cnb, cnr)) goto exit_loop;
-                        break;
-                    }
-                    if (STATS && lane == 0) ++cnt[kCntFailedClaims];
-                    unv &= unv - 1;                                   // lost the race: next one
-                }
-                if (STATS && lane == 0) {
-                    const long long tc4 = clock_after((uint32_t)nbv[0] ^ i);
-                    cnt[kCntTWin] += tc1 - tc0; cnt[kCntTProbe] += tc2 - tc1;
-                    cnt[kCntTClaim] += tc3 - tc2; cnt[kCntTTail] += tc4 - tc3;
-                    tc_prev = tc4;
-                }
-                if (!descended) {
-                    i += 32u;
-                    spec_ok = false;
-                    if (have_nxt) {                                   // next window already loaded
-                        nbv[0] = nxt0; rsv[0] = nxr0;
-                        have_win = true;
-                        win_lanes = 32;
-                    } else {
-                        have_win = false;                             // i >= end: Alg 1 l.14: pop
-                        has_top = pop(u, i);
-                        need_end = true;
-                    }
-                }
-            } else {
-                // ===== warp-level expansion step (Alg 1 l.5-12 over one window) =====
-                // Window = positions [a, a + kWin), a = i rounded down to a multiple of VEC; lane k
-                // holds positions a+VEC*k .. a+VEC*k+VEC-1.  Positions outside [i, end) are masked.
-                if (!have_win) {
-                    if (need_end) {                                   // popped entry: end unknown
-                        const uint32_t e2 = __ldg(P.rp + u + 1);
-                        load_window(i & ~(uint32_t)(VEC - 1), P.m, kHeadLanes, nbv, rsv);
-                        win_lanes = kHeadLanes;
-                        end = e2; need_end = false;
-                    } else {
-                        load_window(i & ~(uint32_t)(VEC - 1), end, 32, nbv, rsv);
-                        win_lanes = 32;
-                    }
-                }
-                {
-                    // complete a head-only window when the list is longer than its loaded lanes
-                    const uint32_t a0 = i & ~(uint32_t)(VEC - 1);
-                    if (win_lanes < 32 && end > a0 + (uint32_t)VEC * (uint32_t)win_lanes) {
-                        int tnb[VEC];
-                        uint32_t trs[VEC];
-                        load_window(a0, end, 32, tnb, trs, win_lanes);
-                        if (lane >= win_lanes) {
-    #pragma unroll
-                            for (int f = 0; f < VEC; ++f) { nbv[f] = tnb[f]; rsv[f] = trs[f]; }
-                        }
-                        win_lanes = 32;
-                    }
-                }
-                if (STATS && lane == 0) ++cnt[kCntWindows];
-                long long tc0 = 0, tc1 = 0;
-                if (STATS) {
-                    tc0 = clock_after(0u);
-                    if (lane == 0 && tc_prev) { cnt[kCntTOut] += tc0 - tc_prev; ++cnt[kCntOutIters]; }
-                    tc1 = clock_after((uint32_t)nbv[0] ^ end);
-                }
-                const uint32_t a = i & ~(uint32_t)(VEC - 1);
-                const uint32_t q0 = a + (uint32_t)VEC * lane;
-                // long list (hubs): load the next window now so it is in flight while this window's
-                // probes resolve (a sequential scan then costs one probe round trip per window)
-                int nxt[VEC];
-                uint32_t nxr[VEC];
-                const bool have_nxt = a + kWin < end;
-                if (have_nxt) load_window(a + kWin, end, 32, nxt, nxr);
-                // speculative claim (fresh child only): the first position whose neighbour is not the
-                // parent we came from is, if unvisited, exactly Alg 1's next tree edge.  Its claim,
-                // its end offset and its first window are all issued in parallel with the probes.
-                int sk = -1, se = 0;
-                uint32_t sv = 0, s_old = 0, s_rs = 0, s_re = 0;
-                int cnb[VEC];
-                uint32_t cnr[VEC];
-                if (P.speculate == 1 && spec_ok) {
-                    uint32_t vm = 0;
-    #pragma unroll
-                    for (int e = 0; e < VEC; ++e) {
-                        const uint32_t p = q0 + e;
-                        if (p >= i && p < end && (uint32_t)nbv[e] != par) vm |= 1u << e;
-                    }
-                    const uint32_t vb = __ballot_sync(kFull, vm != 0);
-                    if (vb) {
-                        sk = __ffs(vb) - 1;
-                        se = __ffs(__shfl_sync(kFull, vm, sk)) - 1;
-                        int pick = nbv[0];
-                        uint32_t pick_rs = rsv[0];
-    #pragma unroll
-                        for (int f = 1; f < VEC; ++f) if (se == f) { pick = nbv[f]; pick_rs = rsv[f]; }
-                        sv = (uint32_t)__shfl_sync(kFull, pick, sk);
-                        s_rs = __shfl_sync(kFull, pick_rs, sk);
-                        if (lane == 0) s_old = atomicOr(P.bitmap + (sv >> 5), 1u << (sv & 31));
-                        s_re = __ldg(P.rp + sv + 1);
-                        load_window(s_rs & ~(uint32_t)(VEC - 1), P.m, kHeadLanes, cnb, cnr);
-                    }
-                }
-                // probe the visited bits of every position in the window
-                uint32_t m4 = 0;
-    #pragma unroll
+            }
+            if (STATS && lane == 0) ++cnt[kCntWindows];
+            long long tc0 = 0, tc1 = 0;
+            if (STATS) {
+                tc0 = clock_after(0u);
+                if (lane == 0 && tc_prev) { cnt[kCntTOut] += tc0 - tc_prev; ++cnt[kCntOutIters]; }
+                tc1 = clock_after((uint32_t)nbv[0] ^ end);
+            }
+            const uint32_t a = i & ~(uint32_t)(VEC - 1);
+            const uint32_t q0 = a + (uint32_t)VEC * lane;
+            // long list (hubs): the next window is in flight while this one's probes resolve
+            int nxt[VEC];
+            const bool have_nxt = a + kWin < end;
+            if (have_nxt) load_window(a + kWin, end, 32, nxt);
+            // speculative claim (fresh child only): the first position whose neighbour is not the
+            // parent we came from is, if unvisited, exactly Alg 1's next tree edge; its claim and
+            // its row_ptr pair are issued before the probes
+            int sk = -1, se = 0;
+            uint32_t sv = 0, s_old = 0, s_rs = 0, s_re = 0;
+            if ((P.speculate == 1 || (P.speculate == 2 && VEC == 1)) && spec_ok) {
+                uint32_t vm = 0;
+#pragma unroll
                 for (int e = 0; e < VEC; ++e) {
                     const uint32_t p = q0 + e;
-                    const int x = nbv[e];
-                    if (p >= i && p < end) {
-                        // a probe that reads "visited" is always right (bits are only ever set), so a
-                        // possibly-stale cached copy is a valid filter: the atomic claim decides
-                        const uint32_t word = __ldcg(P.bitmap + ((uint32_t)x >> 5));
-                        if (!((word >> (x & 31)) & 1u)) m4 |= 1u << e;
-                    }
+                    if (p >= i && p < end && (uint32_t)nbv[e] != par) vm |= 1u << e;
                 }
-                bool descended = false;
-                long long tc2 = 0;
-                if (STATS) tc2 = clock_after(m4);
-                // descend into child v found at window slot (k, e): push <u, next candidate> (Alg 1
-                // l.8 + l.11) unless u is exhausted, then make v the register top.  Positions after
-                // (k, e) whose probe saw a claimed target stay claimed (claims are monotone), so
-                // scanning them again cannot change anything: resume at the next still-unvisited
-                // candidate, or past the window.
-                auto descend = [&](int k, int e, uint32_t v, uint32_t vrs, uint32_t vre) -> bool {
-                    if (STATS && lane == 0) ++cnt[kCntClaims];
-                    ++my_claims;
+                const uint32_t vb = __ballot_sync(kFull, vm != 0);
+                if (vb) {
+                    sk = __ffs(vb) - 1;
+                    if constexpr (VEC == 1) {
+                        se = 0;
+                        sv = (uint32_t)__shfl_sync(kFull, nbv[0], sk);
+                    } else {
+                        se = __ffs(__shfl_sync(kFull, vm, sk)) - 1;
+                        int pick = nbv[0];
+#pragma unroll
+                        for (int f = 1; f < VEC; ++f) if (se == f) pick = nbv[f];
+                        sv = (uint32_t)__shfl_sync(kFull, pick, sk);
+                    }
+                    if (lane == 0) s_old = atomicOr(P.bitmap + (sv >> 5), 1u << (sv & 31));
+                    s_rs = __ldg(P.rp + sv); s_re = __ldg(P.rp + sv + 1);
+                }
+            }
+            // probe the visited bits; the lanes holding the first 8 positions also prefetch their
+            // candidates' row_ptr pairs, so a claim can load the child's window immediately
+            uint32_t m4 = 0;
+            uint32_t prs[VEC], pre[VEC];
+#pragma unroll
+            for (int e = 0; e < VEC; ++e) {
+                const uint32_t p = q0 + e;
+                const int x = nbv[e];
+                prs[e] = 0; pre[e] = 0;
+                if (p >= i && p < end) {
+                    const uint32_t word = __ldcg(P.bitmap + ((uint32_t)x >> 5));
+                    if (lane < kPfLanes) { prs[e] = __ldg(P.rp + x); pre[e] = __ldg(P.rp + x + 1); }
+                    if (!((word >> (x & 31)) & 1u)) m4 |= 1u << e;
+                }
+            }
+            bool descended = false;
+            long long tc2 = 0, tc3 = 0;
+            if (STATS) { tc2 = clock_after(m4); tc3 = tc2; }
+            int cnb[VEC];
+            // descend into the child claimed at window slot (k, e): push <u, next candidate>
+            // (Alg 1 l.8 + l.11) unless u is exhausted — positions whose probe saw a claimed target
+            // stay claimed (claims are monotone), so rescanning them cannot change anything —
+            // then make v the register top with its first window (cnb) loaded
+            auto descend = [&](int k, int e, uint32_t v, uint32_t vrs, uint32_t vre) -> bool {
+                if (STATS && lane == 0) ++cnt[kCntClaims];
+                ++my_claims;
+                uint32_t ni = a + kWin;
+                if constexpr (VEC == 1) {
+                    const uint32_t later = __ballot_sync(kFull, m4 != 0) & ~((2u << k) - 1u);
+                    if (later) ni = a + (uint32_t)(__ffs(later) - 1);
+                } else {
                     const uint32_t mine = (lane == k) ? (m4 & ~((2u << e) - 1u)) : (lane > k ? m4 : 0u);
                     const uint32_t later = __ballot_sync(kFull, mine != 0);
-                    uint32_t ni = a + kWin;
                     if (later) {
                         const int k2 = __ffs(later) - 1;
                         const uint32_t m2 = __shfl_sync(kFull, mine, k2);
                         ni = a + (uint32_t)VEC * (uint32_t)k2 + (uint32_t)(__ffs(m2) - 1);
                     }
-                    if (ni < end) {
-                        if (!push(u, ni)) return false;
-                    }
-                    // the parent store is issued after the push so the push's CTA-scope release does
-                    // not wait for it
-                    if (lane == 0) P.parent[v] = (int32_t)u;                            // Alg 1 l.10
-                    par = u;
-                    u = v; i = vrs; end = vre; have_win = true; need_end = false; spec_ok = true;
-                    win_lanes = kHeadLanes;
-    #pragma unroll
-                    for (int f = 0; f < VEC; ++f) { nbv[f] = cnb[f]; rsv[f] = cnr[f]; }
-                    descended = true;
-                    return true;
-                };
-                long long tc3 = tc2;
-                if (sk >= 0) {
-                    if (lane == sk) m4 &= ~(1u << se);               // p0 is claimed either way
-                    s_old = __shfl_sync(kFull, s_old, 0);
-                    if (STATS) tc3 = clock_after(s_old);
-                    if (!(s_old & (1u << (sv & 31)))) {              // speculative claim won
-                        if (!descend(sk, se, sv, s_rs, s_re)) goto exit_loop;
-                    } else if (STATS && lane == 0) {
-                        ++cnt[kCntFailedClaims];
-                    }
                 }
-                uint32_t any = descended ? 0u : __ballot_sync(kFull, m4 != 0);
-                while (any) {
-                    const int k = __ffs(any) - 1;                      // first lane with a candidate
-                    const uint32_t mk = __shfl_sync(kFull, m4, k);
-                    const int e = __ffs(mk) - 1;                       // first candidate in CSR order
-                    int mine_nb = nbv[0];
-                    uint32_t mine_rs = rsv[0];
-    #pragma unroll
+                if (ni < end) {
+                    if (!push(u, ni)) return false;
+                }
+                if (lane == 0) P.parent[v] = (int32_t)u;                            // Alg 1 l.10
+                par = u;
+                u = v; i = vrs; end = vre; have_win = true; need_end = false; spec_ok = true;
+                win_lanes = 32;
+#pragma unroll
+                for (int f = 0; f < VEC; ++f) nbv[f] = cnb[f];
+                descended = true;
+                return true;
+            };
+            if (sk >= 0) {
+                if (lane == sk) m4 &= ~(1u << se);               // p0 is claimed either way
+                s_old = __shfl_sync(kFull, s_old, 0);
+                if (STATS) tc3 = clock_after(s_old);
+                if (!(s_old & (1u << (sv & 31)))) {              // speculative claim won
+                    load_window(s_rs & ~(uint32_t)(VEC - 1), s_re, 32, cnb);
+                    if (!descend(sk, se, sv, s_rs, s_re)) goto exit_loop;
+                } else if (STATS && lane == 0) {
+                    ++cnt[kCntFailedClaims];
+                }
+            }
+            uint32_t any = descended ? 0u : __ballot_sync(kFull, m4 != 0);
+            while (any) {
+                const int k = __ffs(any) - 1;                      // first lane with a candidate
+                int e = 0;
+                int mine_nb = nbv[0];
+                uint32_t mine_rs = prs[0], mine_re = pre[0];
+                if constexpr (VEC > 1) {
+                    e = __ffs(__shfl_sync(kFull, m4, k)) - 1;      // first candidate in CSR order
+#pragma unroll
                     for (int f = 1; f < VEC; ++f)
-                        if (e == f) { mine_nb = nbv[f]; mine_rs = rsv[f]; }
-                    const uint32_t v = (uint32_t)__shfl_sync(kFull, mine_nb, k);
-                    const uint32_t vrs = __shfl_sync(kFull, mine_rs, k);
-                    const uint32_t bit = 1u << (v & 31);
-                    uint32_t old = 0;
-                    if (lane == 0) old = atomicOr(P.bitmap + (v >> 5), bit);          // claim
-                    // the child's end offset and first window load overlap the claim
-                    const uint32_t vre = __ldg(P.rp + v + 1);
-                    load_window(vrs & ~(uint32_t)(VEC - 1), P.m, kHeadLanes, cnb, cnr);
-                    old = __shfl_sync(kFull, old, 0);
-                    if (!(old & bit)) {
-                        if (!descend(k, e, v, vrs, vre)) goto exit_loop;
-                        break;
-                    }
-                    if (STATS && lane == 0) ++cnt[kCntFailedClaims];
-                    if (lane == k) m4 &= ~(1u << e);                  // lost the race: next candidate
-                    any = __ballot_sync(kFull, m4 != 0);
+                        if (e == f) { mine_nb = nbv[f]; mine_rs = prs[f]; mine_re = pre[f]; }
                 }
-                if (STATS && lane == 0) {
-                    const long long tc4 = clock_after((uint32_t)nbv[0] ^ i);
-                    cnt[kCntTWin] += tc1 - tc0; cnt[kCntTProbe] += tc2 - tc1;
-                    cnt[kCntTClaim] += tc3 - tc2; cnt[kCntTTail] += tc4 - tc3;
-                    tc_prev = tc4;
+                const uint32_t v = (uint32_t)__shfl_sync(kFull, mine_nb, k);
+                uint32_t vrs, vre;
+                if (k < kPfLanes) {
+                    vrs = __shfl_sync(kFull, mine_rs, k); vre = __shfl_sync(kFull, mine_re, k);
+                } else {
+                    vrs = __ldg(P.rp + v); vre = __ldg(P.rp + v + 1);
                 }
-                if (!descended) {
-                    i = a + kWin;
-                    spec_ok = false;
-                    if (have_nxt) {                                   // next window already loaded
-    #pragma unroll
-                        for (int f = 0; f < VEC; ++f) { nbv[f] = nxt[f]; rsv[f] = nxr[f]; }
-                        have_win = true;
-                        win_lanes = 32;
-                    } else {
-                        have_win = false;                             // i >= end: Alg 1 l.14: pop
-                        has_top = pop(u, i);
-                        need_end = true;
-                    }
+                const uint32_t bit = 1u << (v & 31);
+                uint32_t old = 0;
+                if (lane == 0) old = atomicOr(P.bitmap + (v >> 5), bit);          // claim
+                // the child's first window load overlaps the claim
+                load_window(vrs & ~(uint32_t)(VEC - 1), vre, 32, cnb);
+                old = __shfl_sync(kFull, old, 0);
+                if (!(old & bit)) {
+                    if (!descend(k, e, v, vrs, vre)) goto exit_loop;
+                    break;
+                }
+                if (STATS && lane == 0) ++cnt[kCntFailedClaims];
+                if (lane == k) m4 &= ~(1u << e);                  // lost the race: next candidate
+                any = __ballot_sync(kFull, m4 != 0);
+            }
+            if (STATS && lane == 0) {
+                const long long tc4 = clock_after((uint32_t)nbv[0] ^ i);
+                cnt[kCntTWin] += tc1 - tc0; cnt[kCntTProbe] += tc2 - tc1;
+                cnt[kCntTClaim] += tc3 - tc2; cnt[kCntTTail] += tc4 - tc3;
+                tc_prev = tc4;
+            }
+            if (!descended) {
+                i = a + kWin;
+                spec_ok = false;
+                if (have_nxt) {                                   // next window already loaded
+#pragma unroll
+                    for (int f = 0; f < VEC; ++f) nbv[f] = nxt[f];
+                    have_win = true;
+                    win_lanes = 32;
+                } else {
+                    have_win = false;                             // i >= end: Alg 1 l.14: pop
+                    has_top = pop(u, i);
+                    need_end = true;
                 }
             }
             ++iter;
@@ -1192,16 +1049,6 @@ __global__ void dfs_validate_rowptr_kernel(const int64_t* __restrict__ rp64, uin
         if (v < (size_t)n) ok = ok && rp64[v + 1] >= a;
         if (!ok) atomicExch(bad, 1);
         rp32[v] = (uint32_t)a;
-    }
-}
-
-// edge-annotated adjacency: adj[j] = {col_idx[j], row_ptr[col_idx[j]]} (step a1)
-__global__ void dfs_build_adj_kernel(const int32_t* __restrict__ col, const uint32_t* __restrict__ rp,
-                                     uint2* adj, int64_t m) {
-    const size_t stride = (size_t)gridDim.x * blockDim.x;
-    for (size_t j = blockIdx.x * (size_t)blockDim.x + threadIdx.x; j < (size_t)m; j += stride) {
-        const int32_t c = col[j];
-        adj[j] = make_uint2((uint32_t)c, __ldg(rp + c));
     }
 }
 

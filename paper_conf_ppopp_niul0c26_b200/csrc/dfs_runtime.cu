@@ -1,7 +1,7 @@
 // dfs_runtime.cu — host runtime + C ABI (include/dfs.h) of the B200 unordered-DFS library.
 //
-// Owns graph residency (step a1: copy, validate, narrow row_ptr to uint32, build the
-// edge-annotated adjacency {v, row_ptr[v]}), per-traversal scratch "slots" (visited bitmap,
+// Owns graph residency (step a1: copy, validate, narrow row_ptr to uint32), per-traversal
+// scratch "slots" (visited bitmap,
 // per-warp ColdSeg words, chunk table, chunk pool, control block) and the launch sequence
 // reset (a2) -> persistent traversal (a3-a8) -> finalize (a9).  A batch (a10) may run K
 // traversals concurrently on K slots / streams, each on a 1/K share of the SMs (SURVEY
@@ -81,7 +81,7 @@ struct dfs_graph {
     int max_blocks = 0;          // co-resident 32-warp blocks (allocation bound)
     int tab_log2 = 0;
     uint32_t* d_rp = nullptr;
-    uint2* d_adj = nullptr;      // {col_idx[j], row_ptr[col_idx[j]]} per CSR entry (+8 padding)
+    int32_t* d_col = nullptr;    // col_idx (+8 padding for 128-bit window loads)
     Slot slots[kMaxSlots];
     int64_t launches = 0;
     unsigned int* d_timeline = nullptr;   // diagnostics (dfs_debug_timeline)
@@ -107,7 +107,7 @@ static void free_graph(dfs_graph* g) {
     int cur = 0;
     cudaGetDevice(&cur);
     cudaSetDevice(g->device);
-    cudaFree(g->d_rp); cudaFree(g->d_adj); cudaFree(g->d_timeline); cudaFree(g->d_counts);
+    cudaFree(g->d_rp); cudaFree(g->d_col); cudaFree(g->d_timeline); cudaFree(g->d_counts);
     for (int k = 0; k < kMaxSlots; ++k) free_slot(g->slots[k]);
     cudaSetDevice(cur);
     delete g;
@@ -224,7 +224,7 @@ dfs_graph* dfs_graph_create(const int64_t* row_ptr, const int32_t* col_idx, int6
     while (((int64_t)1 << g->tab_log2) < need) ++g->tab_log2;
 
     if (cudaMalloc(&g->d_rp, (size_t)(n + 1) * sizeof(uint32_t)) != cudaSuccess ||
-        cudaMalloc(&g->d_adj, (size_t)(m + 8) * sizeof(uint2)) != cudaSuccess) {   // padded for 128-bit loads
+        cudaMalloc(&g->d_col, (size_t)(m + 8) * sizeof(int32_t)) != cudaSuccess) {   // padded for 128-bit loads
         cudaGetLastError(); free_graph(g); fail(DFS_ENOMEM); return nullptr;
     }
     const int rc = ensure_slot(g, 0);
@@ -235,13 +235,11 @@ dfs_graph* dfs_graph_create(const int64_t* row_ptr, const int32_t* col_idx, int6
     // used in place) and validated by kernels: no O(n) host loop on the create path.
     int* d_bad = nullptr;
     int64_t* d_rp64 = nullptr;                 // staging copy of a host row_ptr
-    int32_t* d_col = nullptr;                  // staging copy of col_idx (freed after adj is built)
     const bool rp_dev = is_device_ptr(row_ptr);
     bool ok = cudaMalloc(&d_bad, sizeof(int)) == cudaSuccess &&
-              (rp_dev || cudaMalloc(&d_rp64, (size_t)(n + 1) * sizeof(int64_t)) == cudaSuccess) &&
-              (m == 0 || cudaMalloc(&d_col, (size_t)m * sizeof(int32_t)) == cudaSuccess);
+              (rp_dev || cudaMalloc(&d_rp64, (size_t)(n + 1) * sizeof(int64_t)) == cudaSuccess);
     if (!ok) {
-        cudaGetLastError(); cudaFree(d_bad); cudaFree(d_rp64); cudaFree(d_col);
+        cudaGetLastError(); cudaFree(d_bad); cudaFree(d_rp64);
         free_graph(g); fail(DFS_ENOMEM); return nullptr;
     }
     cudaMemset(d_bad, 0, sizeof(int));
@@ -256,24 +254,18 @@ dfs_graph* dfs_graph_create(const int64_t* row_ptr, const int32_t* col_idx, int6
         g->launches++;
     }
     if (m > 0) {
-        cudaMemcpy(d_col, col_idx, (size_t)m * sizeof(int32_t), cudaMemcpyDefault);
+        cudaMemcpy(g->d_col, col_idx, (size_t)m * sizeof(int32_t), cudaMemcpyDefault);
         const int blocks = (int)std::min<int64_t>((m + 255) / 256, 65535);
-        dfs_validate_col_kernel<<<blocks, 256>>>(d_col, m, n, d_bad);
+        dfs_validate_col_kernel<<<blocks, 256>>>(g->d_col, m, n, d_bad);
         g->launches++;
     }
     int hbad = 0;
     cudaMemcpy(&hbad, d_bad, sizeof(int), cudaMemcpyDeviceToHost);
     cudaFree(d_bad);
     cudaFree(d_rp64);
-    if (!hbad && m > 0) {
-        const int blocks = (int)std::min<int64_t>((m + 255) / 256, 65535);
-        dfs_build_adj_kernel<<<blocks, 256>>>(d_col, g->d_rp, g->d_adj, m);
-        g->launches++;
-    }
-    cudaFree(d_col);
     if (cudaGetLastError() != cudaSuccess) { free_graph(g); fail(DFS_ECUDA); return nullptr; }
     if (hbad) { free_graph(g); fail(DFS_EINVAL); return nullptr; }
-    cudaMemset(g->d_adj + m, 0xFF, 8 * sizeof(uint2));              // padding (never a valid position)
+    cudaMemset(g->d_col + m, 0xFF, 8 * sizeof(int32_t));            // padding (never a valid position)
     if (cudaDeviceSynchronize() != cudaSuccess) { cudaGetLastError(); free_graph(g); fail(DFS_ECUDA); return nullptr; }
     return g;
 }
@@ -342,7 +334,7 @@ static int launch_one(dfs_graph* g, Slot& sl, cudaStream_t s, int32_t root, int3
     sl.tab_dirty = false;
 
     KParams P;
-    P.rp = g->d_rp; P.adj = g->d_adj; P.bitmap = sl.bitmap; P.parent = d_out;
+    P.rp = g->d_rp; P.col = g->d_col; P.bitmap = sl.bitmap; P.parent = d_out;
     P.cold_tb = sl.cold_tb; P.chunk_tab = sl.tab; P.pool = sl.pool;
     P.chunk_consumed = sl.consumed; P.chunk_next = sl.next; P.block_cold = sl.block_cold;
     P.ctl = sl.ctl;
