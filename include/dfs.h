@@ -116,7 +116,9 @@ typedef struct dfs_options {
     int32_t ring_cap;        /* usable HotRing entries (0 = all 256); 2 makes every push spill: the
                                 "one-level stack" of the paper's v1 (Fig 8)            */
     int32_t backoff_min_ns;  /* first __nanosleep of an idle warp's backoff; default 32           */
-    int32_t reserved[9];     /* zero                                                              */
+    int32_t max_pool_chunks; /* fault injection: cap on ColdSeg chunks a traversal may use (0 = the
+                                whole pool); exhausting it returns DFS_ENOMEM                      */
+    int32_t reserved[8];     /* zero                                                              */
 } dfs_options;
 
 typedef struct dfs_stats {

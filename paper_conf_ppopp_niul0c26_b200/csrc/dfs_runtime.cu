@@ -175,6 +175,7 @@ void dfs_options_default(dfs_options* o) {
     o->concurrency = 0;
     o->ring_cap = 0;
     o->backoff_min_ns = 32;
+    o->max_pool_chunks = 0;
 }
 
 int dfs_last_error(void) { return g_last_error; }
@@ -339,7 +340,8 @@ static int launch_one(dfs_graph* g, Slot& sl, cudaStream_t s, int32_t root, int3
     P.chunk_consumed = sl.consumed; P.chunk_next = sl.next; P.block_cold = sl.block_cold;
     P.ctl = sl.ctl;
     P.n = (uint32_t)g->n; P.m = (uint32_t)g->m; P.root = root; P.tab_log2 = g->tab_log2;
-    P.n_chunks = sl.n_chunks;
+    P.n_chunks = (o.max_pool_chunks > 0 && (uint32_t)o.max_pool_chunks < sl.n_chunks) ? (uint32_t)o.max_pool_chunks
+                                                                                      : sl.n_chunks;
     P.hot_cutoff = o.hot_cutoff; P.cold_cutoff = o.cold_cutoff;
     P.intra = o.intra_steal; P.inter = o.inter_steal; P.policy = o.victim_policy;
     P.collect_stats = o.collect_stats;

@@ -279,3 +279,29 @@ def test_one_level_stack_and_block_claims():
             assert int(st.block_claims.sum()) == r.n_visited - 1
             if opts.get("deterministic"):
                 _exact(g, 0, p)
+
+
+def test_fault_injection_timeout_enomem_and_recovery():
+    """the watchdog and pool exhaustion end the kernel with DFS_ETIMEOUT / DFS_ENOMEM
+    (no hang); the same handle then runs normally again (tables cleared after errors)."""
+    g = graphgen.grid(256, 256)                     # det snake keeps ~65K entries on the stack
+    with Graph(g.row_ptr, g.col_idx) as G:
+        with pytest.raises(DfsError) as e:
+            G.run(0, options=Options(deterministic=True, max_pool_chunks=2))
+        assert e.value.code == -2                                    # DFS_ENOMEM
+        _exact(g, 0, G.run(0, options=det()))                      # recovers
+        with pytest.raises(DfsError) as e:
+            G.run(0, options=Options(deterministic=True, timeout_ms=1))
+        assert e.value.code == -5                                    # DFS_ETIMEOUT
+        _valid(g, 0, G.run(0))
+        with pytest.raises(DfsError) as e:                           # parallel + tiny pool
+            G.run(0, options=Options(max_pool_chunks=1, ring_cap=2))
+        assert e.value.code == -2
+        _valid(g, 5, G.run(5))
+        hb = graphgen.road(600, 600, seed=2)
+    with Graph(hb.row_ptr, hb.col_idx) as G:                         # batch error propagates
+        with pytest.raises(DfsError):
+            G.run_batch([0, 1, 2, 3], options=Options(concurrency=2, ring_cap=2, max_pool_chunks=1))
+        out = G.run_batch([0, 1, 2, 3], options=Options(concurrency=2))
+        for q, r in enumerate([0, 1, 2, 3]):
+            _valid(hb, r, out[q])
