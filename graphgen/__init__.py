@@ -47,6 +47,7 @@ def _L():
             "gg_caterpillar": [I64, I64],
             "gg_random": [I64, I64, U64, I, I, I],
             "gg_from_edges": [I64, I64, P, P, I, I, I],
+            "gg_read_mtx": [ctypes.c_char_p, I],
         }.items():
             f = getattr(lib, name)
             f.argtypes = args
@@ -55,6 +56,7 @@ def _L():
         lib.gg_m.argtypes = [P]; lib.gg_m.restype = I64
         lib.gg_export.argtypes = [P, P, P]; lib.gg_export.restype = None
         lib.gg_destroy.argtypes = [P]; lib.gg_destroy.restype = None
+        lib.gg_write_mtx.argtypes = [ctypes.c_char_p, I64, P, P]; lib.gg_write_mtx.restype = I
         _lib = lib
     return _lib
 
@@ -125,6 +127,23 @@ def from_edges(n: int, src, dst, symmetrize: bool = True, dedup: bool = True,
     d = np.ascontiguousarray(dst, dtype=np.int32)
     return _take(_L().gg_from_edges(n, s.shape[0], s.ctypes.data, d.ctypes.data,
                                     int(symmetrize), int(dedup), int(drop_self)), "edges")
+
+
+def read_mtx(path: str, symmetric: bool = False) -> CSR:
+    """Matrix Market coordinate file -> CSR (1-based entries i j = edge i-1 -> j-1; symmetric
+    files store both directions; self loops / duplicates dropped).  The paper's artifact runs on
+    SuiteSparse .mtx graphs."""
+    h = _L().gg_read_mtx(os.fsencode(path), int(symmetric))
+    if not h:
+        raise ValueError(f"graphgen: cannot parse Matrix Market file {path}")
+    return _take(h, os.path.basename(path))
+
+
+def write_mtx(g: CSR, path: str) -> None:
+    rp = np.ascontiguousarray(g.row_ptr, dtype=np.int64)
+    ci = np.ascontiguousarray(g.col_idx, dtype=np.int32)
+    if _L().gg_write_mtx(os.fsencode(path), g.n, rp.ctypes.data, ci.ctypes.data if g.m else None) != 0:
+        raise OSError(f"cannot write {path}")
 
 
 def path(n: int) -> CSR:

@@ -311,3 +311,60 @@ gg_graph *gg_random(int64_t n, int64_t ne, uint64_t seed, int symmetric, int all
     free(src); free(dst);
     return g;
 }
+
+
+/* ---------------------------------------------------------------- Matrix Market input */
+/* Read a Matrix Market coordinate file (pattern / real / integer; general / symmetric) as a CSR
+ * graph: entry (i, j) (1-based) is the directed edge i-1 -> j-1; symmetric files store both
+ * directions (the artifact converts SuiteSparse .mtx files to CSR).  Self loops and
+ * duplicates are dropped (the SuiteSparse graphs are simple).  Returns NULL on parse errors. */
+#include <stdio.h>
+#include <ctype.h>
+gg_graph *gg_read_mtx(const char *path, int force_symmetric)
+{
+    FILE *f = fopen(path, "r");
+    if (!f) return NULL;
+    char line[1024];
+    if (!fgets(line, sizeof line, f)) { fclose(f); return NULL; }
+    for (char *c = line; *c; ++c) *c = (char)tolower((unsigned char)*c);
+    if (strncmp(line, "%%matrixmarket", 14) != 0 || !strstr(line, "coordinate")) { fclose(f); return NULL; }
+    const int symmetric = force_symmetric || strstr(line, "symmetric") != NULL || strstr(line, "hermitian") != NULL;
+    const int pattern = strstr(line, "pattern") != NULL;
+    const int cplx = strstr(line, "complex") != NULL;
+    do {
+        if (!fgets(line, sizeof line, f)) { fclose(f); return NULL; }
+    } while (line[0] == '%');
+    long long rows = 0, cols = 0, nnz = 0;
+    if (sscanf(line, "%lld %lld %lld", &rows, &cols, &nnz) != 3 || rows <= 0 || cols <= 0 || nnz < 0) { fclose(f); return NULL; }
+    const int64_t n = rows > cols ? rows : cols;
+    int32_t *src = (int32_t *)malloc((size_t)(nnz > 0 ? nnz : 1) * sizeof(int32_t));
+    int32_t *dst = (int32_t *)malloc((size_t)(nnz > 0 ? nnz : 1) * sizeof(int32_t));
+    if (!src || !dst) { free(src); free(dst); fclose(f); return NULL; }
+    int64_t k = 0;
+    while (k < nnz && fgets(line, sizeof line, f)) {
+        if (line[0] == '%' || line[0] == '\n') continue;
+        long long a = 0, b = 0;
+        if (sscanf(line, "%lld %lld", &a, &b) != 2 || a < 1 || b < 1 || a > n || b > n) { free(src); free(dst); fclose(f); return NULL; }
+        (void)pattern; (void)cplx;                 /* values are ignored: the graph is the pattern */
+        src[k] = (int32_t)(a - 1); dst[k] = (int32_t)(b - 1); ++k;
+    }
+    fclose(f);
+    if (k != nnz) { free(src); free(dst); return NULL; }
+    gg_graph *g = gg_from_edges(n, k, src, dst, symmetric, 1, 1);
+    free(src); free(dst);
+    return g;
+}
+
+/* Write a CSR graph as a general pattern Matrix Market file (1-based). */
+int gg_write_mtx(const char *path, int64_t n, const int64_t *row_ptr, const int32_t *col)
+{
+    FILE *f = fopen(path, "w");
+    if (!f) return -1;
+    fprintf(f, "%%%%MatrixMarket matrix coordinate pattern general\n%lld %lld %lld\n",
+            (long long)n, (long long)n, (long long)row_ptr[n]);
+    for (int64_t u = 0; u < n; ++u)
+        for (int64_t j = row_ptr[u]; j < row_ptr[u + 1]; ++j)
+            fprintf(f, "%lld %lld\n", (long long)u + 1, (long long)col[j] + 1);
+    fclose(f);
+    return 0;
+}

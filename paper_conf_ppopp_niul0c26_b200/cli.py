@@ -1,0 +1,76 @@
+"""Command-line driver: unordered DFS on a Matrix Market graph or a named synthetic config.
+
+    python -m paper_conf_ppopp_niul0c26_b200.cli --mtx graph.mtx --roots 64 --csv perf.csv
+    python -m paper_conf_ppopp_niul0c26_b200.cli --config road24m --roots 8
+
+Mirrors the paper's measurement methodology: a set of source vertices (here: the
+given ones, or `--roots` seeded vertices with out-degree > 0), one traversal per source, and the
+average of traversed edges / runtime (MTEPS).  Writes one CSV row per source (the artifact's
+per-graph perf CSV, is the model).  Every traversal runs in libdfs.so.
+"""
+from __future__ import annotations
+
+import argparse
+import csv
+import json
+import sys
+import time
+
+
+def main(argv=None) -> int:
+    ap = argparse.ArgumentParser(prog="paper_conf_ppopp_niul0c26_b200.cli")
+    src = ap.add_mutually_exclusive_group(required=True)
+    src.add_argument("--mtx", help="Matrix Market coordinate file (SuiteSparse format)")
+    src.add_argument("--config", help="named synthetic config (graphgen.CONFIGS)")
+    ap.add_argument("--symmetric", action="store_true", help="store both directions of every entry")
+    ap.add_argument("--roots", type=int, default=64, help="number of seeded source vertices")
+    ap.add_argument("--root", type=int, action="append", help="explicit source vertex (repeatable)")
+    ap.add_argument("--seed", type=int, default=0x6A7)
+    ap.add_argument("--csv", help="write per-source results here")
+    ap.add_argument("--set", action="append", default=[], metavar="KEY=VALUE",
+                    help="dfs_options field, e.g. --set hot_cutoff=32 --set cold_cutoff=64")
+    a = ap.parse_args(argv)
+
+    import graphgen
+    import torch
+
+    from . import Graph, Options
+    t0 = time.time()
+    if a.mtx:
+        g = graphgen.read_mtx(a.mtx, symmetric=a.symmetric)
+        name = a.mtx
+    else:
+        g, _, _, _ = graphgen.config_graph(a.config)
+        name = a.config
+    load_s = time.time() - t0
+    roots = [int(r) for r in (a.root or graphgen.random_roots(g, a.roots, seed=a.seed))]
+    opts = {}
+    for kv in a.set:
+        k, _, v = kv.partition("=")
+        opts[k] = int(v)
+    options = Options(**opts) if opts else None
+    G = Graph(g.row_ptr, g.col_idx)
+    out = torch.empty(g.n, dtype=torch.int32, device="cuda")
+    G.run(roots[0], out=out, options=options)                 # warm-up
+    rows = []
+    for r in roots:
+        _, st = G.run(r, out=out, options=options, stats=True)
+        rows.append(dict(root=r, n_visited=st.n_visited, m_visited=st.m_visited,
+                         ms=round(st.kernel_ms, 4), mteps=round(st.m_visited / st.kernel_ms / 1e3, 2)))
+    G.close()
+    if a.csv:
+        with open(a.csv, "w", newline="") as f:
+            w = csv.DictWriter(f, fieldnames=list(rows[0]))
+            w.writeheader()
+            w.writerows(rows)
+    tot_e = sum(r["m_visited"] for r in rows)
+    tot_ms = sum(r["ms"] for r in rows)
+    summary = dict(graph=name, n=g.n, m=g.m, sources=len(rows), load_s=round(load_s, 2),
+                   avg_mteps=round(sum(r["mteps"] for r in rows) / len(rows), 2),
+                   aggregate_mteps=round(tot_e / tot_ms / 1e3, 2), avg_ms=round(tot_ms / len(rows), 4))
+    print(json.dumps(summary))
+    return 0
+
+
+if __name__ == "__main__":
+    sys.exit(main())

@@ -305,3 +305,19 @@ def test_fault_injection_timeout_enomem_and_recovery():
         out = G.run_batch([0, 1, 2, 3], options=Options(concurrency=2))
         for q, r in enumerate([0, 1, 2, 3]):
             _valid(hb, r, out[q])
+
+
+def test_cli_on_matrix_market(tmp_path, capsys):
+    """The user-facing driver (f-4): .mtx in, per-source CSV + MTEPS summary out."""
+    import json as _json
+    from paper_conf_ppopp_niul0c26_b200 import cli
+    g = graphgen.road(64, 48, seed=6)
+    p = tmp_path / "road.mtx"
+    graphgen.write_mtx(g, str(p))
+    out_csv = tmp_path / "perf.csv"
+    assert cli.main(["--mtx", str(p), "--roots", "4", "--csv", str(out_csv), "--set", "hot_cutoff=4"]) == 0
+    summary = _json.loads(capsys.readouterr().out.strip().splitlines()[-1])
+    assert summary["sources"] == 4 and summary["n"] == g.n and summary["m"] == g.m
+    rows = out_csv.read_text().strip().splitlines()
+    assert len(rows) == 5 and rows[0].startswith("root,n_visited")
+    assert all(int(r.split(",")[1]) == g.n for r in rows[1:])          # connected: all reached

@@ -185,3 +185,21 @@ def test_self_loops_and_duplicates():
     p = oracle.dfs(rp, ci, 0)
     assert p.tolist() == [-1, 0, 1]
     assert oracle.check_tree(rp, ci, 0, p, i7=True).ok
+
+
+def test_matrix_market_roundtrip_and_symmetric(tmp_path):
+    """graphgen.read_mtx (input side, SuiteSparse format P:3294-3296): general files are read
+    as directed edges; symmetric files store both directions; self loops / duplicates dropped."""
+    g = graphgen.road(30, 20, seed=1)
+    p = tmp_path / "g.mtx"
+    graphgen.write_mtx(g, str(p))
+    h = graphgen.read_mtx(str(p))
+    assert np.array_equal(g.row_ptr, h.row_ptr) and np.array_equal(g.col_idx, h.col_idx)
+    s = tmp_path / "s.mtx"
+    s.write_text("%%MatrixMarket matrix coordinate real symmetric\n% c\n4 4 4\n2 1 1.5\n3 2 2\n4 4 7\n3 2 9\n")
+    t = graphgen.read_mtx(str(s))
+    assert t.row_ptr.tolist() == [0, 1, 3, 4, 4] and t.col_idx.tolist() == [1, 0, 2, 1]
+    bad = tmp_path / "bad.mtx"
+    bad.write_text("%%MatrixMarket matrix array real general\n2 2\n1\n2\n3\n4\n")
+    with pytest.raises(ValueError):
+        graphgen.read_mtx(str(bad))
