@@ -21,9 +21,13 @@
 
 using namespace b200dfs;
 
+#ifndef DFS_KRING
+#define DFS_KRING 256
+#endif
+
 namespace {
 
-constexpr int kRing = 256;                   // HotRing entries per warp (P:367 uses 128)
+constexpr int kRing = DFS_KRING;            // HotRing entries per warp (P:367 uses 128)
 constexpr int kMaxSlots = 8;                 // concurrent traversals per handle (batches)
 thread_local int g_last_error = DFS_OK;
 
