@@ -98,6 +98,7 @@ struct KParams {
     int speculate;                           // speculative claim of the child's first neighbour
     int steal_half;                          // steal max(h_s, rest/2) (resp. c_s) entries
     uint32_t ring_cap;                       // usable HotRing entries (<= H); 2 ~ one-level stack (v1)
+    int eager;                               // claim all later unvisited candidates of a window at once
     unsigned long long* block_claims;        // optional: claims per block (Fig 9 task counts)
 };
 
@@ -620,9 +621,25 @@ __global__ void __launch_bounds__(32 * WMAX, 1) dfs_persistent_kernel(const KPar
                 if (STATS && lane == 0) ++cnt[kCntClaims];
                 ++my_claims;
                 uint32_t ni = a + kWin;
+                uint32_t sib = 0;                         // eager: siblings claimed with v
                 if constexpr (VEC == 1) {
                     const uint32_t later = __ballot_sync(kFull, m4 != 0) & ~((2u << k) - 1u);
-                    if (later) ni = a + (uint32_t)(__ffs(later) - 1);
+                    if (later && P.eager) {
+                        // eager siblings (opt-in): every later candidate lane claims its own
+                        // neighbour now; u's scan has then passed the whole window (scan-order
+                        // consistent: u's scanner runs ahead of v's subtree)
+                        const bool c = (later >> lane) & 1u;
+                        const int x = nbv[0];
+                        uint32_t oldw = 0;
+                        if (c) oldw = atomicOr(P.bitmap + ((uint32_t)x >> 5), 1u << (x & 31));
+                        const bool won = c && !(oldw & (1u << (x & 31)));
+                        sib = __ballot_sync(kFull, won);
+                        if (won) P.parent[x] = (int32_t)u;
+                        my_claims += __popc(sib);
+                        if (STATS && lane == 0) cnt[kCntClaims] += __popc(sib);
+                    } else if (later) {
+                        ni = a + (uint32_t)(__ffs(later) - 1);
+                    }
                 } else {
                     const uint32_t mine = (lane == k) ? (m4 & ~((2u << e) - 1u)) : (lane > k ? m4 : 0u);
                     const uint32_t later = __ballot_sync(kFull, mine != 0);
@@ -634,6 +651,15 @@ __global__ void __launch_bounds__(32 * WMAX, 1) dfs_persistent_kernel(const KPar
                 }
                 if (ni < end) {
                     if (!push(u, ni)) return false;
+                }
+                if constexpr (VEC == 1) {
+                    while (sib) {                         // eager siblings: fresh entries on top
+                        const int b = __ffs(sib) - 1;
+                        sib &= sib - 1;
+                        const uint32_t wv = (uint32_t)__shfl_sync(kFull, nbv[0], b);
+                        const uint32_t wrs = b < kPfLanes ? __shfl_sync(kFull, prs[0], b) : __ldg(P.rp + wv);
+                        if (!push(wv, wrs)) return false;
+                    }
                 }
                 if (lane == 0) P.parent[v] = (int32_t)u;                            // Alg 1 l.10
                 par = u;

@@ -180,6 +180,7 @@ void dfs_options_default(dfs_options* o) {
     o->ring_cap = 0;
     o->backoff_min_ns = 32;
     o->max_pool_chunks = 0;
+    o->eager_siblings = 0;
 }
 
 int dfs_last_error(void) { return g_last_error; }
@@ -359,6 +360,7 @@ static int launch_one(dfs_graph* g, Slot& sl, cudaStream_t s, int32_t root, int3
     P.steal_half = o.steal_half;
     P.ring_cap = (o.ring_cap > 0 && o.ring_cap < kRing) ? (uint32_t)o.ring_cap : (uint32_t)kRing;
     P.block_claims = sl.block_claims;
+    P.eager = o.eager_siblings;
     const bool tl = g->d_timeline && &sl == &g->slots[0];
     P.timeline = tl ? g->d_timeline : nullptr;
     P.timeline_len = tl ? g->timeline_len : 0;

@@ -48,7 +48,8 @@ class _Options(ctypes.Structure):
                 ("pub_batch", ctypes.c_int32), ("speculate", ctypes.c_int32),
                 ("steal_half", ctypes.c_int32), ("concurrency", ctypes.c_int32),
                 ("ring_cap", ctypes.c_int32), ("backoff_min_ns", ctypes.c_int32),
-                ("max_pool_chunks", ctypes.c_int32), ("reserved", ctypes.c_int32 * 8)]
+                ("max_pool_chunks", ctypes.c_int32), ("eager_siblings", ctypes.c_int32),
+                ("reserved", ctypes.c_int32 * 7)]
 
 
 class _Stats(ctypes.Structure):
@@ -93,6 +94,7 @@ class Options:
     ring_cap: Optional[int] = None
     backoff_min_ns: Optional[int] = None
     max_pool_chunks: Optional[int] = None
+    eager_siblings: Optional[bool] = None
 
     def to_c(self) -> _Options:
         o = _Options()

@@ -102,6 +102,8 @@ VARIANTS = {
     "bmin1k": dict(backoff_min_ns=1024, backoff_max_ns=4096),
     "bmax512": dict(backoff_max_ns=512),
     "bmax8k": dict(backoff_max_ns=8192),
+    "eager": dict(eager_siblings=True),
+    "eager_h2": dict(eager_siblings=True, hot_cutoff=2, cold_cutoff=2),
 }
 
 
