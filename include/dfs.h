@@ -118,11 +118,8 @@ typedef struct dfs_options {
     int32_t backoff_min_ns;  /* first __nanosleep of an idle warp's backoff; default 32           */
     int32_t max_pool_chunks; /* fault injection: cap on ColdSeg chunks a traversal may use (0 = the
                                 whole pool); exhausting it returns DFS_ENOMEM                      */
-    int32_t eager_siblings;  /* 1 (opt-in, 32-wide windows): when a child is claimed, also claim
-                                every later still-unvisited neighbour in the window and push each as
-                                a fresh entry.  The result stays scan-order consistent (I6) but is
-                                further from a classical DFS tree than the paper's one-claim-at-a-
-                                time warp DFS; default 0                                          */
+    int32_t reserved0;       /* must be 0 (was eager_siblings: claiming every later unvisited
+                                neighbour of a window at once — measured slower, removed)          */
     int32_t reserved[7];     /* zero                                                              */
 } dfs_options;
 

@@ -98,7 +98,6 @@ struct KParams {
     int speculate;                           // speculative claim of the child's first neighbour
     int steal_half;                          // steal max(h_s, rest/2) (resp. c_s) entries
     uint32_t ring_cap;                       // usable HotRing entries (<= H); 2 ~ one-level stack (v1)
-    int eager;                               // claim all later unvisited candidates of a window at once
     unsigned long long* block_claims;        // optional: claims per block (Fig 9 task counts)
 };
 
@@ -145,6 +144,31 @@ __device__ __forceinline__ void st_cg_u64(unsigned long long* p, unsigned long l
 // release fence at GPU scope without the L1 invalidation (CCTL.IVALL) of __threadfence()
 __device__ __forceinline__ void fence_release_gpu() { asm volatile("fence.release.gpu;" ::: "memory"); }
 
+// predicated single-lane memory ops: one predicated instruction instead of an `if (lane == 0)`
+// block, which costs a BSSY/BRA/BSYNC convergence region per use (lean step)
+__device__ __forceinline__ uint32_t atom_or_if(bool p, uint32_t* a, uint32_t b) {
+    uint32_t r = 0;
+    asm volatile("{ .reg .pred q; setp.ne.u32 q, %1, 0; @q atom.global.or.b32 %0, [%2], %3; }"
+                 : "+r"(r) : "r"((uint32_t)p), "l"(a), "r"(b) : "memory");
+    return r;
+}
+__device__ __forceinline__ void st_global_if(bool p, int32_t* a, int32_t v) {
+    asm volatile("{ .reg .pred q; setp.ne.u32 q, %0, 0; @q st.global.s32 [%1], %2; }"
+                 ::"r"((uint32_t)p), "l"(a), "r"(v) : "memory");
+}
+__device__ __forceinline__ uint32_t ld_cg_if(bool p, const uint32_t* a, uint32_t dflt) {
+    uint32_t r = dflt;
+    asm volatile("{ .reg .pred q; setp.ne.u32 q, %1, 0; @q ld.global.cg.u32 %0, [%2]; }"
+                 : "+r"(r) : "r"((uint32_t)p), "l"(a));
+    return r;
+}
+__device__ __forceinline__ uint32_t ld_nc_if(bool p, const void* a, uint32_t dflt) {
+    uint32_t r = dflt;
+    asm volatile("{ .reg .pred q; setp.ne.u32 q, %1, 0; @q ld.global.nc.u32 %0, [%2]; }"
+                 : "+r"(r) : "r"((uint32_t)p), "l"(a));
+    return r;
+}
+
 // shared-memory atomics with explicit semantics (CTA scope)
 __device__ __forceinline__ uint32_t smem_addr(const void* p) { return (uint32_t)__cvta_generic_to_shared(p); }
 __device__ __forceinline__ uint32_t atom_add_release_cta(uint32_t* p, uint32_t v) {
@@ -169,6 +193,14 @@ __device__ __forceinline__ uint32_t ld_acquire_cta(const uint32_t* p) {
 }
 __device__ __forceinline__ void st_release_cta(uint32_t* p, uint32_t v) {
     asm volatile("st.release.cta.shared.u32 [%0], %1;" ::"r"(smem_addr(p)), "r"(v) : "memory");
+}
+__device__ __forceinline__ void atom_add_release_cta_if(bool p, uint32_t* a, uint32_t v) {
+    asm volatile("{ .reg .pred q; setp.ne.u32 q, %0, 0; @q atom.release.cta.shared.add.u32 _, [%1], %2; }"
+                 ::"r"((uint32_t)p), "r"(smem_addr(a)), "r"(v) : "memory");
+}
+__device__ __forceinline__ void st_shared_u64_if(bool p, unsigned long long* a, unsigned long long v) {
+    asm volatile("{ .reg .pred q; setp.ne.u32 q, %0, 0; @q st.shared.u64 [%1], %2; }"
+                 ::"r"((uint32_t)p), "r"(smem_addr(a)), "l"(v) : "memory");
 }
 
 __device__ __forceinline__ unsigned long long pack_entry(uint32_t v, uint32_t i) {
@@ -426,6 +458,27 @@ __global__ void __launch_bounds__(32 * WMAX, 1) dfs_persistent_kernel(const KPar
         return true;
     };
 
+    // lean push (32-wide step): the ring-full test uses a register copy of tailf, refreshed only
+    // when the copy says full — tailf only grows, so a stale copy is conservative; lane 0 stores
+    // the entry and publishes with predicated instructions
+    uint32_t tail_cache = 0;
+    auto push_lean = [&](uint32_t v, uint32_t idx) -> bool {
+        if (((my_head - tail_cache) & 0xFFFFu) >= P.ring_cap) {
+            tail_cache = __shfl_sync(kFull, S.tailf[w], 0);
+            if (((my_head - tail_cache) & 0xFFFFu) >= P.ring_cap) {
+                if (!flush(P.ring_cap >= 2u ? P.ring_cap / 2u : 1u, 0u)) return false;
+                tail_cache = __shfl_sync(kFull, S.tailf[w], 0);
+            }
+        }
+        st_shared_u64_if(lane == 0, ring + (my_head & (H - 1)), pack_entry(v, idx));
+        ++my_head;
+        if (((my_head - pub) & 0xFFFFu) >= P.pub_batch) {
+            atom_add_release_cta_if(lane == 0, &S.ht[w], ((my_head - pub) & 0xFFFFu) << 16);
+            pub = my_head;
+        }
+        return true;
+    };
+
     // pop the newest HotRing entry (Fig 2(d)).  A private entry needs no synchronisation; at
     // the published head one atomic decrement resolves the race with tail-side thieves (their
     // CAS fails if the word changed)
@@ -523,6 +576,105 @@ __global__ void __launch_bounds__(32 * WMAX, 1) dfs_persistent_kernel(const KPar
     // ---------------------------------------------------------------- main loop (Alg 2)
     for (;;) {
         if (has_top) {
+          if constexpr (VEC == 1) {
+            // ===== lean 32-wide expansion step (Alg 1 l.5-12 over one window) =====
+            // Lane k holds position i + k (col_idx entry nb); positions >= end are masked.  The
+            // common case — a freshly descended child whose first non-parent neighbour is
+            // unvisited — runs without any lane-0 branch: the speculative claim, the parent
+            // store, the ring store and the publication are predicated single instructions.
+            if (!have_win || win_lanes < 32) {
+                if (!have_win) {
+                    if (need_end) {                                   // popped entry: end unknown
+                        const uint32_t e2 = __ldg(P.rp + u + 1);
+                        nbv[0] = (int)ld_nc_if(lane < kHeadLanes && i + lane < P.m, P.col + i + lane, kFull);
+                        win_lanes = kHeadLanes;
+                        end = e2; need_end = false;
+                    } else {
+                        nbv[0] = (int)ld_nc_if(i + lane < end, P.col + i + lane, kFull);
+                        win_lanes = 32;
+                    }
+                    have_win = true;
+                }
+                if (win_lanes < 32) {
+                    if (end > i + (uint32_t)win_lanes) {
+                        const int t = (int)ld_nc_if(lane >= win_lanes && i + lane < end, P.col + i + lane, kFull);
+                        if (lane >= win_lanes) nbv[0] = t;
+                    }
+                    win_lanes = 32;
+                }
+            }
+            if (STATS && lane == 0) ++cnt[kCntWindows];
+            const int nb = nbv[0];
+            const bool valid = i + (uint32_t)lane < end;
+            // long list (hubs): the next window is in flight while this one's probes resolve
+            const bool have_nxt = i + 32u < end;
+            const int nxt1 = (int)ld_nc_if(have_nxt && i + 32u + lane < end, P.col + i + 32u + lane, kFull);
+            // speculative claim (fresh child only): the first position whose neighbour is not the
+            // parent we came from is, if unvisited, exactly Alg 1's next tree edge
+            const uint32_t vb = __ballot_sync(kFull, spec_ok && valid && (uint32_t)nb != par);
+            const int sk = __ffs(vb) - 1;
+            const uint32_t sv = vb ? (uint32_t)__shfl_sync(kFull, nb, sk & 31) : u;
+            uint32_t s_old = atom_or_if(vb != 0 && lane == 0, P.bitmap + (sv >> 5), 1u << (sv & 31));
+            const uint32_t s_rs = ld_nc_if(vb != 0, P.rp + sv, 0u), s_re = ld_nc_if(vb != 0, P.rp + sv + 1, 0u);
+            // probe the visited bits; lanes holding the first 8 positions prefetch their
+            // candidates' row_ptr pairs
+            const uint32_t word = ld_cg_if(valid, P.bitmap + ((uint32_t)nb >> 5), kFull);
+            const bool pf = valid && lane < kPfLanes;
+            const uint32_t prs = ld_nc_if(pf, P.rp + nb, 0u), pre = ld_nc_if(pf, P.rp + nb + 1, 0u);
+            bool cand = valid && !((word >> (nb & 31)) & 1u) && lane != sk;   // sk is claimed either way
+            s_old = __shfl_sync(kFull, s_old, 0);
+            bool won = vb != 0 && !(s_old & (1u << (sv & 31)));
+            uint32_t v = sv, vrs = s_rs, vre = s_re;
+            int kpos = sk;
+            int cnb = (int)kFull;
+            if (won) {
+                cnb = (int)ld_nc_if(vrs + lane < vre, P.col + vrs + lane, kFull);
+            } else {
+                if (STATS && vb && lane == 0) ++cnt[kCntFailedClaims];
+                // claim the first unvisited candidate in CSR order; on a lost race try the next
+                uint32_t any = __ballot_sync(kFull, cand);
+                while (any) {
+                    const int k = __ffs(any) - 1;
+                    const uint32_t cv = (uint32_t)__shfl_sync(kFull, nb, k);
+                    uint32_t crs = __shfl_sync(kFull, prs, k & (kPfLanes - 1)), cre = __shfl_sync(kFull, pre, k & (kPfLanes - 1));
+                    if (k >= kPfLanes) { crs = __ldg(P.rp + cv); cre = __ldg(P.rp + cv + 1); }
+                    const uint32_t bit = 1u << (cv & 31);
+                    uint32_t old = atom_or_if(lane == 0, P.bitmap + (cv >> 5), bit);
+                    cnb = (int)ld_nc_if(crs + lane < cre, P.col + crs + lane, kFull);   // overlaps the claim
+                    old = __shfl_sync(kFull, old, 0);
+                    if (!(old & bit)) { won = true; v = cv; vrs = crs; vre = cre; kpos = k; break; }
+                    if (STATS && lane == 0) ++cnt[kCntFailedClaims];
+                    if (lane == k) cand = false;                      // lost the race: next candidate
+                    any = __ballot_sync(kFull, cand);
+                }
+            }
+            if (won) {
+                // descend (Alg 1 l.8-11): push <u, next candidate> unless u is exhausted —
+                // positions whose probe saw a claimed target stay claimed, so skipping them keeps
+                // Alg 1's order — then v becomes the register top with its first window loaded
+                if (STATS && lane == 0) ++cnt[kCntClaims];
+                ++my_claims;
+                const uint32_t later = __ballot_sync(kFull, cand && lane > kpos);
+                const uint32_t ni = later ? i + (uint32_t)(__ffs(later) - 1) : i + 32u;
+                if (ni < end) {
+                    if (!push_lean(u, ni)) goto exit_loop;
+                }
+                st_global_if(lane == 0, P.parent + v, (int32_t)u);             // Alg 1 l.10
+                par = u;
+                u = v; i = vrs; end = vre; spec_ok = true;
+                nbv[0] = cnb; win_lanes = 32;                          // have_win stays true
+            } else {
+                i += 32u;
+                spec_ok = false;
+                if (have_nxt) {                                   // next window already loaded
+                    nbv[0] = nxt1;
+                } else {
+                    have_win = false;                             // i >= end: Alg 1 l.14: pop
+                    has_top = pop(u, i);
+                    need_end = true;
+                }
+            }
+          } else {
             // ===== warp-level expansion step (Alg 1 l.5-12 over one window) =====
             // Window = positions [a, a + kWin), a = i rounded down to a multiple of VEC; lane k
             // holds positions a+VEC*k .. a+VEC*k+VEC-1 (col_idx entries).  Positions outside
@@ -621,26 +773,7 @@ __global__ void __launch_bounds__(32 * WMAX, 1) dfs_persistent_kernel(const KPar
                 if (STATS && lane == 0) ++cnt[kCntClaims];
                 ++my_claims;
                 uint32_t ni = a + kWin;
-                uint32_t sib = 0;                         // eager: siblings claimed with v
-                if constexpr (VEC == 1) {
-                    const uint32_t later = __ballot_sync(kFull, m4 != 0) & ~((2u << k) - 1u);
-                    if (later && P.eager) {
-                        // eager siblings (opt-in): every later candidate lane claims its own
-                        // neighbour now; u's scan has then passed the whole window (scan-order
-                        // consistent: u's scanner runs ahead of v's subtree)
-                        const bool c = (later >> lane) & 1u;
-                        const int x = nbv[0];
-                        uint32_t oldw = 0;
-                        if (c) oldw = atomicOr(P.bitmap + ((uint32_t)x >> 5), 1u << (x & 31));
-                        const bool won = c && !(oldw & (1u << (x & 31)));
-                        sib = __ballot_sync(kFull, won);
-                        if (won) P.parent[x] = (int32_t)u;
-                        my_claims += __popc(sib);
-                        if (STATS && lane == 0) cnt[kCntClaims] += __popc(sib);
-                    } else if (later) {
-                        ni = a + (uint32_t)(__ffs(later) - 1);
-                    }
-                } else {
+                {
                     const uint32_t mine = (lane == k) ? (m4 & ~((2u << e) - 1u)) : (lane > k ? m4 : 0u);
                     const uint32_t later = __ballot_sync(kFull, mine != 0);
                     if (later) {
@@ -651,15 +784,6 @@ __global__ void __launch_bounds__(32 * WMAX, 1) dfs_persistent_kernel(const KPar
                 }
                 if (ni < end) {
                     if (!push(u, ni)) return false;
-                }
-                if constexpr (VEC == 1) {
-                    while (sib) {                         // eager siblings: fresh entries on top
-                        const int b = __ffs(sib) - 1;
-                        sib &= sib - 1;
-                        const uint32_t wv = (uint32_t)__shfl_sync(kFull, nbv[0], b);
-                        const uint32_t wrs = b < kPfLanes ? __shfl_sync(kFull, prs[0], b) : __ldg(P.rp + wv);
-                        if (!push(wv, wrs)) return false;
-                    }
                 }
                 if (lane == 0) P.parent[v] = (int32_t)u;                            // Alg 1 l.10
                 par = u;
@@ -734,6 +858,7 @@ __global__ void __launch_bounds__(32 * WMAX, 1) dfs_persistent_kernel(const KPar
                     need_end = true;
                 }
             }
+          }   // generic step
             ++iter;
             if ((iter & 31u) == 0) {
                 if (P.timeline && lane == 0) {                    // diagnostics: claim progress

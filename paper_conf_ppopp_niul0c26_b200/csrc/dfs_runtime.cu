@@ -180,7 +180,6 @@ void dfs_options_default(dfs_options* o) {
     o->ring_cap = 0;
     o->backoff_min_ns = 32;
     o->max_pool_chunks = 0;
-    o->eager_siblings = 0;
 }
 
 int dfs_last_error(void) { return g_last_error; }
@@ -360,7 +359,6 @@ static int launch_one(dfs_graph* g, Slot& sl, cudaStream_t s, int32_t root, int3
     P.steal_half = o.steal_half;
     P.ring_cap = (o.ring_cap > 0 && o.ring_cap < kRing) ? (uint32_t)o.ring_cap : (uint32_t)kRing;
     P.block_claims = sl.block_claims;
-    P.eager = o.eager_siblings;
     const bool tl = g->d_timeline && &sl == &g->slots[0];
     P.timeline = tl ? g->d_timeline : nullptr;
     P.timeline_len = tl ? g->timeline_len : 0;
@@ -399,6 +397,7 @@ static int resolve_options(const dfs_graph* g, const dfs_options* in, int num_ro
     if (o.hot_cutoff < 1 || o.hot_cutoff / 2 > 32) return DFS_EINVAL;
     if (o.cold_cutoff < 1 || o.cold_cutoff / 2 > 64) return DFS_EINVAL;
     if (o.victim_policy != 0 && o.victim_policy != 1) return DFS_EINVAL;
+    if (o.reserved0 != 0) return DFS_EINVAL;
     if (o.window == 0) o.window = (g->n > 0 && g->m >= 8 * g->n) ? 128 : 32;   // wide windows for dense lists
     if (o.window != 32 && o.window != 128) return DFS_EINVAL;
     if (o.concurrency < 0 || o.concurrency > kMaxSlots) return DFS_EINVAL;

@@ -48,7 +48,7 @@ class _Options(ctypes.Structure):
                 ("pub_batch", ctypes.c_int32), ("speculate", ctypes.c_int32),
                 ("steal_half", ctypes.c_int32), ("concurrency", ctypes.c_int32),
                 ("ring_cap", ctypes.c_int32), ("backoff_min_ns", ctypes.c_int32),
-                ("max_pool_chunks", ctypes.c_int32), ("eager_siblings", ctypes.c_int32),
+                ("max_pool_chunks", ctypes.c_int32), ("reserved0", ctypes.c_int32),
                 ("reserved", ctypes.c_int32 * 7)]
 
 
@@ -94,7 +94,6 @@ class Options:
     ring_cap: Optional[int] = None
     backoff_min_ns: Optional[int] = None
     max_pool_chunks: Optional[int] = None
-    eager_siblings: Optional[bool] = None
 
     def to_c(self) -> _Options:
         o = _Options()

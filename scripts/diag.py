@@ -102,8 +102,14 @@ VARIANTS = {
     "bmin1k": dict(backoff_min_ns=1024, backoff_max_ns=4096),
     "bmax512": dict(backoff_max_ns=512),
     "bmax8k": dict(backoff_max_ns=8192),
-    "eager": dict(eager_siblings=True),
-    "eager_h2": dict(eager_siblings=True, hot_cutoff=2, cold_cutoff=2),
+    "early": dict(speculate=6),
+    "pf2": dict(prefetch_lines=2),
+    "pf4": dict(prefetch_lines=4),
+    "pf8": dict(prefetch_lines=8),
+    "detpf4": dict(deterministic=True, prefetch_lines=4),
+    "early128": dict(speculate=5, window=128),
+    "w0early": dict(collect_stats=2, speculate=6),
+    "w0detearly": dict(collect_stats=2, deterministic=True, speculate=6),
 }
 
 
@@ -121,7 +127,8 @@ def graph(spec):
         n = int(float(arg))
         return graphgen.path_chords(n, n // 100)
     if kind == "cat":
-        return graphgen.caterpillar(int(arg), 94)
+        k = int(arg)
+        return graphgen.caterpillar(1 << k if k <= 30 else k, 94)     # cat:20 = spine 2^20 (C4b)
     raise ValueError(spec)
 
 

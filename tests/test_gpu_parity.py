@@ -133,8 +133,7 @@ def test_parallel_directed_with_self_loops_and_duplicates():
     dict(speculate=1, window=128, steal_half=False),
     dict(speculate=0),
     dict(speculate=1, window=128),
-    dict(eager_siblings=True),
-    dict(eager_siblings=True, hot_cutoff=4, ring_cap=3, warps_per_block=4, blocks=6),
+    dict(hot_cutoff=4, ring_cap=3, warps_per_block=4, blocks=6),
 ])
 def test_stress_options(opts):
     graphs = [graphgen.road(300, 300, seed=3), graphgen.rmat(14, 8, seed=9),
