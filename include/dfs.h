@@ -102,9 +102,12 @@ typedef struct dfs_options {
                                 (four per lane, one 128-bit load); 0 = auto (128 iff m >= 8n)      */
     int32_t pub_batch;       /* the owner publishes its HotRing head to thieves every pub_batch
                                 pushes (entries above it are private); default 1                    */
-    int32_t speculate;       /* 1: claim a freshly descended child's first non-parent neighbour
-                                in parallel with the visited probes; 0: off; 2 (default): on for
-                                32-wide windows only                                               */
+    int32_t speculate;       /* bits 0-1: 1 = claim a freshly descended child's first non-parent
+                                neighbour in parallel with the visited probes; 0 = off; 2 (default)
+                                = on for 32-wide windows only; default 2|8.  bit 2: issue that child's first
+                                window before the claim returns.  bit 3: also claim a popped
+                                entry's next position speculatively (its probe saw it unvisited
+                                when the entry was pushed)                                          */
     int32_t steal_half;      /* 1 (default): a thief takes max(h_s, rest/2) <= 32 HotRing entries
                                 (resp. max(c_s, rest/2) <= 64 ColdSeg entries); 0: exactly h_s/c_s
                                 as in Alg 3/4                                                       */

@@ -327,8 +327,15 @@ __global__ void __launch_bounds__(32 * WMAX, 1) dfs_persistent_kernel(const KPar
     uint32_t my_head = 0;        // owner's true HotRing head (16-bit wrap)
     uint32_t pub = 0;            // head value published in S.ht (entries in [pub, my_head) are
                                  // private: pushed/popped without synchronisation)
-    bool spec_ok = false;        // current window is a freshly descended child's first window
-    uint32_t par = kFull;        // parent of u when spec_ok
+    bool spec_ok = false;        // speculative claim allowed on the current window (fresh child,
+                                 // or a popped entry with speculate & 8)
+    uint32_t par = kFull;        // parent of u when spec_ok (kFull: no position to skip)
+    // speculate: bits 0-1 = mode (0 off, 1 on, 2 on for 32-wide windows), bit 2 = issue the
+    // child's first window before the claim returns (32-wide), bit 3 = also claim a popped
+    // entry's next position speculatively (its probe at push time saw it unvisited)
+    const bool spec_on = (P.speculate & 3) == 1 || ((P.speculate & 3) == 2 && VEC == 1);
+    const bool spec_early = (P.speculate & 4) != 0;
+    const bool spec_pop = spec_on && (P.speculate & 8) != 0;
     uint32_t my_top = 0;         // owner copy of ColdSeg top
     uint32_t hi = 0;             // ColdSeg chunks [.., hi) mapped by this warp
     bool active = false;
@@ -622,13 +629,14 @@ __global__ void __launch_bounds__(32 * WMAX, 1) dfs_persistent_kernel(const KPar
             const bool pf = valid && lane < kPfLanes;
             const uint32_t prs = ld_nc_if(pf, P.rp + nb, 0u), pre = ld_nc_if(pf, P.rp + nb + 1, 0u);
             bool cand = valid && !((word >> (nb & 31)) & 1u) && lane != sk;   // sk is claimed either way
+            int cnb = (int)kFull;
+            if (spec_early) cnb = (int)ld_nc_if(vb != 0 && s_rs + lane < s_re, P.col + s_rs + lane, kFull);
             s_old = __shfl_sync(kFull, s_old, 0);
             bool won = vb != 0 && !(s_old & (1u << (sv & 31)));
             uint32_t v = sv, vrs = s_rs, vre = s_re;
             int kpos = sk;
-            int cnb = (int)kFull;
             if (won) {
-                cnb = (int)ld_nc_if(vrs + lane < vre, P.col + vrs + lane, kFull);
+                if (!spec_early) cnb = (int)ld_nc_if(vrs + lane < vre, P.col + vrs + lane, kFull);
             } else {
                 if (STATS && vb && lane == 0) ++cnt[kCntFailedClaims];
                 // claim the first unvisited candidate in CSR order; on a lost race try the next
@@ -661,7 +669,7 @@ __global__ void __launch_bounds__(32 * WMAX, 1) dfs_persistent_kernel(const KPar
                 }
                 st_global_if(lane == 0, P.parent + v, (int32_t)u);             // Alg 1 l.10
                 par = u;
-                u = v; i = vrs; end = vre; spec_ok = true;
+                u = v; i = vrs; end = vre; spec_ok = spec_on;
                 nbv[0] = cnb; win_lanes = 32;                          // have_win stays true
             } else {
                 i += 32u;
@@ -672,6 +680,7 @@ __global__ void __launch_bounds__(32 * WMAX, 1) dfs_persistent_kernel(const KPar
                     have_win = false;                             // i >= end: Alg 1 l.14: pop
                     has_top = pop(u, i);
                     need_end = true;
+                    spec_ok = spec_pop; par = kFull;
                 }
             }
           } else {
@@ -722,7 +731,7 @@ __global__ void __launch_bounds__(32 * WMAX, 1) dfs_persistent_kernel(const KPar
             // its row_ptr pair are issued before the probes
             int sk = -1, se = 0;
             uint32_t sv = 0, s_old = 0, s_rs = 0, s_re = 0;
-            if ((P.speculate == 1 || (P.speculate == 2 && VEC == 1)) && spec_ok) {
+            if (spec_ok) {
                 uint32_t vm = 0;
 #pragma unroll
                 for (int e = 0; e < VEC; ++e) {
@@ -787,7 +796,7 @@ __global__ void __launch_bounds__(32 * WMAX, 1) dfs_persistent_kernel(const KPar
                 }
                 if (lane == 0) P.parent[v] = (int32_t)u;                            // Alg 1 l.10
                 par = u;
-                u = v; i = vrs; end = vre; have_win = true; need_end = false; spec_ok = true;
+                u = v; i = vrs; end = vre; have_win = true; need_end = false; spec_ok = spec_on;
                 win_lanes = 32;
 #pragma unroll
                 for (int f = 0; f < VEC; ++f) nbv[f] = cnb[f];
@@ -856,6 +865,7 @@ __global__ void __launch_bounds__(32 * WMAX, 1) dfs_persistent_kernel(const KPar
                     have_win = false;                             // i >= end: Alg 1 l.14: pop
                     has_top = pop(u, i);
                     need_end = true;
+                    spec_ok = spec_pop; par = kFull;
                 }
             }
           }   // generic step
@@ -900,6 +910,7 @@ __global__ void __launch_bounds__(32 * WMAX, 1) dfs_persistent_kernel(const KPar
         if (refill() > 0) {
             has_top = pop(u, i);
             need_end = true; have_win = false;
+            spec_ok = spec_pop; par = kFull;
             continue;
         }
 
@@ -1111,6 +1122,7 @@ __global__ void __launch_bounds__(32 * WMAX, 1) dfs_persistent_kernel(const KPar
         active = true;
         has_top = pop(u, i);
         need_end = true; have_win = false;
+        spec_ok = spec_pop; par = kFull;
     }
 exit_loop:
     __syncwarp();

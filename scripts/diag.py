@@ -103,6 +103,9 @@ VARIANTS = {
     "bmax512": dict(backoff_max_ns=512),
     "bmax8k": dict(backoff_max_ns=8192),
     "early": dict(speculate=6),
+    "specpop": dict(speculate=10),
+    "specboth": dict(speculate=14),
+    "specpop128": dict(speculate=9, window=128),
     "pf2": dict(prefetch_lines=2),
     "pf4": dict(prefetch_lines=4),
     "pf8": dict(prefetch_lines=8),
