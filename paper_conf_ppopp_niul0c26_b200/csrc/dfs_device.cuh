@@ -26,8 +26,10 @@
 //     {top,bottom} word and copied into the thief's HotRing.
 //   * demand-driven spill (B200 addition): when many warps are idle, a busy warp
 //     moves the oldest half of a deep HotRing to its ColdSeg so other blocks can steal it.
-//   * global termination (unspecified in the paper, reading S13): a busy counter of warps that
-//     hold work plus registered thieves; the atomic that brings it to 0 raises `done`.
+//   * global termination (unspecified in the paper, reading S13): hierarchical busy counters — a
+//     shared-memory count per block of warps that hold work plus registered thieves, and a global
+//     count of blocks whose local count is non-zero (changed only on the local 0<->1
+//     transitions); the global atomic that brings it to 0 raises `done`.
 //
 // Memory-ordering notes: CTA-scope release (MEMBAR.ALL.CTA) publishes HotRing
 // entries; CTA-scope acquire is free.  GPU-scope publication of ColdSeg data uses
@@ -50,7 +52,7 @@ constexpr int kStatusETIMEOUT = -5;
 constexpr int kStatusEINTERNAL = -6;
 
 struct Ctl {
-    unsigned int busy;                 // warps holding work + registered thieves (S13)
+    unsigned int busy;                 // blocks whose local busy count is non-zero (S13)
     unsigned int done;                 // set once busy reaches 0 (or on error)
     int status;                        // 0 or a negative dfs_status
     unsigned int pool_bump;            // bump allocator over the chunk pool
@@ -89,7 +91,7 @@ struct KParams {
     int inter_any;                           // any idle warp may steal inter-block (else leader of an idle block)
     unsigned int backoff_max_ns;             // idle-loop exponential backoff cap
     unsigned int backoff_min_ns;             // ... and first step
-    unsigned int* timeline;                  // optional: busy-warp samples (block 0 / warp 0)
+    unsigned int* timeline;                  // optional: busy-block samples (block 0 / warp 0)
     unsigned int timeline_len;
     unsigned int timeline_dt_ns;
     unsigned long long timeout_ns;
@@ -227,6 +229,7 @@ struct SmemCtl {
     volatile uint32_t tailf[kMaxWarps];    // 16-bit: slots below tailf are free for reuse
     uint32_t lock[kMaxWarps];              // per-warp lock for tail-side ops (thieves, flush)
     unsigned int warp_mask;                // 1 = warp active
+    unsigned int lbusy;                    // warps of this block holding work + registered thieves
     volatile int done;                     // block-local copy of ctl->done
     uint32_t inter_token;                  // one idle warp per block scans other blocks at a time
     unsigned long long cnt[kMaxWarps][kNumCounters]; // per-warp stats counters (collect_stats)
@@ -311,7 +314,10 @@ __global__ void __launch_bounds__(32 * WMAX, 1) dfs_persistent_kernel(const KPar
     if (threadIdx.x < kMaxWarps) {
         S.ht[threadIdx.x] = 0; S.tailf[threadIdx.x] = 0; S.lock[threadIdx.x] = 0;
     }
-    if (threadIdx.x == 0) { S.warp_mask = (blockIdx.x == 0) ? 1u : 0u; S.done = 0; S.inter_token = 0; }
+    if (threadIdx.x == 0) {
+        S.warp_mask = (blockIdx.x == 0) ? 1u : 0u; S.done = 0; S.inter_token = 0;
+        S.lbusy = (blockIdx.x == 0) ? 1u : 0u;        // block 0 / warp 0 holds the root (ctl->busy = 1)
+    }
     unsigned long long* const cnt = S.cnt[w];     // lane 0 updates its warp's counters
     if (STATS && lane < kNumCounters) cnt[lane] = 0;
     __syncthreads();
@@ -561,11 +567,24 @@ __global__ void __launch_bounds__(32 * WMAX, 1) dfs_persistent_kernel(const KPar
     auto set_done_local = [&]() {
         if (lane == 0) S.done = 1;
     };
+    // termination counters (reading S13), lane 0 only.  A warp registers BEFORE it reserves
+    // stolen work and deregisters when it holds none; the block's count going 0->1 / 1->0 adds /
+    // removes the block from the global count.  When a count goes 0->1 the registering warp is an
+    // inter-block thief whose victim's block is still counted, so the global count cannot reach 0
+    // while any entry exists; the global increment's result is consumed before the reservation
+    // is attempted (completion order).
+    auto register_thief = [&]() {
+        if (atomicAdd(&S.lbusy, 1u) == 0u) {
+            if (atomicAdd(&P.ctl->busy, 1u) == 0xFFFFFFFFu) raise_error(P, kStatusEINTERNAL);
+        }
+    };
     auto deregister = [&]() {      // lane 0: leave the busy count; the last one raises done
-        if (atomicSub(&P.ctl->busy, 1u) == 1u) { atomicExch(&P.ctl->done, 1u); S.done = 1; }
+        if (atomicSub(&S.lbusy, 1u) == 1u) {
+            if (atomicSub(&P.ctl->busy, 1u) == 1u) { atomicExch(&P.ctl->done, 1u); S.done = 1; }
+        }
     };
 
-    // diagnostics: block 0 / warp 0 samples the busy counter every timeline_dt_ns
+    // diagnostics: block 0 / warp 0 samples the busy-block counter every timeline_dt_ns
     unsigned int tl_next = 0;
     auto sample = [&]() {
         if (P.timeline && blockIdx.x == 0 && w == 0 && lane == 0) {
@@ -884,8 +903,9 @@ __global__ void __launch_bounds__(32 * WMAX, 1) dfs_persistent_kernel(const KPar
                 if (lane == 0) {
                     const uint32_t rest = (my_head - ht_tail(ld_acquire_cta(&S.ht[w]))) & 0xFFFFu;
                     if (rest >= 2u * (uint32_t)P.cold_cutoff) {
-                        const uint32_t busy = *(volatile unsigned int*)&P.ctl->busy;
-                        if ((int)(gridDim.x * W - busy) >= P.spill_idle) want = rest / 2;
+                        // idle warps elsewhere ~ W x (blocks with no busy warp)
+                        const uint32_t busy_blocks = *(volatile unsigned int*)&P.ctl->busy;
+                        if ((int)((gridDim.x - busy_blocks) * W) >= P.spill_idle) want = rest / 2;
                     }
                 }
                 want = __shfl_sync(kFull, want, 0);
@@ -950,8 +970,8 @@ __global__ void __launch_bounds__(32 * WMAX, 1) dfs_persistent_kernel(const KPar
                     if (STATS && lane == 0) ++cnt[kCntStealAttempts];
                     uint32_t ok = 0, t = 0, kst = 0;
                     if (lane == 0) {
-                        atomicAdd(&P.ctl->busy, 1u);                 // register before reserving
                         if (smem_trylock(&S.lock[vwarp])) {
+                            register_thief();                        // before reserving
                             uint32_t old = *(volatile uint32_t*)&S.ht[vwarp];
                             for (int tries = 0; tries < 8; ++tries) {
                                 const int r = ht_rest(old);
@@ -966,9 +986,8 @@ __global__ void __launch_bounds__(32 * WMAX, 1) dfs_persistent_kernel(const KPar
                                 if (got == old) { ok = 1; break; }
                                 old = got;
                             }
-                            if (!ok) smem_unlock(&S.lock[vwarp]);
+                            if (!ok) { smem_unlock(&S.lock[vwarp]); deregister(); }
                         }
-                        if (!ok) deregister();
                     }
                     ok = __shfl_sync(kFull, ok, 0);
                     if (ok) {
@@ -1051,7 +1070,7 @@ __global__ void __launch_bounds__(32 * WMAX, 1) dfs_persistent_kernel(const KPar
                         if (STATS && lane == 0) ++cnt[kCntStealAttempts];
                         uint32_t ok = 0, bot = 0, kst = 0;
                         if (lane == 0) {
-                            atomicAdd(&P.ctl->busy, 1u);
+                            register_thief();
                             unsigned long long old = ld_relaxed_u64(&P.cold_tb[vwg]);
                             for (int tries = 0; tries < 4; ++tries) {
                                 const uint32_t top = (uint32_t)(old >> 32), b = (uint32_t)old;
