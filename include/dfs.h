@@ -103,11 +103,10 @@ typedef struct dfs_options {
     int32_t pub_batch;       /* the owner publishes its HotRing head to thieves every pub_batch
                                 pushes (entries above it are private); default 1                    */
     int32_t speculate;       /* bits 0-1: 1 = claim a freshly descended child's first non-parent
-                                neighbour in parallel with the visited probes; 0 = off; 2 (default)
-                                = on for 32-wide windows only; default 2|8.  bit 2: issue that child's first
-                                window before the claim returns.  bit 3: also claim a popped
-                                entry's next position speculatively (its probe saw it unvisited
-                                when the entry was pushed)                                          */
+                                neighbour in parallel with the visited probes; 0 = off; 2 = on for
+                                32-wide windows only.  bit 3: also claim a popped entry's next
+                                position speculatively (its probe saw it unvisited when the entry
+                                was pushed).  Default 2|8                                          */
     int32_t steal_half;      /* 1 (default): a thief takes max(h_s, rest/2) <= 32 HotRing entries
                                 (resp. max(c_s, rest/2) <= 64 ColdSeg entries); 0: exactly h_s/c_s
                                 as in Alg 3/4                                                       */
@@ -123,7 +122,11 @@ typedef struct dfs_options {
                                 whole pool); exhausting it returns DFS_ENOMEM                      */
     int32_t reserved0;       /* must be 0 (was eager_siblings: claiming every later unvisited
                                 neighbour of a window at once — measured slower, removed)          */
-    int32_t reserved[7];     /* zero                                                              */
+    int32_t leaf_skip;       /* 1 (default): a claimed child whose list is empty or holds only its
+                                parent is finished in place — Alg 1 would descend and pop straight
+                                back — so the parent's window scan continues without a push/pop
+                                round trip; 0: always descend                                      */
+    int32_t reserved[6];     /* zero                                                              */
 } dfs_options;
 
 typedef struct dfs_stats {

@@ -22,7 +22,8 @@ def build(force: bool = False, verbose: bool = False) -> str:
     newest = max(os.path.getmtime(p) for p in _deps())
     if force or not os.path.exists(SO) or os.path.getmtime(SO) < newest:
         tmp = SO + f".tmp{os.getpid()}"
-        cmd = [NVCC, *FLAGS, *SOURCES, "-o", tmp]
+        extra = os.environ.get("DFS_NVCC_EXTRA", "").split()      # A/B builds (e.g. -DDFS_KRING=128)
+        cmd = [NVCC, *FLAGS, *extra, *SOURCES, "-o", tmp]
         r = subprocess.run(cmd, capture_output=True, text=True)
         if r.returncode != 0:
             raise RuntimeError("nvcc failed:\n" + r.stdout + r.stderr)

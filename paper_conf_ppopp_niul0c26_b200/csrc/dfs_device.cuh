@@ -100,6 +100,7 @@ struct KParams {
     int speculate;                           // speculative claim of the child's first neighbour
     int steal_half;                          // steal max(h_s, rest/2) (resp. c_s) entries
     uint32_t ring_cap;                       // usable HotRing entries (<= H); 2 ~ one-level stack (v1)
+    int leaf_skip;                           // claim children whose list is empty or [parent] in place
     unsigned long long* block_claims;        // optional: claims per block (Fig 9 task counts)
 };
 
@@ -123,12 +124,6 @@ __device__ __forceinline__ int ld_relaxed_s32(const int* p) {
 }
 __device__ __forceinline__ void st_relaxed_u32(uint32_t* p, uint32_t v) {
     asm volatile("st.relaxed.gpu.global.u32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
-}
-// SM clock read that waits for `dep` to be ready (scoreboard dependency on the asm input)
-__device__ __forceinline__ long long clock_after(uint32_t dep) {
-    long long t;
-    asm volatile("mov.u64 %0, %%clock64;" : "=l"(t) : "r"(dep) : "memory");
-    return t;
 }
 __device__ __forceinline__ unsigned long long globaltimer() {
     unsigned long long t;
@@ -336,12 +331,11 @@ __global__ void __launch_bounds__(32 * WMAX, 1) dfs_persistent_kernel(const KPar
     bool spec_ok = false;        // speculative claim allowed on the current window (fresh child,
                                  // or a popped entry with speculate & 8)
     uint32_t par = kFull;        // parent of u when spec_ok (kFull: no position to skip)
-    // speculate: bits 0-1 = mode (0 off, 1 on, 2 on for 32-wide windows), bit 2 = issue the
-    // child's first window before the claim returns (32-wide), bit 3 = also claim a popped
-    // entry's next position speculatively (its probe at push time saw it unvisited)
+    // speculate: bits 0-1 = mode (0 off, 1 on, 2 on for 32-wide windows), bit 3 = also claim a
+    // popped entry's next position speculatively (its probe at push time saw it unvisited)
     const bool spec_on = (P.speculate & 3) == 1 || ((P.speculate & 3) == 2 && VEC == 1);
-    const bool spec_early = (P.speculate & 4) != 0;
     const bool spec_pop = spec_on && (P.speculate & 8) != 0;
+    const uint32_t leaf_deg = P.leaf_skip ? 1u : 0u;   // children of degree <= this may be leaves
     uint32_t my_top = 0;         // owner copy of ColdSeg top
     uint32_t hi = 0;             // ColdSeg chunks [.., hi) mapped by this warp
     bool active = false;
@@ -349,7 +343,6 @@ __global__ void __launch_bounds__(32 * WMAX, 1) dfs_persistent_kernel(const KPar
     if (rng == 0) rng = 1;
     const unsigned long long t_start = globaltimer();
     unsigned long long t_idle0 = 0;
-    long long tc_prev = 0;                       // STATS: end of the previous expansion step
     uint32_t iter = 0;
     unsigned long long my_claims = 0;            // for P.block_claims (Fig 9 task distribution)
     unsigned long long tl_reported = 0;          // timeline diagnostics
@@ -370,7 +363,7 @@ __global__ void __launch_bounds__(32 * WMAX, 1) dfs_persistent_kernel(const KPar
             if (ld) x = __ldg(reinterpret_cast<const int4*>(P.col + q));    // col padded
             nb[0] = x.x; nb[1] = x.y; nb[2] = x.z; nb[3] = x.w;
         } else {
-            nb[0] = ld ? __ldg(P.col + q) : -1;
+            nb[0] = (int)ld_nc_if(ld, P.col + q, kFull);
         }
     };
     // lanes of the current window that hold data (the rest are loaded on demand)
@@ -649,13 +642,12 @@ __global__ void __launch_bounds__(32 * WMAX, 1) dfs_persistent_kernel(const KPar
             const uint32_t prs = ld_nc_if(pf, P.rp + nb, 0u), pre = ld_nc_if(pf, P.rp + nb + 1, 0u);
             bool cand = valid && !((word >> (nb & 31)) & 1u) && lane != sk;   // sk is claimed either way
             int cnb = (int)kFull;
-            if (spec_early) cnb = (int)ld_nc_if(vb != 0 && s_rs + lane < s_re, P.col + s_rs + lane, kFull);
             s_old = __shfl_sync(kFull, s_old, 0);
             bool won = vb != 0 && !(s_old & (1u << (sv & 31)));
             uint32_t v = sv, vrs = s_rs, vre = s_re;
             int kpos = sk;
             if (won) {
-                if (!spec_early) cnb = (int)ld_nc_if(vrs + lane < vre, P.col + vrs + lane, kFull);
+                cnb = (int)ld_nc_if(vrs + lane < vre, P.col + vrs + lane, kFull);
             } else {
                 if (STATS && vb && lane == 0) ++cnt[kCntFailedClaims];
                 // claim the first unvisited candidate in CSR order; on a lost race try the next
@@ -671,10 +663,12 @@ __global__ void __launch_bounds__(32 * WMAX, 1) dfs_persistent_kernel(const KPar
                     old = __shfl_sync(kFull, old, 0);
                     if (!(old & bit)) { won = true; v = cv; vrs = crs; vre = cre; kpos = k; break; }
                     if (STATS && lane == 0) ++cnt[kCntFailedClaims];
-                    if (lane == k) cand = false;                      // lost the race: next candidate
+                    if (lane == k) cand = false;                  // lost the race: next candidate
                     any = __ballot_sync(kFull, cand);
                 }
             }
+            uint32_t next_i = i + 32u;                            // u's scan resumes here
+            bool advance = !won;
             if (won) {
                 // descend (Alg 1 l.8-11): push <u, next candidate> unless u is exhausted —
                 // positions whose probe saw a claimed target stay claimed, so skipping them keeps
@@ -683,18 +677,33 @@ __global__ void __launch_bounds__(32 * WMAX, 1) dfs_persistent_kernel(const KPar
                 ++my_claims;
                 const uint32_t later = __ballot_sync(kFull, cand && lane > kpos);
                 const uint32_t ni = later ? i + (uint32_t)(__ffs(later) - 1) : i + 32u;
-                if (ni < end) {
-                    if (!push_lean(u, ni)) goto exit_loop;
-                }
                 st_global_if(lane == 0, P.parent + v, (int32_t)u);             // Alg 1 l.10
-                par = u;
-                u = v; i = vrs; end = vre; spec_ok = spec_on;
-                nbv[0] = cnb; win_lanes = 32;                          // have_win stays true
-            } else {
-                i += 32u;
-                spec_ok = false;
-                if (have_nxt) {                                   // next window already loaded
+                // leaf skip: v's list is empty or exactly [u] — Alg 1 would descend, find
+                // nothing unvisited and pop straight back to <u, ni>; stay on u instead
+                if (vre - vrs <= leaf_deg && (vre == vrs || (uint32_t)__shfl_sync(kFull, cnb, 0) == u)) {
+                    next_i = ni; advance = true;
+                } else {
+                    if (ni < end) {
+                        if (!push_lean(u, ni)) goto exit_loop;
+                    }
+                    par = u;
+                    u = v; i = vrs; end = vre; spec_ok = spec_on;
+                    nbv[0] = cnb; win_lanes = 32;                      // have_win stays true
+                }
+            }
+            if (advance) {
+                // continue u's scan at next_i: shift the window down when it still overlaps
+                // (leaf skip), take the prefetched next window, or pop when u is exhausted
+                const uint32_t d = next_i - i;
+                i = next_i;
+                if (i < end && d < 32u) {
+                    int x = __shfl_down_sync(kFull, nb, d);
+                    const int y = (int)ld_nc_if(lane >= 32 - (int)d && i + lane < end, P.col + i + lane, kFull);
+                    nbv[0] = lane >= 32 - (int)d ? y : x;
+                    spec_ok = spec_on; par = kFull;               // next position: claim at once
+                } else if (have_nxt) {                            // next window already loaded
                     nbv[0] = nxt1;
+                    spec_ok = false;
                 } else {
                     have_win = false;                             // i >= end: Alg 1 l.14: pop
                     has_top = pop(u, i);
@@ -703,183 +712,178 @@ __global__ void __launch_bounds__(32 * WMAX, 1) dfs_persistent_kernel(const KPar
                 }
             }
           } else {
-            // ===== warp-level expansion step (Alg 1 l.5-12 over one window) =====
+            // ===== lean expansion step (Alg 1 l.5-12 over one window) =====
             // Window = positions [a, a + kWin), a = i rounded down to a multiple of VEC; lane k
-            // holds positions a+VEC*k .. a+VEC*k+VEC-1 (col_idx entries).  Positions outside
+            // holds positions a+VEC*k .. a+VEC*k+VEC-1 (col_idx entries); positions outside
             // [i, end) are masked.  A popped entry's window is fetched together with its end
-            // offset for the first kHeadLanes lanes, and completed only if the list is longer.
-            if (!have_win) {
-                const uint32_t a0 = i & ~(uint32_t)(VEC - 1);
-                if (need_end) {                                   // popped entry: end unknown
-                    const uint32_t e2 = __ldg(P.rp + u + 1);
-                    load_window(a0, P.m, kHeadLanes, nbv);
-                    win_lanes = kHeadLanes;
-                    end = e2; need_end = false;
-                } else {
-                    load_window(a0, end, 32, nbv);
-                    win_lanes = 32;
+            // offset for the first kHeadLanes lanes and completed only if the list is longer.
+            // The common case — a claim that wins — runs without lane-0 branches: the claim, the
+            // parent store, the ring store and the publication are predicated instructions.
+            const uint32_t a = i & ~(uint32_t)(VEC - 1);
+            if (!have_win || win_lanes < 32) {
+                if (!have_win) {
+                    if (need_end) {                                   // popped entry: end unknown
+                        const uint32_t e2 = __ldg(P.rp + u + 1);
+                        load_window(a, P.m, kHeadLanes, nbv);
+                        win_lanes = kHeadLanes;
+                        end = e2; need_end = false;
+                    } else {
+                        load_window(a, end, 32, nbv);
+                        win_lanes = 32;
+                    }
+                    have_win = true;
                 }
-            }
-            {
-                const uint32_t a0 = i & ~(uint32_t)(VEC - 1);
-                if (win_lanes < 32 && end > a0 + (uint32_t)VEC * (uint32_t)win_lanes) {
-                    int tnb[VEC];
-                    load_window(a0, end, 32, tnb, win_lanes);
-                    if (lane >= win_lanes) {
+                if (win_lanes < 32) {
+                    if (end > a + (uint32_t)VEC * (uint32_t)win_lanes) {
+                        int tnb[VEC];
+                        load_window(a, end, 32, tnb, win_lanes);
+                        if (lane >= win_lanes) {
 #pragma unroll
-                        for (int f = 0; f < VEC; ++f) nbv[f] = tnb[f];
+                            for (int f = 0; f < VEC; ++f) nbv[f] = tnb[f];
+                        }
                     }
                     win_lanes = 32;
                 }
             }
             if (STATS && lane == 0) ++cnt[kCntWindows];
-            long long tc0 = 0, tc1 = 0;
-            if (STATS) {
-                tc0 = clock_after(0u);
-                if (lane == 0 && tc_prev) { cnt[kCntTOut] += tc0 - tc_prev; ++cnt[kCntOutIters]; }
-                tc1 = clock_after((uint32_t)nbv[0] ^ end);
-            }
-            const uint32_t a = i & ~(uint32_t)(VEC - 1);
             const uint32_t q0 = a + (uint32_t)VEC * lane;
+            uint32_t vm = 0;                                      // valid elements of this lane
+#pragma unroll
+            for (int e = 0; e < VEC; ++e)
+                if (q0 + e >= i && q0 + e < end) vm |= 1u << e;
             // long list (hubs): the next window is in flight while this one's probes resolve
-            int nxt[VEC];
             const bool have_nxt = a + kWin < end;
+            int nxt[VEC];
+#pragma unroll
+            for (int e = 0; e < VEC; ++e) nxt[e] = -1;
             if (have_nxt) load_window(a + kWin, end, 32, nxt);
-            // speculative claim (fresh child only): the first position whose neighbour is not the
-            // parent we came from is, if unvisited, exactly Alg 1's next tree edge; its claim and
-            // its row_ptr pair are issued before the probes
-            int sk = -1, se = 0;
-            uint32_t sv = 0, s_old = 0, s_rs = 0, s_re = 0;
+            // speculative claim: the first valid position whose neighbour is not the parent we
+            // came from (par = kFull: none to skip) is, if unvisited, exactly Alg 1's next tree
+            // edge; its claim and row_ptr pair are issued before the probes
+            uint32_t sm = 0;
             if (spec_ok) {
-                uint32_t vm = 0;
 #pragma unroll
-                for (int e = 0; e < VEC; ++e) {
-                    const uint32_t p = q0 + e;
-                    if (p >= i && p < end && (uint32_t)nbv[e] != par) vm |= 1u << e;
-                }
-                const uint32_t vb = __ballot_sync(kFull, vm != 0);
-                if (vb) {
-                    sk = __ffs(vb) - 1;
-                    if constexpr (VEC == 1) {
-                        se = 0;
-                        sv = (uint32_t)__shfl_sync(kFull, nbv[0], sk);
-                    } else {
-                        se = __ffs(__shfl_sync(kFull, vm, sk)) - 1;
-                        int pick = nbv[0];
+                for (int e = 0; e < VEC; ++e)
+                    if (((vm >> e) & 1u) && (uint32_t)nbv[e] != par) sm |= 1u << e;
+            }
+            const uint32_t vb = __ballot_sync(kFull, sm != 0);
+            const int sk = __ffs(vb) - 1;
+            int se = 0;
+            uint32_t sv = u;
+            if (vb) {
+                if constexpr (VEC == 1) {
+                    sv = (uint32_t)__shfl_sync(kFull, nbv[0], sk);
+                } else {
+                    se = __ffs(__shfl_sync(kFull, sm, sk)) - 1;
+                    int pick = nbv[0];
 #pragma unroll
-                        for (int f = 1; f < VEC; ++f) if (se == f) pick = nbv[f];
-                        sv = (uint32_t)__shfl_sync(kFull, pick, sk);
-                    }
-                    if (lane == 0) s_old = atomicOr(P.bitmap + (sv >> 5), 1u << (sv & 31));
-                    s_rs = __ldg(P.rp + sv); s_re = __ldg(P.rp + sv + 1);
+                    for (int f = 1; f < VEC; ++f) if (se == f) pick = nbv[f];
+                    sv = (uint32_t)__shfl_sync(kFull, pick, sk);
                 }
             }
-            // probe the visited bits; the lanes holding the first 8 positions also prefetch their
-            // candidates' row_ptr pairs, so a claim can load the child's window immediately
-            uint32_t m4 = 0;
+            uint32_t s_old = atom_or_if(vb != 0 && lane == 0, P.bitmap + (sv >> 5), 1u << (sv & 31));
+            const uint32_t s_rs = ld_nc_if(vb != 0, P.rp + sv, 0u), s_re = ld_nc_if(vb != 0, P.rp + sv + 1, 0u);
+            // probe the visited bits; the lanes holding the first 8 positions also prefetch
+            // their candidates' row_ptr pairs
+            uint32_t cm = 0;                                      // unvisited candidates
             uint32_t prs[VEC], pre[VEC];
 #pragma unroll
             for (int e = 0; e < VEC; ++e) {
-                const uint32_t p = q0 + e;
-                const int x = nbv[e];
-                prs[e] = 0; pre[e] = 0;
-                if (p >= i && p < end) {
-                    const uint32_t word = __ldcg(P.bitmap + ((uint32_t)x >> 5));
-                    if (lane < kPfLanes) { prs[e] = __ldg(P.rp + x); pre[e] = __ldg(P.rp + x + 1); }
-                    if (!((word >> (x & 31)) & 1u)) m4 |= 1u << e;
-                }
+                const bool ok = (vm >> e) & 1u;
+                const uint32_t x = (uint32_t)nbv[e];
+                const uint32_t word = ld_cg_if(ok, P.bitmap + (x >> 5), kFull);
+                const bool pf = ok && lane < kPfLanes;
+                prs[e] = ld_nc_if(pf, P.rp + x, 0u); pre[e] = ld_nc_if(pf, P.rp + x + 1, 0u);
+                if (ok && !((word >> (x & 31)) & 1u)) cm |= 1u << e;
             }
-            bool descended = false;
-            long long tc2 = 0, tc3 = 0;
-            if (STATS) { tc2 = clock_after(m4); tc3 = tc2; }
+            if (lane == sk) cm &= ~(1u << se);                    // claimed either way
+            s_old = __shfl_sync(kFull, s_old, 0);
+            bool won = vb != 0 && !(s_old & (1u << (sv & 31)));
+            if (STATS && vb && !won && lane == 0) ++cnt[kCntFailedClaims];
+            uint32_t v = sv, vrs = s_rs, vre = s_re;
+            int kl = sk, ke = se;                                 // window slot of v
             int cnb[VEC];
-            // descend into the child claimed at window slot (k, e): push <u, next candidate>
-            // (Alg 1 l.8 + l.11) unless u is exhausted — positions whose probe saw a claimed target
-            // stay claimed (claims are monotone), so rescanning them cannot change anything —
-            // then make v the register top with its first window (cnb) loaded
-            auto descend = [&](int k, int e, uint32_t v, uint32_t vrs, uint32_t vre) -> bool {
+            if (won) load_window(vrs & ~(uint32_t)(VEC - 1), vre, 32, cnb);
+            for (;;) {
+                if (won) {
+                    // leaf skip: v's list is empty or exactly [u] — Alg 1 would descend, find
+                    // nothing unvisited and pop straight back to <u, next>; record the tree edge
+                    // and go on with u's window (its probes are still valid: claims are monotone)
+                    bool leaf = vre == vrs;
+                    if (P.leaf_skip && vre == vrs + 1u) {
+                        int first = cnb[0];
+                        if constexpr (VEC > 1) {
+#pragma unroll
+                            for (int f = 1; f < VEC; ++f) if ((int)(vrs & (VEC - 1)) == f) first = cnb[f];
+                        }
+                        leaf = (uint32_t)__shfl_sync(kFull, first, 0) == u;
+                    }
+                    if (!(leaf && P.leaf_skip)) break;
+                    st_global_if(lane == 0, P.parent + v, (int32_t)u);     // Alg 1 l.10
+                    ++my_claims;
+                    if (STATS && lane == 0) ++cnt[kCntClaims];
+                    won = false;
+                    // only candidates after v's slot remain (those before it were taken)
+                    cm = lane > kl ? cm : (lane == kl ? (cm & ~((2u << ke) - 1u)) : 0u);
+                }
+                // claim the first unvisited candidate in CSR order; on a lost race, the next
+                const uint32_t any = __ballot_sync(kFull, cm != 0);
+                if (!any) break;
+                const int k = __ffs(any) - 1;
+                int e = 0;
+                int mine_nb = nbv[0];
+                uint32_t mine_rs = prs[0], mine_re = pre[0];
+                if constexpr (VEC > 1) {
+                    e = __ffs(__shfl_sync(kFull, cm, k)) - 1;
+#pragma unroll
+                    for (int f = 1; f < VEC; ++f)
+                        if (e == f) { mine_nb = nbv[f]; mine_rs = prs[f]; mine_re = pre[f]; }
+                }
+                const uint32_t cv = (uint32_t)__shfl_sync(kFull, mine_nb, k);
+                uint32_t crs = __shfl_sync(kFull, mine_rs, k & (kPfLanes - 1));
+                uint32_t cre = __shfl_sync(kFull, mine_re, k & (kPfLanes - 1));
+                if (k >= kPfLanes) { crs = __ldg(P.rp + cv); cre = __ldg(P.rp + cv + 1); }
+                const uint32_t bit = 1u << (cv & 31);
+                uint32_t old = atom_or_if(lane == 0, P.bitmap + (cv >> 5), bit);
+                load_window(crs & ~(uint32_t)(VEC - 1), cre, 32, cnb);   // overlaps the claim
+                old = __shfl_sync(kFull, old, 0);
+                if (!(old & bit)) { won = true; v = cv; vrs = crs; vre = cre; kl = k; ke = e; continue; }
+                if (STATS && lane == 0) ++cnt[kCntFailedClaims];
+                if (lane == k) cm &= ~(1u << e);                  // lost the race: next candidate
+            }
+            if (won) {
+                // descend (Alg 1 l.8-11): push <u, next candidate> unless u is exhausted —
+                // positions whose probe saw a claimed target stay claimed, so skipping them keeps
+                // Alg 1's order — then v becomes the register top with its first window loaded
                 if (STATS && lane == 0) ++cnt[kCntClaims];
                 ++my_claims;
+                const uint32_t mine = lane > kl ? cm : (lane == kl ? (cm & ~((2u << ke) - 1u)) : 0u);
+                const uint32_t later = __ballot_sync(kFull, mine != 0);
                 uint32_t ni = a + kWin;
-                {
-                    const uint32_t mine = (lane == k) ? (m4 & ~((2u << e) - 1u)) : (lane > k ? m4 : 0u);
-                    const uint32_t later = __ballot_sync(kFull, mine != 0);
-                    if (later) {
-                        const int k2 = __ffs(later) - 1;
+                if (later) {
+                    const int k2 = __ffs(later) - 1;
+                    if constexpr (VEC == 1) {
+                        ni = a + (uint32_t)k2;
+                    } else {
                         const uint32_t m2 = __shfl_sync(kFull, mine, k2);
                         ni = a + (uint32_t)VEC * (uint32_t)k2 + (uint32_t)(__ffs(m2) - 1);
                     }
                 }
                 if (ni < end) {
-                    if (!push(u, ni)) return false;
+                    if (!push_lean(u, ni)) goto exit_loop;
                 }
-                if (lane == 0) P.parent[v] = (int32_t)u;                            // Alg 1 l.10
+                st_global_if(lane == 0, P.parent + v, (int32_t)u);             // Alg 1 l.10
                 par = u;
-                u = v; i = vrs; end = vre; have_win = true; need_end = false; spec_ok = spec_on;
-                win_lanes = 32;
+                u = v; i = vrs; end = vre; spec_ok = spec_on;
+                have_win = true; need_end = false; win_lanes = 32;
 #pragma unroll
                 for (int f = 0; f < VEC; ++f) nbv[f] = cnb[f];
-                descended = true;
-                return true;
-            };
-            if (sk >= 0) {
-                if (lane == sk) m4 &= ~(1u << se);               // p0 is claimed either way
-                s_old = __shfl_sync(kFull, s_old, 0);
-                if (STATS) tc3 = clock_after(s_old);
-                if (!(s_old & (1u << (sv & 31)))) {              // speculative claim won
-                    load_window(s_rs & ~(uint32_t)(VEC - 1), s_re, 32, cnb);
-                    if (!descend(sk, se, sv, s_rs, s_re)) goto exit_loop;
-                } else if (STATS && lane == 0) {
-                    ++cnt[kCntFailedClaims];
-                }
-            }
-            uint32_t any = descended ? 0u : __ballot_sync(kFull, m4 != 0);
-            while (any) {
-                const int k = __ffs(any) - 1;                      // first lane with a candidate
-                int e = 0;
-                int mine_nb = nbv[0];
-                uint32_t mine_rs = prs[0], mine_re = pre[0];
-                if constexpr (VEC > 1) {
-                    e = __ffs(__shfl_sync(kFull, m4, k)) - 1;      // first candidate in CSR order
-#pragma unroll
-                    for (int f = 1; f < VEC; ++f)
-                        if (e == f) { mine_nb = nbv[f]; mine_rs = prs[f]; mine_re = pre[f]; }
-                }
-                const uint32_t v = (uint32_t)__shfl_sync(kFull, mine_nb, k);
-                uint32_t vrs, vre;
-                if (k < kPfLanes) {
-                    vrs = __shfl_sync(kFull, mine_rs, k); vre = __shfl_sync(kFull, mine_re, k);
-                } else {
-                    vrs = __ldg(P.rp + v); vre = __ldg(P.rp + v + 1);
-                }
-                const uint32_t bit = 1u << (v & 31);
-                uint32_t old = 0;
-                if (lane == 0) old = atomicOr(P.bitmap + (v >> 5), bit);          // claim
-                // the child's first window load overlaps the claim
-                load_window(vrs & ~(uint32_t)(VEC - 1), vre, 32, cnb);
-                old = __shfl_sync(kFull, old, 0);
-                if (!(old & bit)) {
-                    if (!descend(k, e, v, vrs, vre)) goto exit_loop;
-                    break;
-                }
-                if (STATS && lane == 0) ++cnt[kCntFailedClaims];
-                if (lane == k) m4 &= ~(1u << e);                  // lost the race: next candidate
-                any = __ballot_sync(kFull, m4 != 0);
-            }
-            if (STATS && lane == 0) {
-                const long long tc4 = clock_after((uint32_t)nbv[0] ^ i);
-                cnt[kCntTWin] += tc1 - tc0; cnt[kCntTProbe] += tc2 - tc1;
-                cnt[kCntTClaim] += tc3 - tc2; cnt[kCntTTail] += tc4 - tc3;
-                tc_prev = tc4;
-            }
-            if (!descended) {
+            } else {
                 i = a + kWin;
                 spec_ok = false;
                 if (have_nxt) {                                   // next window already loaded
 #pragma unroll
                     for (int f = 0; f < VEC; ++f) nbv[f] = nxt[f];
-                    have_win = true;
-                    win_lanes = 32;
                 } else {
                     have_win = false;                             // i >= end: Alg 1 l.14: pop
                     has_top = pop(u, i);
@@ -887,7 +891,7 @@ __global__ void __launch_bounds__(32 * WMAX, 1) dfs_persistent_kernel(const KPar
                     spec_ok = spec_pop; par = kFull;
                 }
             }
-          }   // generic step
+          }   // VEC == 4 step
             ++iter;
             if ((iter & 31u) == 0) {
                 if (P.timeline && lane == 0) {                    // diagnostics: claim progress
@@ -945,7 +949,6 @@ __global__ void __launch_bounds__(32 * WMAX, 1) dfs_persistent_kernel(const KPar
         }
         bool got_work = false;
         uint32_t backoff = P.backoff_min_ns;
-        tc_prev = 0;
         t_idle0 = STATS ? globaltimer() : 0ull;
         while (!got_work) {
             if (__shfl_sync(kFull, S.done, 0)) goto exit_loop;

@@ -180,6 +180,7 @@ void dfs_options_default(dfs_options* o) {
     o->ring_cap = 0;
     o->backoff_min_ns = 32;
     o->max_pool_chunks = 0;
+    o->leaf_skip = 1;
 }
 
 int dfs_last_error(void) { return g_last_error; }
@@ -357,6 +358,7 @@ static int launch_one(dfs_graph* g, Slot& sl, cudaStream_t s, int32_t root, int3
     P.pub_batch = o.pub_batch > 0 ? (uint32_t)o.pub_batch : 1u;
     P.speculate = o.speculate;
     P.steal_half = o.steal_half;
+    P.leaf_skip = o.leaf_skip ? 1 : 0;
     P.ring_cap = (o.ring_cap > 0 && o.ring_cap < kRing) ? (uint32_t)o.ring_cap : (uint32_t)kRing;
     P.block_claims = sl.block_claims;
     const bool tl = g->d_timeline && &sl == &g->slots[0];

@@ -49,7 +49,7 @@ class _Options(ctypes.Structure):
                 ("steal_half", ctypes.c_int32), ("concurrency", ctypes.c_int32),
                 ("ring_cap", ctypes.c_int32), ("backoff_min_ns", ctypes.c_int32),
                 ("max_pool_chunks", ctypes.c_int32), ("reserved0", ctypes.c_int32),
-                ("reserved", ctypes.c_int32 * 7)]
+                ("leaf_skip", ctypes.c_int32), ("reserved", ctypes.c_int32 * 6)]
 
 
 class _Stats(ctypes.Structure):
@@ -94,6 +94,7 @@ class Options:
     ring_cap: Optional[int] = None
     backoff_min_ns: Optional[int] = None
     max_pool_chunks: Optional[int] = None
+    leaf_skip: Optional[bool] = None
 
     def to_c(self) -> _Options:
         o = _Options()

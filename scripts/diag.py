@@ -104,6 +104,8 @@ VARIANTS = {
     "bmax8k": dict(backoff_max_ns=8192),
     "early": dict(speculate=6),
     "specpop": dict(speculate=10),
+    "noleaf": dict(leaf_skip=False),
+    "detnoleaf": dict(deterministic=True, leaf_skip=False),
     "specboth": dict(speculate=14),
     "specpop128": dict(speculate=9, window=128),
     "pf2": dict(prefetch_lines=2),
