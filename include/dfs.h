@@ -122,10 +122,12 @@ typedef struct dfs_options {
                                 whole pool); exhausting it returns DFS_ENOMEM                      */
     int32_t reserved0;       /* must be 0 (was eager_siblings: claiming every later unvisited
                                 neighbour of a window at once — measured slower, removed)          */
-    int32_t leaf_skip;       /* 1 (default): a claimed child whose list is empty or holds only its
-                                parent is finished in place — Alg 1 would descend and pop straight
-                                back — so the parent's window scan continues without a push/pop
-                                round trip; 0: always descend                                      */
+    int32_t leaf_skip;       /* 1: a claimed child whose list is empty or holds only its parent is
+                                finished in place — Alg 1 would descend and pop straight back — so
+                                the parent's window scan continues without a push/pop round trip.
+                                2 (default): in addition, 128-wide windows claim every unvisited
+                                leaf candidate at once (leaf map built at create: out-degree 0, or
+                                1 whose only in-list is its neighbour's).  0: always descend       */
     int32_t reserved[6];     /* zero                                                              */
 } dfs_options;
 

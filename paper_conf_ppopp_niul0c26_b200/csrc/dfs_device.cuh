@@ -71,6 +71,7 @@ struct KParams {
     const uint32_t* __restrict__ rp;         // n+1 (narrowed row_ptr; m < 2^32)
     const int32_t* __restrict__ col;         // m (+8 padding)
     uint32_t* bitmap;                        // ceil(n/32) visited words
+    const uint32_t* __restrict__ leafmap;    // ceil(n/32) leaf bits (create time), or null
     int32_t* parent;                         // n output
     unsigned long long* cold_tb;             // n_warps: (top << 32) | bottom
     uint32_t* chunk_tab;                     // n_warps << tab_log2
@@ -225,6 +226,7 @@ struct SmemCtl {
     uint32_t lock[kMaxWarps];              // per-warp lock for tail-side ops (thieves, flush)
     unsigned int warp_mask;                // 1 = warp active
     unsigned int lbusy;                    // warps of this block holding work + registered thieves
+    unsigned long long t_start;            // globaltimer at kernel start (watchdog, timeline)
     volatile int done;                     // block-local copy of ctl->done
     uint32_t inter_token;                  // one idle warp per block scans other blocks at a time
     unsigned long long cnt[kMaxWarps][kNumCounters]; // per-warp stats counters (collect_stats)
@@ -312,6 +314,7 @@ __global__ void __launch_bounds__(32 * WMAX, 1) dfs_persistent_kernel(const KPar
     if (threadIdx.x == 0) {
         S.warp_mask = (blockIdx.x == 0) ? 1u : 0u; S.done = 0; S.inter_token = 0;
         S.lbusy = (blockIdx.x == 0) ? 1u : 0u;        // block 0 / warp 0 holds the root (ctl->busy = 1)
+        S.t_start = globaltimer();
     }
     unsigned long long* const cnt = S.cnt[w];     // lane 0 updates its warp's counters
     if (STATS && lane < kNumCounters) cnt[lane] = 0;
@@ -341,11 +344,10 @@ __global__ void __launch_bounds__(32 * WMAX, 1) dfs_persistent_kernel(const KPar
     bool active = false;
     uint32_t rng = P.seed ^ (0x9E3779B9u * (uint32_t)(gw + 1));
     if (rng == 0) rng = 1;
-    const unsigned long long t_start = globaltimer();
     unsigned long long t_idle0 = 0;
     uint32_t iter = 0;
-    unsigned long long my_claims = 0;            // for P.block_claims (Fig 9 task distribution)
-    unsigned long long tl_reported = 0;          // timeline diagnostics
+    uint32_t my_claims = 0;                      // for P.block_claims (Fig 9 task distribution)
+    uint32_t tl_reported = 0;                    // timeline diagnostics
 
     if (blockIdx.x == 0 && w == 0) {
         // Alg 1 l.1-3: root claimed by the reset kernel; <root, row_ptr[root]> is our top
@@ -581,7 +583,7 @@ __global__ void __launch_bounds__(32 * WMAX, 1) dfs_persistent_kernel(const KPar
     unsigned int tl_next = 0;
     auto sample = [&]() {
         if (P.timeline && blockIdx.x == 0 && w == 0 && lane == 0) {
-            const unsigned long long now = globaltimer() - t_start;
+            const unsigned long long now = globaltimer() - S.t_start;
             const unsigned int slot = (unsigned int)(now / P.timeline_dt_ns);
             if (slot >= tl_next && slot < P.timeline_len / 2) {
                 P.timeline[slot] = *(volatile unsigned int*)&P.ctl->busy + 1u;   // 0 = no sample
@@ -751,12 +753,11 @@ __global__ void __launch_bounds__(32 * WMAX, 1) dfs_persistent_kernel(const KPar
 #pragma unroll
             for (int e = 0; e < VEC; ++e)
                 if (q0 + e >= i && q0 + e < end) vm |= 1u << e;
-            // long list (hubs): the next window is in flight while this one's probes resolve
+            // long list (hubs): the next window is pulled into L1 while this one's probes
+            // resolve (a prefetch holds no registers; the window is loaded when it is reached)
             const bool have_nxt = a + kWin < end;
-            int nxt[VEC];
-#pragma unroll
-            for (int e = 0; e < VEC; ++e) nxt[e] = -1;
-            if (have_nxt) load_window(a + kWin, end, 32, nxt);
+            if (have_nxt && a + kWin + (uint32_t)VEC * lane < end)
+                asm volatile("prefetch.global.L1 [%0];" ::"l"(P.col + a + kWin + (uint32_t)VEC * lane));
             // speculative claim: the first valid position whose neighbour is not the parent we
             // came from (par = kFull: none to skip) is, if unvisited, exactly Alg 1's next tree
             // edge; its claim and row_ptr pair are issued before the probes
@@ -786,17 +787,42 @@ __global__ void __launch_bounds__(32 * WMAX, 1) dfs_persistent_kernel(const KPar
             // probe the visited bits; the lanes holding the first 8 positions also prefetch
             // their candidates' row_ptr pairs
             uint32_t cm = 0;                                      // unvisited candidates
+            uint32_t lcm = 0;                                     // ... that are leaves
             uint32_t prs[VEC], pre[VEC];
 #pragma unroll
             for (int e = 0; e < VEC; ++e) {
                 const bool ok = (vm >> e) & 1u;
                 const uint32_t x = (uint32_t)nbv[e];
                 const uint32_t word = ld_cg_if(ok, P.bitmap + (x >> 5), kFull);
+                const uint32_t lword = ld_nc_if(ok && P.leafmap != nullptr, P.leafmap + (x >> 5), 0u);
                 const bool pf = ok && lane < kPfLanes;
                 prs[e] = ld_nc_if(pf, P.rp + x, 0u); pre[e] = ld_nc_if(pf, P.rp + x + 1, 0u);
-                if (ok && !((word >> (x & 31)) & 1u)) cm |= 1u << e;
+                if (ok && !((word >> (x & 31)) & 1u)) {
+                    if ((lword >> (x & 31)) & 1u) lcm |= 1u << e; else cm |= 1u << e;
+                }
             }
-            if (lane == sk) cm &= ~(1u << se);                    // claimed either way
+            if (lane == sk) { cm &= ~(1u << se); lcm &= ~(1u << se); }   // claimed either way
+            // bulk leaf claims (leaf_skip = 2, 128-wide windows): every unvisited leaf candidate
+            // of the window is claimed at once — each is exactly Alg 1's descend-and-pop-back
+            // (a leaf's only in-list is u's, so its parent is u in any order)
+            if (__any_sync(kFull, lcm != 0)) {
+                uint32_t lold[VEC];
+#pragma unroll
+                for (int e = 0; e < VEC; ++e)
+                    lold[e] = atom_or_if((lcm >> e) & 1u, P.bitmap + ((uint32_t)nbv[e] >> 5), 1u << (nbv[e] & 31));
+                uint32_t nl = 0;
+#pragma unroll
+                for (int e = 0; e < VEC; ++e) {
+                    const bool lwon = ((lcm >> e) & 1u) && !(lold[e] & (1u << (nbv[e] & 31)));
+                    st_global_if(lwon, P.parent + nbv[e], (int32_t)u);           // Alg 1 l.10
+                    nl += lwon;
+                }
+                if (STATS || P.block_claims || P.timeline) {
+                    nl = __reduce_add_sync(kFull, nl);
+                    my_claims += nl;
+                    if (STATS && lane == 0) cnt[kCntClaims] += nl;
+                }
+            }
             s_old = __shfl_sync(kFull, s_old, 0);
             bool won = vb != 0 && !(s_old & (1u << (sv & 31)));
             if (STATS && vb && !won && lane == 0) ++cnt[kCntFailedClaims];
@@ -881,9 +907,8 @@ __global__ void __launch_bounds__(32 * WMAX, 1) dfs_persistent_kernel(const KPar
             } else {
                 i = a + kWin;
                 spec_ok = false;
-                if (have_nxt) {                                   // next window already loaded
-#pragma unroll
-                    for (int f = 0; f < VEC; ++f) nbv[f] = nxt[f];
+                if (have_nxt) {                                   // next window (prefetched)
+                    load_window(i, end, 32, nbv);
                 } else {
                     have_win = false;                             // i >= end: Alg 1 l.14: pop
                     has_top = pop(u, i);
@@ -895,7 +920,7 @@ __global__ void __launch_bounds__(32 * WMAX, 1) dfs_persistent_kernel(const KPar
             ++iter;
             if ((iter & 31u) == 0) {
                 if (P.timeline && lane == 0) {                    // diagnostics: claim progress
-                    atomicAdd(&P.ctl->claims_progress, my_claims - tl_reported);
+                    atomicAdd(&P.ctl->claims_progress, (unsigned long long)(my_claims - tl_reported));
                     tl_reported = my_claims;
                 }
                 sample();
@@ -921,7 +946,7 @@ __global__ void __launch_bounds__(32 * WMAX, 1) dfs_persistent_kernel(const KPar
             if ((iter & 1023u) == 0) {
                 const int stop = __shfl_sync(kFull, (int)(*(volatile unsigned int*)&P.ctl->done), 0);
                 if (stop) { set_done_local(); break; }
-                if (__shfl_sync(kFull, (int)(globaltimer() - t_start > P.timeout_ns), 0)) {
+                if (__shfl_sync(kFull, (int)(globaltimer() - S.t_start > P.timeout_ns), 0)) {
                     if (lane == 0) raise_error(P, kStatusETIMEOUT);
                     set_done_local();
                     break;
@@ -958,7 +983,7 @@ __global__ void __launch_bounds__(32 * WMAX, 1) dfs_persistent_kernel(const KPar
                     goto exit_loop;
                 }
             }
-            if (__shfl_sync(kFull, (int)(globaltimer() - t_start > P.timeout_ns), 0)) {
+            if (__shfl_sync(kFull, (int)(globaltimer() - S.t_start > P.timeout_ns), 0)) {
                 if (lane == 0) raise_error(P, kStatusETIMEOUT);
                 set_done_local();
                 goto exit_loop;
@@ -1160,7 +1185,7 @@ exit_loop:
             if (ld_relaxed_u32(slot) != kEmptySlot) st_relaxed_u32(slot, kEmptySlot);
         }
     }
-    if (P.block_claims && lane == 0 && my_claims) atomicAdd(&P.block_claims[blockIdx.x], my_claims);
+    if (P.block_claims && lane == 0 && my_claims) atomicAdd(&P.block_claims[blockIdx.x], (unsigned long long)my_claims);
     if (STATS && (P.collect_stats != 2 || gw == 0)) {     // 2: the root warp's counters only
 #pragma unroll
         for (int k = 0; k < kNumCounters; ++k)
@@ -1220,6 +1245,36 @@ __global__ void dfs_count_kernel(const uint32_t* __restrict__ bitmap, const uint
         mv += __shfl_down_sync(kFull, mv, o);
     }
     if ((threadIdx.x & 31) == 0) { atomicAdd(&out2[0], nv); atomicAdd(&out2[1], mv); }
+}
+
+// leaf map (create time, step a1): bit v is set iff every list that contains v leaves nothing
+// for v to explore once claimed — out-degree 0, or out-degree 1 whose single neighbour w is v
+// itself or the only vertex with an edge into v.  Claiming such a v from u is exactly Alg 1's
+// "descend, scan, pop straight back", so the expansion step claims all leaf candidates of a
+// window at once.
+__global__ void dfs_leaf_init_kernel(const uint32_t* __restrict__ rp, uint32_t n, uint32_t* leaf) {
+    const size_t stride = (size_t)gridDim.x * blockDim.x;
+    for (size_t wd = blockIdx.x * (size_t)blockDim.x + threadIdx.x; wd < ((size_t)n + 31) / 32; wd += stride) {
+        uint32_t bits = 0;
+        for (uint32_t b = 0; b < 32; ++b) {
+            const size_t v = wd * 32 + b;
+            if (v < n && rp[v + 1] - rp[v] <= 1u) bits |= 1u << b;
+        }
+        leaf[wd] = bits;
+    }
+}
+// clear the bit of a degree-1 target v reached from a row u other than its own neighbour w
+__global__ void dfs_leaf_edges_kernel(const uint32_t* __restrict__ rp, const int32_t* __restrict__ col,
+                                      uint32_t n, uint32_t* leaf) {
+    const size_t stride = (size_t)gridDim.x * blockDim.x;
+    for (size_t u = blockIdx.x * (size_t)blockDim.x + threadIdx.x; u < n; u += stride) {
+        for (uint32_t j = rp[u]; j < rp[u + 1]; ++j) {
+            const uint32_t v = (uint32_t)col[j];
+            if (rp[v + 1] - rp[v] != 1u) continue;
+            const uint32_t wv = (uint32_t)col[rp[v]];
+            if (wv != (uint32_t)u && wv != v) atomicAnd(&leaf[v >> 5], ~(1u << (v & 31)));
+        }
+    }
 }
 
 // CSR validation + narrowing of row_ptr to uint32 (step a1)

@@ -105,6 +105,13 @@ VARIANTS = {
     "early": dict(speculate=6),
     "specpop": dict(speculate=10),
     "noleaf": dict(leaf_skip=False),
+    "bulk": dict(leaf_skip=2),
+    "bulkw16": dict(leaf_skip=2, warps_per_block=16),
+    "pb4": dict(pub_batch=4),
+    "pb16": dict(pub_batch=16),
+    "spill128": dict(spill_idle=128),
+    "spill1k": dict(spill_idle=1024),
+    "nointra": dict(intra_steal=False),
     "detnoleaf": dict(deterministic=True, leaf_skip=False),
     "specboth": dict(speculate=14),
     "specpop128": dict(speculate=9, window=128),
