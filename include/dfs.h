@@ -104,7 +104,10 @@ typedef struct dfs_options {
                                 pushes (entries above it are private); default 1                    */
     int32_t speculate;       /* bits 0-1: 1 = claim a freshly descended child's first non-parent
                                 neighbour in parallel with the visited probes; 0 = off; 2 = on for
-                                32-wide windows only.  bit 3: also claim a popped entry's next
+                                32-wide windows only.  bit 2: load the claimed child's first
+                                32-wide window as soon as its row_ptr pair arrives, before the
+                                claim's result (discarded if the claim fails).  bit 3: also claim
+                                a popped entry's next
                                 position speculatively (its probe saw it unvisited when the entry
                                 was pushed).  Default 2|8                                          */
     int32_t steal_half;      /* 1 (default): a thief takes max(h_s, rest/2) <= 32 HotRing entries
@@ -128,7 +131,17 @@ typedef struct dfs_options {
                                 2 (default): in addition, 128-wide windows claim every unvisited
                                 leaf candidate at once (leaf map built at create: out-degree 0, or
                                 1 whose only in-list is its neighbour's).  0: always descend       */
-    int32_t reserved[6];     /* zero                                                              */
+    int32_t cluster;         /* cluster steal tier: 2, 4 or 8 = launch the persistent
+                                grid as thread-block clusters of that many CTAs; an idle warp that
+                                finds no Alg 3 victim in its own CTA steals from the HotRings of the
+                                other CTAs of its cluster through distributed shared memory (same
+                                reservation protocol as Alg 3) before trying Alg 4.  The grid is
+                                rounded down to whole co-resident clusters.  0 = off; 1 = the
+                                cluster build launched as clusters of one CTA (diagnostic: the
+                                cost of cluster-visible publication alone)                       */
+    int32_t cluster_late;    /* 1: an idle warp tries the cluster tier after Alg 4 instead of
+                                between Alg 3 and Alg 4                                            */
+    int32_t reserved[4];     /* zero                                                              */
 } dfs_options;
 
 typedef struct dfs_stats {
@@ -154,6 +167,7 @@ typedef struct dfs_stats {
     /* optional, caller-owned host array of `blocks` int64 (NULL = not wanted; single traversals):
        claims (tree vertices discovered) per block — the task distribution of Fig 9 */
     int64_t *block_claims;
+    int64_t cluster_steals;  /* steals through distributed shared memory (cluster tier)           */
 } dfs_stats;
 
 void dfs_options_default(dfs_options *opt);

@@ -64,7 +64,7 @@ struct Ctl {
 enum CounterIdx {
     kCntClaims = 0, kCntFailedClaims, kCntFlushes, kCntRefills, kCntIntraSteals, kCntInterSteals,
     kCntStealAttempts, kCntChunks, kCntWindows, kCntIdleNs, kCntInterScans, kCntSpills,
-    kCntTWin, kCntTProbe, kCntTClaim, kCntTTail, kCntTOut, kCntOutIters, kNumCounters
+    kCntTWin, kCntTProbe, kCntTClaim, kCntTTail, kCntTOut, kCntOutIters, kCntClusterSteals, kNumCounters
 };
 
 struct KParams {
@@ -103,6 +103,7 @@ struct KParams {
     uint32_t ring_cap;                       // usable HotRing entries (<= H); 2 ~ one-level stack (v1)
     int leaf_skip;                           // claim children whose list is empty or [parent] in place
     unsigned long long* block_claims;        // optional: claims per block (Fig 9 task counts)
+    int cluster_late;                        // cluster tier after Alg 4 instead of before it
 };
 
 // ------------------------------------------------------------------------------------------
@@ -201,6 +202,52 @@ __device__ __forceinline__ void st_shared_u64_if(bool p, unsigned long long* a, 
                  ::"r"((uint32_t)p), "r"(smem_addr(a)), "l"(v) : "memory");
 }
 
+// ---- thread-block-cluster (DSMEM) helpers for the cluster steal tier ----
+// Publication for cluster-scope readers: fence.release restricted to shared::cta state (SASS
+// MEMBAR.ALL.CTA + FENCE.VIEW.ASYNC.S — an unrestricted release.cluster is MEMBAR.ALL.GPU) and a
+// relaxed cluster-scope atomic; the remote side pairs it with the restricted acquire fence (no
+// SASS: an unrestricted acquire.cluster would invalidate the SM's L1, CCTL.IVALL).
+__device__ __forceinline__ void fence_release_cta_for_cluster() {
+    asm volatile("fence.release.sync_restrict::shared::cta.cluster;" ::: "memory");
+}
+__device__ __forceinline__ void fence_acquire_cluster_smem() {
+    asm volatile("fence.acquire.sync_restrict::shared::cluster.cluster;" ::: "memory");
+}
+__device__ __forceinline__ void atom_add_relaxed_cluster_if(bool p, uint32_t* a, uint32_t v) {
+    asm volatile("{ .reg .pred q; setp.ne.u32 q, %0, 0; @q atom.relaxed.cluster.shared.add.u32 _, [%1], %2; }"
+                 ::"r"((uint32_t)p), "r"(smem_addr(a)), "r"(v) : "memory");
+}
+__device__ __forceinline__ uint32_t cluster_ctarank() {
+    uint32_t r; asm volatile("mov.u32 %0, %%cluster_ctarank;" : "=r"(r)); return r;
+}
+__device__ __forceinline__ uint32_t cluster_nctarank() {
+    uint32_t r; asm volatile("mov.u32 %0, %%cluster_nctarank;" : "=r"(r)); return r;
+}
+// shared::cluster address of the same variable in CTA `rank` of the cluster
+__device__ __forceinline__ uint32_t dsmem_map(const void* p, uint32_t rank) {
+    uint32_t r; asm volatile("mapa.shared::cluster.u32 %0, %1, %2;" : "=r"(r) : "r"(smem_addr(p)), "r"(rank)); return r;
+}
+__device__ __forceinline__ uint32_t dsmem_ld_u32(uint32_t a) {
+    uint32_t v; asm volatile("ld.relaxed.cluster.shared::cluster.u32 %0, [%1];" : "=r"(v) : "r"(a) : "memory"); return v;
+}
+__device__ __forceinline__ unsigned long long dsmem_ld_u64(uint32_t a) {
+    unsigned long long v; asm volatile("ld.shared::cluster.u64 %0, [%1];" : "=l"(v) : "r"(a) : "memory"); return v;
+}
+__device__ __forceinline__ uint32_t dsmem_cas_u32(uint32_t a, uint32_t cmp, uint32_t v) {
+    uint32_t r;
+    asm volatile("atom.relaxed.cluster.shared::cluster.cas.b32 %0, [%1], %2, %3;" : "=r"(r) : "r"(a), "r"(cmp), "r"(v) : "memory");
+    return r;
+}
+__device__ __forceinline__ void dsmem_st_u32(uint32_t a, uint32_t v) {
+    asm volatile("st.relaxed.cluster.shared::cluster.u32 [%0], %1;" ::"r"(a), "r"(v) : "memory");
+}
+__device__ __forceinline__ void dsmem_st_release_u32(uint32_t a, uint32_t v) {
+    asm volatile("st.release.cluster.shared::cluster.u32 [%0], %1;" ::"r"(a), "r"(v) : "memory");
+}
+__device__ __forceinline__ void cluster_sync_all() {
+    asm volatile("barrier.cluster.arrive.release.aligned;\n\tbarrier.cluster.wait.acquire.aligned;" ::: "memory");
+}
+
 __device__ __forceinline__ unsigned long long pack_entry(uint32_t v, uint32_t i) {
     return (unsigned long long)v | ((unsigned long long)i << 32);
 }
@@ -282,10 +329,12 @@ __device__ __forceinline__ void raise_error(const KParams& P, int code) {
 //   VEC = neighbours per lane per window (1: 32-wide window; 4: 128-wide, 128-bit loads)
 //   WMAX = max warps per block (launch bounds: 32 -> 64 registers, 16 -> 128 registers)
 //   STATS = compile the diagnostic counters in
+//   CL  = compile the cluster (DSMEM) steal tier in: HotRing publication becomes cluster-visible
+//         and idle warps steal from the HotRings of the other CTAs of their thread-block cluster
 // Launched with blockDim.x = 32 * W (W <= WMAX) and dynamic shared memory
 // sizeof(SmemCtl) (16-byte padded) + W * H * 8 bytes.
 // ------------------------------------------------------------------------------------------
-template <int H, int VEC, int WMAX, bool STATS>
+template <int H, int VEC, int WMAX, bool STATS, bool CL>
 __global__ void __launch_bounds__(32 * WMAX, 1) dfs_persistent_kernel(const KParams P) {
     static_assert((H & (H - 1)) == 0 && H >= 64 && H <= 32768, "H must be a power of two in [64, 2^15]");
     static_assert(VEC == 1 || VEC == 4, "VEC is 1 or 4");
@@ -297,6 +346,14 @@ __global__ void __launch_bounds__(32 * WMAX, 1) dfs_persistent_kernel(const KPar
     SmemCtl& S = *reinterpret_cast<SmemCtl*>(smem_raw);
     constexpr int kCtlBytes = (sizeof(SmemCtl) + 15) & ~15;
     unsigned long long* const rings = reinterpret_cast<unsigned long long*>(smem_raw + kCtlBytes);
+    // HotRing publication (owner -> thieves, lane 0 issues): a CTA-scope release, or made
+    // visible to the cluster when the DSMEM steal tier is compiled in
+    auto pub_add = [&](bool p, uint32_t* a, uint32_t v) {
+        if constexpr (CL) { fence_release_cta_for_cluster(); atom_add_relaxed_cluster_if(p, a, v); }
+        else atom_add_release_cta_if(p, a, v);
+    };
+    const uint32_t crank = CL ? cluster_ctarank() : 0u;     // rank in the thread-block cluster
+    const uint32_t ncta = CL ? cluster_nctarank() : 1u;     // CTAs per cluster (1: tier off)
 
     const int lane = threadIdx.x & 31;
     const int w = threadIdx.x >> 5;
@@ -334,10 +391,12 @@ __global__ void __launch_bounds__(32 * WMAX, 1) dfs_persistent_kernel(const KPar
     bool spec_ok = false;        // speculative claim allowed on the current window (fresh child,
                                  // or a popped entry with speculate & 8)
     uint32_t par = kFull;        // parent of u when spec_ok (kFull: no position to skip)
-    // speculate: bits 0-1 = mode (0 off, 1 on, 2 on for 32-wide windows), bit 3 = also claim a
-    // popped entry's next position speculatively (its probe at push time saw it unvisited)
+    // speculate: bits 0-1 = mode (0 off, 1 on, 2 on for 32-wide windows), bit 2 = issue the
+    // child's first window before the claim returns (32-wide), bit 3 = also claim a popped
+    // entry's next position speculatively (its probe at push time saw it unvisited)
     const bool spec_on = (P.speculate & 3) == 1 || ((P.speculate & 3) == 2 && VEC == 1);
     const bool spec_pop = spec_on && (P.speculate & 8) != 0;
+    const bool spec_early = spec_on && (P.speculate & 4) != 0;
     const uint32_t leaf_deg = P.leaf_skip ? 1u : 0u;   // children of degree <= this may be leaves
     uint32_t my_top = 0;         // owner copy of ColdSeg top
     uint32_t hi = 0;             // ColdSeg chunks [.., hi) mapped by this warp
@@ -375,7 +434,7 @@ __global__ void __launch_bounds__(32 * WMAX, 1) dfs_persistent_kernel(const KPar
     // publish the private entries [pub, my_head) to thieves (CTA-scope release)
     auto publish = [&]() {
         if (my_head != pub) {
-            if (lane == 0) atom_add_release_cta(&S.ht[w], ((my_head - pub) & 0xFFFFu) << 16);
+            pub_add(lane == 0, &S.ht[w], ((my_head - pub) & 0xFFFFu) << 16);
             pub = my_head;
         }
     };
@@ -481,7 +540,7 @@ __global__ void __launch_bounds__(32 * WMAX, 1) dfs_persistent_kernel(const KPar
         st_shared_u64_if(lane == 0, ring + (my_head & (H - 1)), pack_entry(v, idx));
         ++my_head;
         if (((my_head - pub) & 0xFFFFu) >= P.pub_batch) {
-            atom_add_release_cta_if(lane == 0, &S.ht[w], ((my_head - pub) & 0xFFFFu) << 16);
+            pub_add(lane == 0, &S.ht[w], ((my_head - pub) & 0xFFFFu) << 16);
             pub = my_head;
         }
         return true;
@@ -552,8 +611,8 @@ __global__ void __launch_bounds__(32 * WMAX, 1) dfs_persistent_kernel(const KPar
         __syncwarp();
         if (lane == 0) {
             atomicSub(&P.block_cold[blockIdx.x], (int)k);
-            atom_add_release_cta(&S.ht[w], k << 16);              // publish (ring was empty)
         }
+        pub_add(lane == 0, &S.ht[w], k << 16);                    // publish (ring was empty)
         my_head += k; pub = my_head;
         if (STATS && lane == 0) ++cnt[kCntRefills];
         return k;
@@ -592,6 +651,74 @@ __global__ void __launch_bounds__(32 * WMAX, 1) dfs_persistent_kernel(const KPar
                 tl_next = slot + 1;
             }
         }
+    };
+
+    // cluster tier: Alg 3 over distributed shared memory — the peer HotRing with
+    // max hot_rest >= hot_cutoff among the other CTAs of the thread-block cluster; same
+    // reservation protocol (victim lock + CAS on the packed head/tail word), the entries move
+    // SM-to-SM without touching global memory.  Returns true with the entries in our ring.
+    auto cluster_steal = [&]() -> bool {
+        if constexpr (CL) {
+            if (!P.intra || ncta < 2) return false;
+            int best = -1, bw = 0;
+            uint32_t bp = 0;
+            for (uint32_t d = 1; d < ncta; ++d) {
+                const uint32_t pr = (crank + d) % ncta;
+                int rest = -1;
+                if (lane < W) rest = ht_rest(dsmem_ld_u32(dsmem_map(&S.ht[lane], pr)));
+                const int b = __reduce_max_sync(kFull, rest);
+                if (b > best) { best = b; bp = pr; bw = __ffs(__ballot_sync(kFull, rest == b)) - 1; }
+            }
+            if (best >= P.hot_cutoff) {
+                if (STATS && lane == 0) ++cnt[kCntStealAttempts];
+                const uint32_t rlock = dsmem_map(&S.lock[bw], bp);
+                const uint32_t rht = dsmem_map(&S.ht[bw], bp);
+                uint32_t ok = 0, t = 0, kst = 0;
+                if (lane == 0) {
+                    if (dsmem_cas_u32(rlock, 0u, 1u) == 0u) {
+                        fence_acquire_cluster_smem();
+                        register_thief();                        // before reserving
+                        uint32_t old = dsmem_ld_u32(rht);
+                        for (int tries = 0; tries < 8; ++tries) {
+                            const int r = ht_rest(old);
+                            if (r < P.hot_cutoff) break;
+                            t = ht_tail(old);
+                            kst = hs;
+                            if (P.steal_half && (uint32_t)(r / 2) > kst) kst = (uint32_t)(r / 2);
+                            if (kst > 32u) kst = 32u;
+                            if ((int)kst > r) kst = (uint32_t)r;
+                            const uint32_t nw = (old & 0xFFFF0000u) | ((t + kst) & 0xFFFFu);
+                            const uint32_t got = dsmem_cas_u32(rht, old, nw);   // reserve
+                            if (got == old) { ok = 1; break; }
+                            old = got;
+                        }
+                        fence_acquire_cluster_smem();            // entries published before `old`
+                        if (!ok) { dsmem_st_release_u32(rlock, 0u); deregister(); }
+                    }
+                }
+                ok = __shfl_sync(kFull, ok, 0);
+                if (ok) {
+                    t = __shfl_sync(kFull, t, 0);
+                    kst = __shfl_sync(kFull, kst, 0);
+                    __syncwarp();                                // lane 0's acquire -> all lanes
+                    if (lane < (int)kst)
+                        ring[(my_head + lane) & (H - 1)] =
+                            dsmem_ld_u64(dsmem_map(rings + (size_t)bw * H + ((t + lane) & (H - 1)), bp));
+                    __syncwarp();
+                    if (lane == 0) {
+                        dsmem_st_u32(dsmem_map((const void*)&S.tailf[bw], bp), (t + kst) & 0xFFFFu);
+                        dsmem_st_release_u32(rlock, 0u);        // copies done before unlock
+                        atomicOr(&S.warp_mask, 1u << w);
+                    }
+                    pub_add(lane == 0, &S.ht[w], kst << 16);     // publish into our ring
+                    __syncwarp();
+                    my_head += kst; pub = my_head;
+                    if (STATS && lane == 0) ++cnt[kCntClusterSteals];
+                    return true;
+                }
+            }
+        }
+        return false;
     };
 
     // ---------------------------------------------------------------- main loop (Alg 2)
@@ -642,14 +769,16 @@ __global__ void __launch_bounds__(32 * WMAX, 1) dfs_persistent_kernel(const KPar
             const uint32_t word = ld_cg_if(valid, P.bitmap + ((uint32_t)nb >> 5), kFull);
             const bool pf = valid && lane < kPfLanes;
             const uint32_t prs = ld_nc_if(pf, P.rp + nb, 0u), pre = ld_nc_if(pf, P.rp + nb + 1, 0u);
+            // early child window (speculate & 4): issued once the row_ptr pair arrives, before
+            // the claim returns (the probes are already in flight)
+            int cnb = (int)ld_nc_if(spec_early && vb != 0 && s_rs + lane < s_re, P.col + s_rs + lane, kFull);
             bool cand = valid && !((word >> (nb & 31)) & 1u) && lane != sk;   // sk is claimed either way
-            int cnb = (int)kFull;
             s_old = __shfl_sync(kFull, s_old, 0);
             bool won = vb != 0 && !(s_old & (1u << (sv & 31)));
             uint32_t v = sv, vrs = s_rs, vre = s_re;
             int kpos = sk;
             if (won) {
-                cnb = (int)ld_nc_if(vrs + lane < vre, P.col + vrs + lane, kFull);
+                if (!spec_early) cnb = (int)ld_nc_if(vrs + lane < vre, P.col + vrs + lane, kFull);
             } else {
                 if (STATS && vb && lane == 0) ++cnt[kCntFailedClaims];
                 // claim the first unvisited candidate in CSR order; on a lost race try the next
@@ -1028,9 +1157,9 @@ __global__ void __launch_bounds__(32 * WMAX, 1) dfs_persistent_kernel(const KPar
                         if (lane == 0) {
                             S.tailf[vwarp] = (t + kst) & 0xFFFFu;    // slots reusable by the owner
                             smem_unlock(&S.lock[vwarp]);
-                            atom_add_release_cta(&S.ht[w], kst << 16); // publish into our ring
                             atomicOr(&S.warp_mask, 1u << w);         // mark active
                         }
+                        pub_add(lane == 0, &S.ht[w], kst << 16);     // publish into our ring
                         __syncwarp();
                         my_head += kst; pub = my_head;
                         if (STATS && lane == 0) ++cnt[kCntIntraSteals];
@@ -1039,6 +1168,7 @@ __global__ void __launch_bounds__(32 * WMAX, 1) dfs_persistent_kernel(const KPar
                     }
                 }
             }
+            if (CL && !P.cluster_late && cluster_steal()) { got_work = true; break; }
             // ---- Alg 4: steal c_s entries from a remote ColdSeg bottom ----
             int token = 0;
             if (P.inter && gridDim.x > 1 &&
@@ -1145,9 +1275,9 @@ __global__ void __launch_bounds__(32 * WMAX, 1) dfs_persistent_kernel(const KPar
                                     p += part; left -= part;
                                 }
                                 atomicSub(&P.block_cold[vb], (int)kst);
-                                atom_add_release_cta(&S.ht[w], kst << 16);     // publish into our ring
                                 atomicOr(&S.warp_mask, 1u << w);               // mark w, b active
                             }
+                            pub_add(lane == 0, &S.ht[w], kst << 16);           // publish into our ring
                             __syncwarp();
                             my_head += kst; pub = my_head;
                             if (STATS && lane == 0) ++cnt[kCntInterSteals];
@@ -1159,6 +1289,7 @@ __global__ void __launch_bounds__(32 * WMAX, 1) dfs_persistent_kernel(const KPar
                 }
             }
             if (token && lane == 0) smem_unlock(&S.inter_token);
+            if (CL && P.cluster_late && cluster_steal()) { got_work = true; break; }
             sample();
             __nanosleep(backoff);
             if (backoff < P.backoff_max_ns) backoff <<= 1;
@@ -1192,6 +1323,8 @@ exit_loop:
             if (lane == 0 && cnt[k]) atomicAdd(&P.ctl->counters[k], cnt[k]);
         __syncwarp();
     }
+    // no CTA may exit while a cluster peer can still read or lock its HotRings
+    if constexpr (CL) cluster_sync_all();
 }
 
 // ------------------------------------------------------------------------------------------
@@ -1247,33 +1380,44 @@ __global__ void dfs_count_kernel(const uint32_t* __restrict__ bitmap, const uint
     if ((threadIdx.x & 31) == 0) { atomicAdd(&out2[0], nv); atomicAdd(&out2[1], mv); }
 }
 
-// leaf map (create time, step a1): bit v is set iff every list that contains v leaves nothing
-// for v to explore once claimed — out-degree 0, or out-degree 1 whose single neighbour w is v
-// itself or the only vertex with an edge into v.  Claiming such a v from u is exactly Alg 1's
-// "descend, scan, pop straight back", so the expansion step claims all leaf candidates of a
-// window at once.
-__global__ void dfs_leaf_init_kernel(const uint32_t* __restrict__ rp, uint32_t n, uint32_t* leaf) {
+// leaf map (create time, step a1).  Claiming a leaf v from u at once (bulk, out of Alg 1's
+// order) is exactly Alg 1's "descend, scan, pop straight back" iff no other list can claim v and
+// v's own list leads nowhere: bit v is set iff every in-edge of v (self-loops aside) comes from
+// one vertex w, and v's out-list is empty or the single entry w or v.  Pass 1 finds the unique
+// in-neighbour of every out-degree <= 1 vertex (kInUnset / kInMulti otherwise); pass 2 sets bits.
+constexpr uint32_t kInUnset = 0xFFFFFFFFu;
+constexpr uint32_t kInMulti = 0xFFFFFFFEu;
+__global__ void dfs_leaf_in_kernel(const uint32_t* __restrict__ rp, const int32_t* __restrict__ col,
+                                   uint32_t n, uint32_t* inn) {
+    const size_t stride = (size_t)gridDim.x * blockDim.x;
+    for (size_t u = blockIdx.x * (size_t)blockDim.x + threadIdx.x; u < n; u += stride) {
+        for (uint32_t j = rp[u]; j < rp[u + 1]; ++j) {
+            const uint32_t v = (uint32_t)col[j];
+            if (v == (uint32_t)u || rp[v + 1] - rp[v] > 1u) continue;
+            const uint32_t old = atomicCAS(&inn[v], kInUnset, (uint32_t)u);
+            if (old != kInUnset && old != (uint32_t)u) atomicExch(&inn[v], kInMulti);
+        }
+    }
+}
+__global__ void dfs_leaf_init_kernel(const uint32_t* __restrict__ rp, const int32_t* __restrict__ col,
+                                     const uint32_t* __restrict__ inn, uint32_t n, uint32_t* leaf) {
     const size_t stride = (size_t)gridDim.x * blockDim.x;
     for (size_t wd = blockIdx.x * (size_t)blockDim.x + threadIdx.x; wd < ((size_t)n + 31) / 32; wd += stride) {
         uint32_t bits = 0;
         for (uint32_t b = 0; b < 32; ++b) {
             const size_t v = wd * 32 + b;
-            if (v < n && rp[v + 1] - rp[v] <= 1u) bits |= 1u << b;
+            if (v >= n) break;
+            const uint32_t deg = rp[v + 1] - rp[v];
+            if (deg > 1u) continue;
+            const uint32_t w = inn[v];
+            if (w == kInMulti) continue;
+            if (deg == 1u) {
+                const uint32_t x = (uint32_t)col[rp[v]];
+                if (x != (uint32_t)v && x != w && w != kInUnset) continue;
+            }
+            bits |= 1u << b;
         }
         leaf[wd] = bits;
-    }
-}
-// clear the bit of a degree-1 target v reached from a row u other than its own neighbour w
-__global__ void dfs_leaf_edges_kernel(const uint32_t* __restrict__ rp, const int32_t* __restrict__ col,
-                                      uint32_t n, uint32_t* leaf) {
-    const size_t stride = (size_t)gridDim.x * blockDim.x;
-    for (size_t u = blockIdx.x * (size_t)blockDim.x + threadIdx.x; u < n; u += stride) {
-        for (uint32_t j = rp[u]; j < rp[u + 1]; ++j) {
-            const uint32_t v = (uint32_t)col[j];
-            if (rp[v + 1] - rp[v] != 1u) continue;
-            const uint32_t wv = (uint32_t)col[rp[v]];
-            if (wv != (uint32_t)u && wv != v) atomicAnd(&leaf[v >> 5], ~(1u << (v & 31)));
-        }
     }
 }
 

@@ -39,15 +39,18 @@ bool is_device_ptr(const void* p) {
     return a.type == cudaMemoryTypeDevice || a.type == cudaMemoryTypeManaged;
 }
 
-// the 8 instantiations of the persistent kernel: [vec128][wmax16][stats]
+// the 16 instantiations of the persistent kernel: [cluster tier][vec128][wmax16][stats]
+#define DFS_K(V, W, S, C) (const void*)dfs_persistent_kernel<kRing, V, W, S, C>
 const void* const* kernel_table() {
-    static const void* const t[8] = {
-        (const void*)dfs_persistent_kernel<kRing, 1, 32, false>, (const void*)dfs_persistent_kernel<kRing, 1, 32, true>,
-        (const void*)dfs_persistent_kernel<kRing, 1, 16, false>, (const void*)dfs_persistent_kernel<kRing, 1, 16, true>,
-        (const void*)dfs_persistent_kernel<kRing, 4, 32, false>, (const void*)dfs_persistent_kernel<kRing, 4, 32, true>,
-        (const void*)dfs_persistent_kernel<kRing, 4, 16, false>, (const void*)dfs_persistent_kernel<kRing, 4, 16, true>};
+    static const void* const t[16] = {
+        DFS_K(1, 32, false, false), DFS_K(1, 32, true, false), DFS_K(1, 16, false, false), DFS_K(1, 16, true, false),
+        DFS_K(4, 32, false, false), DFS_K(4, 32, true, false), DFS_K(4, 16, false, false), DFS_K(4, 16, true, false),
+        DFS_K(1, 32, false, true), DFS_K(1, 32, true, true), DFS_K(1, 16, false, true), DFS_K(1, 16, true, true),
+        DFS_K(4, 32, false, true), DFS_K(4, 32, true, true), DFS_K(4, 16, false, true), DFS_K(4, 16, true, true)};
     return t;
 }
+#undef DFS_K
+constexpr int kNumKernels = 16;
 
 size_t smem_bytes(int warps) {
     return ((sizeof(SmemCtl) + 15) & ~size_t(15)) + (size_t)warps * kRing * sizeof(unsigned long long);
@@ -83,6 +86,7 @@ struct dfs_graph {
     int64_t n = 0, m = 0;
     int sms = 0;
     int max_blocks = 0;          // co-resident 32-warp blocks (allocation bound)
+    int max_clusters[4] = {0, 0, 0, 0};   // co-resident clusters of 1/2/4/8 CTAs (lazy)
     int tab_log2 = 0;
     uint32_t* d_rp = nullptr;
     int32_t* d_col = nullptr;    // col_idx (+8 padding for 128-bit window loads)
@@ -214,13 +218,13 @@ dfs_graph* dfs_graph_create(const int64_t* row_ptr, const int32_t* col_idx, int6
     g->sms = prop.multiProcessorCount;
     const size_t sm32 = smem_bytes(32);
     bool attr_ok = true;
-    for (int kf = 0; kf < 8; ++kf) {
+    for (int kf = 0; kf < kNumKernels; ++kf) {
         if (cudaFuncSetAttribute(kernel_table()[kf], cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm32) != cudaSuccess)
             attr_ok = false;
     }
     if (!attr_ok) { cudaGetLastError(); delete g; fail(DFS_ECUDA); return nullptr; }
     int per_sm = 0;
-    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, dfs_persistent_kernel<kRing, 4, 32, false>, 1024, sm32) !=
+    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, dfs_persistent_kernel<kRing, 4, 32, false, false>, 1024, sm32) !=
             cudaSuccess || per_sm < 1) {
         cudaGetLastError(); per_sm = 1;
     }
@@ -275,10 +279,16 @@ dfs_graph* dfs_graph_create(const int64_t* row_ptr, const int32_t* col_idx, int6
     if (hbad) { free_graph(g); fail(DFS_EINVAL); return nullptr; }
     cudaMemset(g->d_col + m, 0xFF, 8 * sizeof(int32_t));            // padding (never a valid position)
     {
+        uint32_t* d_inn = nullptr;                                    // unique in-neighbours (temporary)
+        if (cudaMalloc(&d_inn, (size_t)n * sizeof(uint32_t)) != cudaSuccess) {
+            cudaGetLastError(); free_graph(g); fail(DFS_ENOMEM); return nullptr;
+        }
+        cudaMemset(d_inn, 0xFF, (size_t)n * sizeof(uint32_t));      // kInUnset
+        dfs_leaf_in_kernel<<<(int)std::min<int64_t>((n + 255) / 256, 65535), 256>>>(g->d_rp, g->d_col, (uint32_t)n, d_inn);
         const int blocks = (int)std::min<int64_t>(((n + 31) / 32 + 255) / 256 + 1, 65535);
-        dfs_leaf_init_kernel<<<blocks, 256>>>(g->d_rp, (uint32_t)n, g->d_leaf);
-        dfs_leaf_edges_kernel<<<(int)std::min<int64_t>((n + 255) / 256, 65535), 256>>>(g->d_rp, g->d_col, (uint32_t)n, g->d_leaf);
+        dfs_leaf_init_kernel<<<blocks, 256>>>(g->d_rp, g->d_col, d_inn, (uint32_t)n, g->d_leaf);
         g->launches += 2;
+        cudaFree(d_inn);
     }
     if (cudaDeviceSynchronize() != cudaSuccess) { cudaGetLastError(); free_graph(g); fail(DFS_ECUDA); return nullptr; }
     return g;
@@ -370,6 +380,7 @@ static int launch_one(dfs_graph* g, Slot& sl, cudaStream_t s, int32_t root, int3
     P.leaf_skip = o.leaf_skip ? 1 : 0;
     P.ring_cap = (o.ring_cap > 0 && o.ring_cap < kRing) ? (uint32_t)o.ring_cap : (uint32_t)kRing;
     P.block_claims = sl.block_claims;
+    P.cluster_late = o.cluster_late;
     const bool tl = g->d_timeline && &sl == &g->slots[0];
     P.timeline = tl ? g->d_timeline : nullptr;
     P.timeline_len = tl ? g->timeline_len : 0;
@@ -377,10 +388,25 @@ static int launch_one(dfs_graph* g, Slot& sl, cudaStream_t s, int32_t root, int3
     P.timeout_ns = (unsigned long long)o.timeout_ms * 1000000ull;
     P.seed = o.seed;
     void* args[] = {(void*)&P};
-    const void* kfn = kernel_table()[(o.window == 128 ? 4 : 0) + (warps <= 16 ? 2 : 0) + (o.collect_stats ? 1 : 0)];
+    const int cl = o.cluster > 1 ? o.cluster : 1;
+    const void* kfn = kernel_table()[(o.cluster >= 1 ? 8 : 0) + (o.window == 128 ? 4 : 0) + (warps <= 16 ? 2 : 0) +
+                                     (o.collect_stats ? 1 : 0)];
     if (timed) cudaEventRecord(sl.evk0, s);
     cudaError_t e;
-    if (cooperative) {
+    if (o.cluster >= 1) {
+        // cluster tier: clusters of `cl` CTAs; blocks is a multiple of cl and at
+        // most cl x the co-resident cluster count (resolve_options)
+        cudaLaunchConfig_t cfg = {};
+        cudaLaunchAttribute at[2];
+        at[0].id = cudaLaunchAttributeClusterDimension;
+        at[0].val.clusterDim.x = (unsigned)cl; at[0].val.clusterDim.y = 1; at[0].val.clusterDim.z = 1;
+        at[1].id = cudaLaunchAttributeCooperative;
+        at[1].val.cooperative = cooperative ? 1 : 0;
+        cfg.gridDim = dim3(blocks); cfg.blockDim = dim3(32 * warps);
+        cfg.dynamicSmemBytes = smem_bytes(warps); cfg.stream = s;
+        cfg.attrs = at; cfg.numAttrs = 2;
+        e = cudaLaunchKernelExC(&cfg, kfn, args);
+    } else if (cooperative) {
         e = cudaLaunchCooperativeKernel(kfn, dim3(blocks), dim3(32 * warps), args, smem_bytes(warps), s);
     } else {
         // concurrent batch slots: co-residency is not required for progress — a block that starts
@@ -396,7 +422,27 @@ static int launch_one(dfs_graph* g, Slot& sl, cudaStream_t s, int32_t root, int3
     return DFS_OK;
 }
 
-static int resolve_options(const dfs_graph* g, const dfs_options* in, int num_roots, dfs_options& o,
+// co-resident clusters of `cl` CTAs of the persistent kernel (cudaOccupancyMaxActiveClusters;
+// cached per cluster size)
+static int max_clusters(dfs_graph* g, int cl, int warps, int window, bool stats) {
+    int idx = 0;
+    while ((1 << idx) < cl) ++idx;
+    if (g->max_clusters[idx] > 0) return g->max_clusters[idx];
+    (void)warps;   // the 32-warp instantiation bounds the smaller blocks' footprint
+    const void* kfn = kernel_table()[8 + (window == 128 ? 4 : 0) + (stats ? 1 : 0)];
+    cudaLaunchConfig_t cfg = {};
+    cudaLaunchAttribute at[1];
+    at[0].id = cudaLaunchAttributeClusterDimension;
+    at[0].val.clusterDim.x = (unsigned)cl; at[0].val.clusterDim.y = 1; at[0].val.clusterDim.z = 1;
+    cfg.gridDim = dim3((unsigned)(g->max_blocks / cl * cl)); cfg.blockDim = dim3(1024);
+    cfg.dynamicSmemBytes = smem_bytes(32); cfg.attrs = at; cfg.numAttrs = 1;
+    int n = 0;
+    if (cudaOccupancyMaxActiveClusters(&n, kfn, &cfg) != cudaSuccess) { cudaGetLastError(); n = 0; }
+    g->max_clusters[idx] = n;
+    return n;
+}
+
+static int resolve_options(dfs_graph* g, const dfs_options* in, int num_roots, dfs_options& o,
                            int& blocks, int& warps, int& conc) {
     dfs_options_default(&o);
     if (in) o = *in;
@@ -409,6 +455,7 @@ static int resolve_options(const dfs_graph* g, const dfs_options* in, int num_ro
     if (o.cold_cutoff < 1 || o.cold_cutoff / 2 > 64) return DFS_EINVAL;
     if (o.victim_policy != 0 && o.victim_policy != 1) return DFS_EINVAL;
     if (o.reserved0 != 0) return DFS_EINVAL;
+    if (o.cluster < 0 || o.cluster > 8 || (o.cluster > 1 && (o.cluster & (o.cluster - 1)))) return DFS_EINVAL;
     if (o.window == 0) o.window = (g->n > 0 && g->m >= 8 * g->n) ? 128 : 32;   // wide windows for dense lists
     if (o.window != 32 && o.window != 128) return DFS_EINVAL;
     if (o.concurrency < 0 || o.concurrency > kMaxSlots) return DFS_EINVAL;
@@ -420,7 +467,14 @@ static int resolve_options(const dfs_graph* g, const dfs_options* in, int num_ro
     const int share = std::max(1, g->max_blocks / conc);
     blocks = o.blocks <= 0 ? share : o.blocks;
     if (blocks > g->max_blocks || (conc > 1 && blocks * conc > g->max_blocks)) return DFS_EINVAL;
-    if (o.deterministic) { blocks = 1; warps = 1; o.intra_steal = 0; o.inter_steal = 0; }
+    if (o.deterministic) { blocks = 1; warps = 1; o.intra_steal = 0; o.inter_steal = 0; o.cluster = 0; }
+    if (o.cluster > 1) {
+        // whole clusters only, no more than can be co-resident
+        const int maxc = max_clusters(g, o.cluster, warps, o.window, o.collect_stats != 0);
+        if (maxc < 1) return DFS_EINVAL;
+        blocks = std::min(blocks, maxc * o.cluster) / o.cluster * o.cluster;
+        if (blocks < o.cluster) return DFS_EINVAL;
+    }
     return DFS_OK;
 }
 
@@ -456,6 +510,7 @@ static void fill_stats(dfs_stats* stats, int blocks, int warps, float total_ms, 
     stats->cyc_claim = (int64_t)counters[kCntTClaim];
     stats->cyc_tail = (int64_t)counters[kCntTTail];
     stats->cyc_outside = (int64_t)counters[kCntTOut];
+    stats->cluster_steals = (int64_t)counters[kCntClusterSteals];
 }
 
 // per-root count buffer (2 x u64 per root) for stats calls

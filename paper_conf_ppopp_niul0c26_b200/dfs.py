@@ -49,7 +49,8 @@ class _Options(ctypes.Structure):
                 ("steal_half", ctypes.c_int32), ("concurrency", ctypes.c_int32),
                 ("ring_cap", ctypes.c_int32), ("backoff_min_ns", ctypes.c_int32),
                 ("max_pool_chunks", ctypes.c_int32), ("reserved0", ctypes.c_int32),
-                ("leaf_skip", ctypes.c_int32), ("reserved", ctypes.c_int32 * 6)]
+                ("leaf_skip", ctypes.c_int32), ("cluster", ctypes.c_int32),
+                ("cluster_late", ctypes.c_int32), ("reserved", ctypes.c_int32 * 4)]
 
 
 class _Stats(ctypes.Structure):
@@ -65,7 +66,7 @@ class _Stats(ctypes.Structure):
                 ("cyc_window", ctypes.c_int64), ("cyc_probe", ctypes.c_int64),
                 ("cyc_claim", ctypes.c_int64), ("cyc_tail", ctypes.c_int64),
                 ("cyc_outside", ctypes.c_int64), ("root_counts", ctypes.c_void_p),
-                ("block_claims", ctypes.c_void_p)]
+                ("block_claims", ctypes.c_void_p), ("cluster_steals", ctypes.c_int64)]
 
 
 @dataclass
@@ -95,6 +96,8 @@ class Options:
     backoff_min_ns: Optional[int] = None
     max_pool_chunks: Optional[int] = None
     leaf_skip: Optional[bool] = None
+    cluster: Optional[int] = None
+    cluster_late: Optional[bool] = None
 
     def to_c(self) -> _Options:
         o = _Options()
@@ -131,6 +134,7 @@ class Stats:
     cyc_claim: int
     cyc_tail: int
     cyc_outside: int
+    cluster_steals: int = 0
     root_counts: Optional[np.ndarray] = None
     block_claims: Optional[np.ndarray] = None
 

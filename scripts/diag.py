@@ -122,6 +122,16 @@ VARIANTS = {
     "early128": dict(speculate=5, window=128),
     "w0early": dict(collect_stats=2, speculate=6),
     "w0detearly": dict(collect_stats=2, deterministic=True, speculate=6),
+    "cl2": dict(cluster=2),
+    "cl4": dict(cluster=4),
+    "cl8": dict(cluster=8),
+    "cl2stats": dict(cluster=2, collect_stats=True),
+    "cl4nospill": dict(cluster=4, spill=False),
+    "cl1": dict(cluster=1),
+    "early2": dict(speculate=2 | 4 | 8),
+    "detearly": dict(deterministic=True, speculate=2 | 4 | 8),
+    "cl2late": dict(cluster=2, cluster_late=True),
+    "cl2late_stats": dict(cluster=2, cluster_late=True, collect_stats=True),
 }
 
 
@@ -184,7 +194,7 @@ def main():
                        total_ms=round(st.kernel_ms, 3), gteps=round(st.m_visited / st.traversal_ms / 1e6, 4),
                        n_visited=st.n_visited, util=round(util, 4), claims=st.claims,
                        failed=st.failed_claims, windows=st.windows, flushes=st.flushes,
-                       refills=st.refills, intra=st.intra_steals, inter=st.inter_steals,
+                       refills=st.refills, intra=st.intra_steals, inter=st.inter_steals, cl=st.cluster_steals, blocks=st.blocks,
                        attempts=st.steal_attempts, scans=st.inter_scans, spills=st.spills, chunks=st.chunks_allocated,
                        us_per_claim_per_warp=round(st.traversal_ms * 1e3 * warps * util / max(1, st.claims), 3),
                        windows_per_claim=round(st.windows / max(1, st.claims), 3),

@@ -70,6 +70,33 @@ def test_deterministic_bit_exact(name, build, root):
             _exact(g, root, p)
 
 
+def test_bulk_leaf_claims_respect_shared_in_lists():
+    """Leaf map (bulk claims in 128-wide windows): a sink with two in-neighbours is not a leaf —
+    Alg 1 reaches it through the first child, so claiming it early from the root would differ."""
+    #   0 -> [1, 2];  1 -> [2];  2 -> []  (directed);  Alg 1 from 0: parent = [-1, 0, 1]
+    rp = np.array([0, 2, 3, 3], dtype=np.int64)
+    ci = np.array([1, 2, 2], dtype=np.int32)
+    with Graph(rp, ci) as G:
+        for win in (32, 128):
+            assert G.run(0, options=Options(deterministic=True, window=win)).cpu().tolist() == [-1, 0, 1]
+    # many sinks shared by two hubs, deterministic 128-wide windows: bit-exact with Alg 1
+    rng = np.random.default_rng(5)
+    n, k = 3000, 400
+    rows = [[] for _ in range(n)]
+    rows[0] = [1] + list(range(2 + 0, 2 + k))                 # root: hub 1, then sinks
+    rows[1] = list(range(2, 2 + k)) + list(range(2 + k, n))   # hub 1 reaches the same sinks first
+    for v in range(2 + k, n):
+        rows[v] = sorted(rng.choice(n, 2, replace=False).tolist())
+    rp = np.zeros(n + 1, dtype=np.int64)
+    rp[1:] = np.cumsum([len(r) for r in rows])
+    ci = np.array([x for r in rows for x in r], dtype=np.int32)
+    g = graphgen.CSR(rp, ci, "shared_sinks")
+    with Graph(rp, ci) as G:
+        for win in (32, 128):
+            _exact(g, 0, G.run(0, options=Options(deterministic=True, window=win)))
+            _valid(g, 0, G.run(0, options=Options(window=win)), undirected=False)
+
+
 # ------------------------------------------------------------------ unique trees: exact in parallel
 @pytest.mark.parametrize("name,build,roots", [
     ("path", lambda: graphgen.path(200_001), [0, 100_000, 200_000]),
@@ -134,6 +161,10 @@ def test_parallel_directed_with_self_loops_and_duplicates():
     dict(speculate=0),
     dict(speculate=1, window=128),
     dict(hot_cutoff=4, ring_cap=3, warps_per_block=4, blocks=6),
+    dict(cluster=2),                                                  # §8(f)-3 DSMEM tier
+    dict(cluster=4, hot_cutoff=2, window=128),
+    dict(cluster=2, warps_per_block=4, blocks=8, spill=False, inter_steal=False),
+    dict(cluster=8, warps_per_block=2, hot_cutoff=1, intra_steal=True, spill_idle=1),
 ])
 def test_stress_options(opts):
     graphs = [graphgen.road(300, 300, seed=3), graphgen.rmat(14, 8, seed=9),
@@ -206,6 +237,8 @@ def test_errors():
             G.run(0, options=Options(window=64))
         with pytest.raises(DfsError):
             G.run(0, options=Options(blocks=100000))
+        with pytest.raises(DfsError):
+            G.run(0, options=Options(cluster=3))                  # cluster sizes 2, 4, 8
     bad = g.row_ptr.copy(); bad[5] = bad[4] - 1                   # non-monotone row_ptr
     with pytest.raises(DfsError):
         Graph(bad, g.col_idx)
@@ -322,3 +355,26 @@ def test_cli_on_matrix_market(tmp_path, capsys):
     rows = out_csv.read_text().strip().splitlines()
     assert len(rows) == 5 and rows[0].startswith("root,n_visited")
     assert all(int(r.split(",")[1]) == g.n for r in rows[1:])          # connected: all reached
+
+
+@pytest.mark.parametrize("cl", [2, 4])
+def test_cluster_tier_moves_work_through_dsmem(cl):
+    """§8(f)-3: with Alg 4 and the spill off, work leaves a CTA only through the cluster tier —
+    every CTA of the root's cluster claims vertices, the steals are counted, the tree is valid
+    (I1-I6), and the grid is whole clusters."""
+    g = graphgen.road(512, 512, seed=21)
+    with Graph(g.row_ptr, g.col_idx) as G:
+        o = Options(cluster=cl, inter_steal=False, spill=False, collect_stats=True)
+        p, st = G.run(0, options=o, stats=True, block_claims=True)
+        _valid(g, 0, p)
+        assert st.cluster_steals > 0
+        assert st.blocks % cl == 0
+        bc = st.block_claims
+        assert int(bc.sum()) == st.n_visited - 1
+        assert (bc[:cl] > 0).all() and (bc[cl:] == 0).all()       # work stayed in cluster 0
+        # default-tier run on the same handle, then the cluster tier on a batch
+        _valid(g, 5, G.run(5))
+        roots = graphgen.random_roots(g, 4, seed=cl)
+        out = G.run_batch(roots, options=Options(cluster=cl, concurrency=2))
+        for q, r in enumerate(roots):
+            _valid(g, int(r), out[q])
