@@ -109,7 +109,7 @@ typedef struct dfs_options {
                                 claim's result (discarded if the claim fails).  bit 3: also claim
                                 a popped entry's next
                                 position speculatively (its probe saw it unvisited when the entry
-                                was pushed).  Default 2|8                                          */
+                                was pushed).  Default 2|4|8                                          */
     int32_t steal_half;      /* 1 (default): a thief takes max(h_s, rest/2) <= 32 HotRing entries
                                 (resp. max(c_s, rest/2) <= 64 ColdSeg entries); 0: exactly h_s/c_s
                                 as in Alg 3/4                                                       */
@@ -141,7 +141,11 @@ typedef struct dfs_options {
                                 cost of cluster-visible publication alone)                       */
     int32_t cluster_late;    /* 1: an idle warp tries the cluster tier after Alg 4 instead of
                                 between Alg 3 and Alg 4                                            */
-    int32_t reserved[4];     /* zero                                                              */
+    int32_t steal_tries;     /* Alg 3 victims an idle warp tries per round, best first: when the
+                                max-hot_rest victim is locked by another thief (or falls below
+                                hot_cutoff) it moves on to the next best; 1 = Alg 3 as written;
+                                default 8                                                          */
+    int32_t reserved[3];     /* zero                                                              */
 } dfs_options;
 
 typedef struct dfs_stats {

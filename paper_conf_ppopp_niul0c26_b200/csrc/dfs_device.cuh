@@ -104,6 +104,7 @@ struct KParams {
     int leaf_skip;                           // claim children whose list is empty or [parent] in place
     unsigned long long* block_claims;        // optional: claims per block (Fig 9 task counts)
     int cluster_late;                        // cluster tier after Alg 4 instead of before it
+    int steal_tries;                         // Alg 3 victims tried per idle round (best first)
 };
 
 // ------------------------------------------------------------------------------------------
@@ -1046,39 +1047,40 @@ __global__ void __launch_bounds__(32 * WMAX, 1) dfs_persistent_kernel(const KPar
                 }
             }
           }   // VEC == 4 step
-            ++iter;
-            if ((iter & 31u) == 0) {
+            // periodic work, one branch per step: diagnostics and the spill check every 32
+            // steps, the done flag and the watchdog every 1024
+            if ((++iter & 31u) == 0) {
                 if (P.timeline && lane == 0) {                    // diagnostics: claim progress
                     atomicAdd(&P.ctl->claims_progress, (unsigned long long)(my_claims - tl_reported));
                     tl_reported = my_claims;
                 }
                 sample();
-            }
-            if (P.spill && (iter & 31u) == 0) {
-                // demand-driven spill: many warps idle and a deep HotRing -> make the oldest half
-                // of it visible to other blocks (Alg 4 steals ColdSeg bottoms only)
-                uint32_t want = 0;
-                if (lane == 0) {
-                    const uint32_t rest = (my_head - ht_tail(ld_acquire_cta(&S.ht[w]))) & 0xFFFFu;
-                    if (rest >= 2u * (uint32_t)P.cold_cutoff) {
-                        // idle warps elsewhere ~ W x (blocks with no busy warp)
-                        const uint32_t busy_blocks = *(volatile unsigned int*)&P.ctl->busy;
-                        if ((int)((gridDim.x - busy_blocks) * W) >= P.spill_idle) want = rest / 2;
+                if (P.spill) {
+                    // demand-driven spill: many warps idle and a deep HotRing -> make the oldest
+                    // half of it visible to other blocks (Alg 4 steals ColdSeg bottoms only)
+                    uint32_t want = 0;
+                    if (lane == 0) {
+                        const uint32_t rest = (my_head - ht_tail(ld_acquire_cta(&S.ht[w]))) & 0xFFFFu;
+                        if (rest >= 2u * (uint32_t)P.cold_cutoff) {
+                            // idle warps elsewhere ~ W x (blocks with no busy warp)
+                            const uint32_t busy_blocks = *(volatile unsigned int*)&P.ctl->busy;
+                            if ((int)((gridDim.x - busy_blocks) * W) >= P.spill_idle) want = rest / 2;
+                        }
+                    }
+                    want = __shfl_sync(kFull, want, 0);
+                    if (want) {
+                        if (!flush(want, want)) break;
+                        if (STATS && lane == 0) ++cnt[kCntSpills];
                     }
                 }
-                want = __shfl_sync(kFull, want, 0);
-                if (want) {
-                    if (!flush(want, want)) break;
-                    if (STATS && lane == 0) ++cnt[kCntSpills];
-                }
-            }
-            if ((iter & 1023u) == 0) {
-                const int stop = __shfl_sync(kFull, (int)(*(volatile unsigned int*)&P.ctl->done), 0);
-                if (stop) { set_done_local(); break; }
-                if (__shfl_sync(kFull, (int)(globaltimer() - S.t_start > P.timeout_ns), 0)) {
-                    if (lane == 0) raise_error(P, kStatusETIMEOUT);
-                    set_done_local();
-                    break;
+                if ((iter & 1023u) == 0) {
+                    const int stop = __shfl_sync(kFull, (int)(*(volatile unsigned int*)&P.ctl->done), 0);
+                    if (stop) { set_done_local(); break; }
+                    if (__shfl_sync(kFull, (int)(globaltimer() - S.t_start > P.timeout_ns), 0)) {
+                        if (lane == 0) raise_error(P, kStatusETIMEOUT);
+                        set_done_local();
+                        break;
+                    }
                 }
             }
             continue;
@@ -1118,11 +1120,14 @@ __global__ void __launch_bounds__(32 * WMAX, 1) dfs_persistent_kernel(const KPar
                 goto exit_loop;
             }
             // ---- Alg 3: intra-block stealing from the peer HotRing with max hot_rest ----
+            // (steal_tries > 1: when the best victim is locked by another thief or drops below
+            // the cutoff, try the next best instead of backing off)
             if (P.intra && W > 1) {
                 int rest = -1;
                 if (lane < W && lane != w) rest = ht_rest(*(volatile uint32_t*)&S.ht[lane]);
-                const int best = __reduce_max_sync(kFull, rest);
-                if (best >= P.hot_cutoff) {
+                for (int att = 0; att < P.steal_tries; ++att) {
+                    const int best = __reduce_max_sync(kFull, rest);
+                    if (best < P.hot_cutoff) break;
                     const int vwarp = __ffs(__ballot_sync(kFull, rest == best)) - 1;
                     if (STATS && lane == 0) ++cnt[kCntStealAttempts];
                     uint32_t ok = 0, t = 0, kst = 0;
@@ -1147,26 +1152,29 @@ __global__ void __launch_bounds__(32 * WMAX, 1) dfs_persistent_kernel(const KPar
                         }
                     }
                     ok = __shfl_sync(kFull, ok, 0);
-                    if (ok) {
-                        t = __shfl_sync(kFull, t, 0);
-                        kst = __shfl_sync(kFull, kst, 0);
-                        __syncwarp();                                // lane 0's acquire -> all lanes
-                        const unsigned long long* vring = rings + (size_t)vwarp * H;
-                        if (lane < (int)kst) ring[(my_head + lane) & (H - 1)] = vring[(t + lane) & (H - 1)];
-                        __syncwarp();
-                        if (lane == 0) {
-                            S.tailf[vwarp] = (t + kst) & 0xFFFFu;    // slots reusable by the owner
-                            smem_unlock(&S.lock[vwarp]);
-                            atomicOr(&S.warp_mask, 1u << w);         // mark active
-                        }
-                        pub_add(lane == 0, &S.ht[w], kst << 16);     // publish into our ring
-                        __syncwarp();
-                        my_head += kst; pub = my_head;
-                        if (STATS && lane == 0) ++cnt[kCntIntraSteals];
-                        got_work = true;
-                        break;
+                    if (!ok) {
+                        if (lane == vwarp) rest = -1;                // next best
+                        continue;
                     }
+                    t = __shfl_sync(kFull, t, 0);
+                    kst = __shfl_sync(kFull, kst, 0);
+                    __syncwarp();                                    // lane 0's acquire -> all lanes
+                    const unsigned long long* vring = rings + (size_t)vwarp * H;
+                    if (lane < (int)kst) ring[(my_head + lane) & (H - 1)] = vring[(t + lane) & (H - 1)];
+                    __syncwarp();
+                    if (lane == 0) {
+                        S.tailf[vwarp] = (t + kst) & 0xFFFFu;        // slots reusable by the owner
+                        smem_unlock(&S.lock[vwarp]);
+                        atomicOr(&S.warp_mask, 1u << w);             // mark active
+                    }
+                    pub_add(lane == 0, &S.ht[w], kst << 16);         // publish into our ring
+                    __syncwarp();
+                    my_head += kst; pub = my_head;
+                    if (STATS && lane == 0) ++cnt[kCntIntraSteals];
+                    got_work = true;
+                    break;
                 }
+                if (got_work) break;
             }
             if (CL && !P.cluster_late && cluster_steal()) { got_work = true; break; }
             // ---- Alg 4: steal c_s entries from a remote ColdSeg bottom ----

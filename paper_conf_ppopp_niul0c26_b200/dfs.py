@@ -50,7 +50,8 @@ class _Options(ctypes.Structure):
                 ("ring_cap", ctypes.c_int32), ("backoff_min_ns", ctypes.c_int32),
                 ("max_pool_chunks", ctypes.c_int32), ("reserved0", ctypes.c_int32),
                 ("leaf_skip", ctypes.c_int32), ("cluster", ctypes.c_int32),
-                ("cluster_late", ctypes.c_int32), ("reserved", ctypes.c_int32 * 4)]
+                ("cluster_late", ctypes.c_int32), ("steal_tries", ctypes.c_int32),
+                ("reserved", ctypes.c_int32 * 3)]
 
 
 class _Stats(ctypes.Structure):
@@ -98,6 +99,7 @@ class Options:
     leaf_skip: Optional[bool] = None
     cluster: Optional[int] = None
     cluster_late: Optional[bool] = None
+    steal_tries: Optional[int] = None
 
     def to_c(self) -> _Options:
         o = _Options()

@@ -128,6 +128,13 @@ VARIANTS = {
     "cl2stats": dict(cluster=2, collect_stats=True),
     "cl4nospill": dict(cluster=4, spill=False),
     "cl1": dict(cluster=1),
+    "noearly": dict(speculate=2 | 8),
+    "st1": dict(steal_tries=1),
+    "early2st8": dict(speculate=2 | 4 | 8, steal_tries=8),
+    "st2": dict(steal_tries=2),
+    "st4": dict(steal_tries=4),
+    "st8": dict(steal_tries=8),
+    "st4stats": dict(steal_tries=4, collect_stats=True),
     "early2": dict(speculate=2 | 4 | 8),
     "detearly": dict(deterministic=True, speculate=2 | 4 | 8),
     "cl2late": dict(cluster=2, cluster_late=True),

@@ -64,7 +64,7 @@ def test_deterministic_bit_exact(name, build, root):
     if root is None:
         root = int(graphgen.random_roots(g, 1, seed=1)[0])
     with Graph(g.row_ptr, g.col_idx) as G:
-        for win, sp in ((32, 2), (128, 2), (32, 0), (128, 1)):
+        for win, sp in ((32, 2), (128, 2), (32, 0), (128, 1), (32, 2 | 4 | 8)):
             p = G.run(root, options=Options(deterministic=True, window=win, speculate=sp))
             torch.cuda.synchronize()
             _exact(g, root, p)
@@ -165,6 +165,10 @@ def test_parallel_directed_with_self_loops_and_duplicates():
     dict(cluster=4, hot_cutoff=2, window=128),
     dict(cluster=2, warps_per_block=4, blocks=8, spill=False, inter_steal=False),
     dict(cluster=8, warps_per_block=2, hot_cutoff=1, intra_steal=True, spill_idle=1),
+    dict(cluster=2, cluster_late=True, steal_tries=3, hot_cutoff=2),
+    dict(steal_tries=4),
+    dict(steal_tries=8, warps_per_block=8, blocks=4, spill=False),
+    dict(speculate=2 | 4 | 8),
 ])
 def test_stress_options(opts):
     graphs = [graphgen.road(300, 300, seed=3), graphgen.rmat(14, 8, seed=9),
