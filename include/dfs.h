@@ -145,7 +145,13 @@ typedef struct dfs_options {
                                 max-hot_rest victim is locked by another thief (or falls below
                                 hot_cutoff) it moves on to the next best; 1 = Alg 3 as written;
                                 default 8                                                          */
-    int32_t reserved[3];     /* zero                                                              */
+    int32_t bulk_copy;       /* 1: flush and refill move the 16-byte-aligned part of each piece with
+                                cp.async.bulk (shared->global, resp. global->shared completing on a
+                                per-warp mbarrier) — the paper's TMA variant;
+                                0 (default): warp-wide 8-byte copies                               */
+    int32_t spill_period;    /* a busy warp checks the spill condition every spill_period expansion
+                                steps (power of two <= 1024; 0 = 32)                               */
+    int32_t reserved[1];     /* zero                                                              */
 } dfs_options;
 
 typedef struct dfs_stats {

@@ -105,6 +105,8 @@ struct KParams {
     unsigned long long* block_claims;        // optional: claims per block (Fig 9 task counts)
     int cluster_late;                        // cluster tier after Alg 4 instead of before it
     int steal_tries;                         // Alg 3 victims tried per idle round (best first)
+    int bulk_copy;                           // flush/refill with cp.async.bulk (TMA ablation)
+    uint32_t period_mask;                    // spill_period - 1
 };
 
 // ------------------------------------------------------------------------------------------
@@ -249,6 +251,32 @@ __device__ __forceinline__ void cluster_sync_all() {
     asm volatile("barrier.cluster.arrive.release.aligned;\n\tbarrier.cluster.wait.acquire.aligned;" ::: "memory");
 }
 
+// ---- bulk async copies (cp.async.bulk, the TMA engine's non-tensor path) for the optional
+// bulk flush/refill (dfs_options.bulk_copy; the paper's TMA ablation) ----
+__device__ __forceinline__ void bulk_s2g(void* g, const void* sm, uint32_t bytes) {
+    asm volatile("cp.async.bulk.global.shared::cta.bulk_group [%0], [%1], %2;"
+                 ::"l"(g), "r"(smem_addr(sm)), "r"(bytes) : "memory");
+}
+__device__ __forceinline__ void bulk_commit_wait() {
+    asm volatile("cp.async.bulk.commit_group;\n\tcp.async.bulk.wait_group 0;" ::: "memory");
+}
+__device__ __forceinline__ void bulk_g2s(void* sm, const void* g, uint32_t bytes, uint64_t* mbar) {
+    asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];"
+                 ::"r"(smem_addr(sm)), "l"(g), "r"(bytes), "r"(smem_addr(mbar)) : "memory");
+}
+__device__ __forceinline__ void fence_proxy_async_smem() { asm volatile("fence.proxy.async.shared::cta;" ::: "memory"); }
+__device__ __forceinline__ void fence_proxy_async_global() { asm volatile("fence.proxy.async.global;" ::: "memory"); }
+__device__ __forceinline__ void mbar_init(uint64_t* m) {
+    asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" ::"r"(smem_addr(m)) : "memory");
+}
+__device__ __forceinline__ void mbar_expect_tx(uint64_t* m, uint32_t bytes) {
+    asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_addr(m)), "r"(bytes) : "memory");
+}
+__device__ __forceinline__ void mbar_wait(uint64_t* m, uint32_t parity) {
+    asm volatile("{ .reg .pred p; W: mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1; @!p bra W; }"
+                 ::"r"(smem_addr(m)), "r"(parity) : "memory");
+}
+
 __device__ __forceinline__ unsigned long long pack_entry(uint32_t v, uint32_t i) {
     return (unsigned long long)v | ((unsigned long long)i << 32);
 }
@@ -277,6 +305,7 @@ struct SmemCtl {
     unsigned long long t_start;            // globaltimer at kernel start (watchdog, timeline)
     volatile int done;                     // block-local copy of ctl->done
     uint32_t inter_token;                  // one idle warp per block scans other blocks at a time
+    uint64_t mbar[kMaxWarps];              // per-warp mbarrier of the bulk refill (bulk_copy)
     unsigned long long cnt[kMaxWarps][kNumCounters]; // per-warp stats counters (collect_stats)
 };
 
@@ -376,6 +405,8 @@ __global__ void __launch_bounds__(32 * WMAX, 1) dfs_persistent_kernel(const KPar
     }
     unsigned long long* const cnt = S.cnt[w];     // lane 0 updates its warp's counters
     if (STATS && lane < kNumCounters) cnt[lane] = 0;
+    if (P.bulk_copy && lane == 0) { mbar_init(&S.mbar[w]); asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory"); }
+    uint32_t mbar_phase = 0;                      // parity of this warp's next refill wait
     __syncthreads();
 
     // ---- per-warp state (warp-uniform registers) ----
@@ -484,12 +515,36 @@ __global__ void __launch_bounds__(32 * WMAX, 1) dfs_persistent_kernel(const KPar
             __syncwarp();
             return false;
         }
-        // warp copy, one 8-byte entry per lane per step
-        for (uint32_t q = lane; q < kf; q += 32u) {
-            const unsigned long long e = ring[(t + q) & (H - 1)];
-            const uint32_t p = my_top + q;
-            const uint32_t c = ld_relaxed_u32(&my_tab[(p >> kChunkLog2) & tmask]);
-            st_cg_u64(P.pool + ((size_t)c << kChunkLog2) + (p & (kChunk - 1)), e);
+        if (P.bulk_copy) {
+            // bulk variant: per contiguous piece (split at the ring wrap and at chunk ends) lane
+            // 0 issues one cp.async.bulk shared->global for the 16-byte-aligned middle when ring
+            // slot and ColdSeg position have equal parity; lanes store the rest
+            fence_proxy_async_smem();                 // generic ring writes -> async proxy
+            uint32_t r = t, c = my_top, left = kf;
+            bool any_bulk = false;
+            while (left) {
+                const uint32_t a = H - (r & (H - 1)), b = kChunk - (c & (kChunk - 1));
+                const uint32_t L = left < a ? (left < b ? left : b) : (a < b ? a : b);
+                const uint32_t ch = ld_relaxed_u32(&my_tab[(c >> kChunkLog2) & tmask]);
+                unsigned long long* gp = P.pool + ((size_t)ch << kChunkLog2) + (c & (kChunk - 1));
+                const unsigned long long* sp = ring + (r & (H - 1));
+                uint32_t head = 0, body = 0;
+                if (((r ^ c) & 1u) == 0) { head = r & 1u; if (head > L) head = L; body = (L - head) & ~1u; }
+                if (body && lane == 0) { bulk_s2g(gp + head, sp + head, body * 8u); any_bulk = true; }
+                for (uint32_t q = lane; q < L; q += 32u)
+                    if (q < head || q >= head + body) st_cg_u64(gp + q, sp[q]);
+                r += L; c += L; left -= L;
+            }
+            if (lane == 0 && any_bulk) { bulk_commit_wait(); fence_proxy_async_global(); }
+            __syncwarp();
+        } else {
+            // warp copy, one 8-byte entry per lane per step
+            for (uint32_t q = lane; q < kf; q += 32u) {
+                const unsigned long long e = ring[(t + q) & (H - 1)];
+                const uint32_t p = my_top + q;
+                const uint32_t c = ld_relaxed_u32(&my_tab[(p >> kChunkLog2) & tmask]);
+                st_cg_u64(P.pool + ((size_t)c << kChunkLog2) + (p & (kChunk - 1)), e);
+            }
         }
         fence_release_gpu();                          // every lane: its stores before the publish
         __syncwarp();
@@ -593,10 +648,42 @@ __global__ void __launch_bounds__(32 * WMAX, 1) dfs_persistent_kernel(const KPar
         if (k == 0) return 0;
         const uint32_t base = my_top - k;
         // ring is empty (my_head == tail); place entries oldest first
-        for (uint32_t q = lane; q < k; q += 32u) {
-            const uint32_t p = base + q;
-            const uint32_t c = ld_relaxed_u32(&my_tab[(p >> kChunkLog2) & tmask]);
-            ring[(my_head + q) & (H - 1)] = ld_cg_u64(P.pool + ((size_t)c << kChunkLog2) + (p & (kChunk - 1)));
+        if (P.bulk_copy) {
+            // bulk variant: one cp.async.bulk global->shared per aligned piece, completion on the
+            // warp's mbarrier (expect_tx = the bulk bytes); lanes load the unaligned rest
+            uint32_t r = my_head, c = base, left = k, tx = 0;
+            for (int pass = 0; pass < 2; ++pass) {    // pass 0: count bytes, pass 1: issue
+                r = my_head; c = base; left = k;
+                if (pass == 1 && tx && lane == 0) mbar_expect_tx(&S.mbar[w], tx);
+                while (left) {
+                    const uint32_t a = H - (r & (H - 1)), b = kChunk - (c & (kChunk - 1));
+                    const uint32_t L = left < a ? (left < b ? left : b) : (a < b ? a : b);
+                    uint32_t head = 0, body = 0;
+                    if (((r ^ c) & 1u) == 0) { head = r & 1u; if (head > L) head = L; body = (L - head) & ~1u; }
+                    if (pass == 0) {
+                        tx += body * 8u;
+                    } else {
+                        const uint32_t ch = ld_relaxed_u32(&my_tab[(c >> kChunkLog2) & tmask]);
+                        const unsigned long long* gp = P.pool + ((size_t)ch << kChunkLog2) + (c & (kChunk - 1));
+                        unsigned long long* sp = ring + (r & (H - 1));
+                        if (body && lane == 0) bulk_g2s(sp + head, gp + head, body * 8u, &S.mbar[w]);
+                        for (uint32_t q = lane; q < L; q += 32u)
+                            if (q < head || q >= head + body) sp[q] = ld_cg_u64(gp + q);
+                    }
+                    r += L; c += L; left -= L;
+                }
+            }
+            if (tx) {
+                if (lane == 0) mbar_wait(&S.mbar[w], mbar_phase);
+                mbar_phase ^= 1u;
+            }
+            __syncwarp();
+        } else {
+            for (uint32_t q = lane; q < k; q += 32u) {
+                const uint32_t p = base + q;
+                const uint32_t c = ld_relaxed_u32(&my_tab[(p >> kChunkLog2) & tmask]);
+                ring[(my_head + q) & (H - 1)] = ld_cg_u64(P.pool + ((size_t)c << kChunkLog2) + (p & (kChunk - 1)));
+            }
         }
         my_top = base;
         // release chunks that lie wholly above top + one spare chunk (never read by thieves)
@@ -1047,9 +1134,9 @@ __global__ void __launch_bounds__(32 * WMAX, 1) dfs_persistent_kernel(const KPar
                 }
             }
           }   // VEC == 4 step
-            // periodic work, one branch per step: diagnostics and the spill check every 32
-            // steps, the done flag and the watchdog every 1024
-            if ((++iter & 31u) == 0) {
+            // periodic work, one branch per step: diagnostics and the spill check every
+            // spill_period (power of two <= 1024) steps, the done flag and the watchdog every 1024
+            if ((++iter & P.period_mask) == 0) {
                 if (P.timeline && lane == 0) {                    // diagnostics: claim progress
                     atomicAdd(&P.ctl->claims_progress, (unsigned long long)(my_claims - tl_reported));
                     tl_reported = my_claims;

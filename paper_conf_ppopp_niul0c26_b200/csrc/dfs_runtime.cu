@@ -384,6 +384,8 @@ static int launch_one(dfs_graph* g, Slot& sl, cudaStream_t s, int32_t root, int3
     P.block_claims = sl.block_claims;
     P.cluster_late = o.cluster_late;
     P.steal_tries = o.steal_tries > 0 ? o.steal_tries : 1;
+    P.bulk_copy = o.bulk_copy;
+    P.period_mask = (uint32_t)(o.spill_period > 0 ? o.spill_period : 32) - 1u;
     const bool tl = g->d_timeline && &sl == &g->slots[0];
     P.timeline = tl ? g->d_timeline : nullptr;
     P.timeline_len = tl ? g->timeline_len : 0;
@@ -458,6 +460,7 @@ static int resolve_options(dfs_graph* g, const dfs_options* in, int num_roots, d
     if (o.cold_cutoff < 1 || o.cold_cutoff / 2 > 64) return DFS_EINVAL;
     if (o.victim_policy != 0 && o.victim_policy != 1) return DFS_EINVAL;
     if (o.reserved0 != 0) return DFS_EINVAL;
+    if (o.spill_period < 0 || o.spill_period > 1024 || (o.spill_period & (o.spill_period - 1))) return DFS_EINVAL;
     if (o.cluster < 0 || o.cluster > 8 || (o.cluster > 1 && (o.cluster & (o.cluster - 1)))) return DFS_EINVAL;
     if (o.window == 0) o.window = (g->n > 0 && g->m >= 8 * g->n) ? 128 : 32;   // wide windows for dense lists
     if (o.window != 32 && o.window != 128) return DFS_EINVAL;

@@ -51,7 +51,8 @@ class _Options(ctypes.Structure):
                 ("max_pool_chunks", ctypes.c_int32), ("reserved0", ctypes.c_int32),
                 ("leaf_skip", ctypes.c_int32), ("cluster", ctypes.c_int32),
                 ("cluster_late", ctypes.c_int32), ("steal_tries", ctypes.c_int32),
-                ("reserved", ctypes.c_int32 * 3)]
+                ("bulk_copy", ctypes.c_int32), ("spill_period", ctypes.c_int32),
+                ("reserved", ctypes.c_int32 * 1)]
 
 
 class _Stats(ctypes.Structure):
@@ -100,6 +101,8 @@ class Options:
     cluster: Optional[int] = None
     cluster_late: Optional[bool] = None
     steal_tries: Optional[int] = None
+    bulk_copy: Optional[bool] = None
+    spill_period: Optional[int] = None
 
     def to_c(self) -> _Options:
         o = _Options()

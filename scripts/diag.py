@@ -130,6 +130,13 @@ VARIANTS = {
     "cl1": dict(cluster=1),
     "noearly": dict(speculate=2 | 8),
     "st1": dict(steal_tries=1),
+    "bulk_copy": dict(bulk_copy=True),
+    "bulk_copy_v1": dict(bulk_copy=True, ring_cap=2),
+    "v1": dict(ring_cap=2),
+    "sp8": dict(spill_period=8),
+    "sp16": dict(spill_period=16),
+    "sp64": dict(spill_period=64),
+    "detbulk": dict(deterministic=True, bulk_copy=True),
     "early2st8": dict(speculate=2 | 4 | 8, steal_tries=8),
     "st2": dict(steal_tries=2),
     "st4": dict(steal_tries=4),

@@ -58,6 +58,9 @@ def test_sass_is_sm100a_and_ours(lib):
     # warp-level expansion: ballot (VOTE) + global atomics; 128-bit stack copies
     assert "VOTE.ANY" in sass or "VOTE.ALL" in sass or "VOTE" in sass
     assert "ATOMG" in sass or "RED" in sass
+    # bulk async copies of the TMA flush/refill variant; cluster tier: DSMEM barrier
+    assert "UBLKCP.G.S" in sass and "UBLKCP.S.G" in sass
+    assert "UCGABAR_ARV" in sass
 
 
 def test_null_handle_is_einval(lib):

@@ -169,6 +169,8 @@ def test_parallel_directed_with_self_loops_and_duplicates():
     dict(steal_tries=4),
     dict(steal_tries=8, warps_per_block=8, blocks=4, spill=False),
     dict(speculate=2 | 4 | 8),
+    dict(bulk_copy=True),                                             # cp.async.bulk flush/refill
+    dict(bulk_copy=True, ring_cap=3, hot_cutoff=2, cold_cutoff=2, window=128),
 ])
 def test_stress_options(opts):
     graphs = [graphgen.road(300, 300, seed=3), graphgen.rmat(14, 8, seed=9),
@@ -382,3 +384,17 @@ def test_cluster_tier_moves_work_through_dsmem(cl):
         out = G.run_batch(roots, options=Options(cluster=cl, concurrency=2))
         for q, r in enumerate(roots):
             _valid(g, int(r), out[q])
+
+
+def test_bulk_copy_flush_refill_exact():
+    """cp.async.bulk flush/refill (TMA ablation): deterministic mode stays bit-exact on
+    deep stacks that flush and refill thousands of times (odd ring_cap makes every parity of ring
+    slot vs ColdSeg position occur), and parallel runs stay valid."""
+    for g, root in ((graphgen.grid(256, 256), 0), (graphgen.caterpillar(4096, 94), 0),
+                    (graphgen.path_chords(200_000, 2_000, seed=4), 7)):
+        with Graph(g.row_ptr, g.col_idx) as G:
+            for rc in (0, 7, 64, 3):
+                o = Options(deterministic=True, bulk_copy=True, ring_cap=rc)
+                _exact(g, root, G.run(root, options=o))
+                p, st = G.run(root, options=Options(bulk_copy=True, ring_cap=rc, collect_stats=True), stats=True)
+                _valid(g, root, p)
