@@ -1192,6 +1192,7 @@ __global__ void __launch_bounds__(32 * WMAX, 1) dfs_persistent_kernel(const KPar
         }
         bool got_work = false;
         uint32_t backoff = P.backoff_min_ns;
+        uint32_t idle_iter = 0;
         t_idle0 = STATS ? globaltimer() : 0ull;
         while (!got_work) {
             if (__shfl_sync(kFull, S.done, 0)) goto exit_loop;
@@ -1201,7 +1202,9 @@ __global__ void __launch_bounds__(32 * WMAX, 1) dfs_persistent_kernel(const KPar
                     goto exit_loop;
                 }
             }
-            if (__shfl_sync(kFull, (int)(globaltimer() - S.t_start > P.timeout_ns), 0)) {
+            // watchdog every 16th idle round (idle polling competes with busy warps for issue)
+            if ((idle_iter++ & 15u) == 0 &&
+                __shfl_sync(kFull, (int)(globaltimer() - S.t_start > P.timeout_ns), 0)) {
                 if (lane == 0) raise_error(P, kStatusETIMEOUT);
                 set_done_local();
                 goto exit_loop;
@@ -1268,7 +1271,8 @@ __global__ void __launch_bounds__(32 * WMAX, 1) dfs_persistent_kernel(const KPar
             int token = 0;
             if (P.inter && gridDim.x > 1 &&
                 (P.inter_any || (w == 0 && __shfl_sync(kFull, *(volatile unsigned int*)&S.warp_mask, 0) == 0u))) {
-                if (lane == 0) token = smem_trylock(&S.inter_token) ? 1 : 0;
+                // test before the CAS: most rounds find the token taken
+                if (lane == 0) token = (*(volatile uint32_t*)&S.inter_token == 0u && smem_trylock(&S.inter_token)) ? 1 : 0;
                 token = __shfl_sync(kFull, token, 0);
             }
             if (token) {
