@@ -148,7 +148,8 @@ typedef struct dfs_options {
     int32_t bulk_copy;       /* 1: flush and refill move the 16-byte-aligned part of each piece with
                                 cp.async.bulk (shared->global, resp. global->shared completing on a
                                 per-warp mbarrier) — the paper's TMA variant;
-                                0 (default): warp-wide 8-byte copies                               */
+                                0 (default): warp-wide 8-byte copies.  Not combinable with
+                                cluster (DFS_EINVAL)                                               */
     int32_t spill_period;    /* a busy warp checks the spill condition every spill_period expansion
                                 steps (power of two <= 1024; 0 = 32)                               */
     int32_t reserved[1];     /* zero                                                              */

@@ -306,6 +306,8 @@ struct SmemCtl {
     volatile int done;                     // block-local copy of ctl->done
     uint32_t inter_token;                  // one idle warp per block scans other blocks at a time
     uint64_t mbar[kMaxWarps];              // per-warp mbarrier of the bulk refill (bulk_copy)
+    uint32_t mbar_phase[kMaxWarps];        // ... and the parity of its next wait (not a register:
+                                           // the 128-wide step runs at the 64-register cap)
     unsigned long long cnt[kMaxWarps][kNumCounters]; // per-warp stats counters (collect_stats)
 };
 
@@ -353,18 +355,82 @@ __device__ __forceinline__ void raise_error(const KParams& P, int code) {
     atomicExch(&P.ctl->done, 1u);
 }
 
+// bulk flush / refill copies (bulk_copy = 1), compiled only into the BULK instantiations of the
+// traversal kernel: inlined into the default kernels they made the 128-wide kernel's hot loop 16%
+// slower on RMAT (instruction footprint), and out of line the call ABI forced spills.
+// A contiguous piece of a flush or refill is split at the ring wrap and at ColdSeg chunk ends;
+// when ring slot and ColdSeg position have equal parity, lane 0 moves the piece's 16-byte-aligned
+// middle with one cp.async.bulk and the lanes copy the rest.
+template <int H>
+__device__ __forceinline__ void bulk_flush_copy(unsigned long long* ring, uint32_t t, uint32_t top, uint32_t kf,
+                                             const uint32_t* tab, uint32_t tmask, unsigned long long* pool,
+                                             int lane) {
+    fence_proxy_async_smem();                         // generic ring writes -> async proxy
+    uint32_t r = t, c = top, left = kf;
+    bool any_bulk = false;
+    while (left) {
+        const uint32_t a = H - (r & (H - 1)), b = kChunk - (c & (kChunk - 1));
+        const uint32_t L = left < a ? (left < b ? left : b) : (a < b ? a : b);
+        const uint32_t ch = ld_relaxed_u32(&tab[(c >> kChunkLog2) & tmask]);
+        unsigned long long* gp = pool + ((size_t)ch << kChunkLog2) + (c & (kChunk - 1));
+        const unsigned long long* sp = ring + (r & (H - 1));
+        uint32_t head = 0, body = 0;
+        if (((r ^ c) & 1u) == 0) { head = r & 1u; if (head > L) head = L; body = (L - head) & ~1u; }
+        if (body && lane == 0) { bulk_s2g(gp + head, sp + head, body * 8u); any_bulk = true; }
+        for (uint32_t q = lane; q < L; q += 32u)
+            if (q < head || q >= head + body) st_cg_u64(gp + q, sp[q]);
+        r += L; c += L; left -= L;
+    }
+    if (lane == 0 && any_bulk) { bulk_commit_wait(); fence_proxy_async_global(); }
+    __syncwarp();
+}
+
+template <int H>
+__device__ __forceinline__ void bulk_refill_copy(unsigned long long* ring, uint32_t head0, uint32_t base, uint32_t k,
+                                              const uint32_t* tab, uint32_t tmask, const unsigned long long* pool,
+                                              int lane, uint64_t* mbar, uint32_t* phase) {
+    uint32_t tx = 0;
+    for (int pass = 0; pass < 2; ++pass) {            // pass 0: count the bulk bytes, pass 1: issue
+        uint32_t r = head0, c = base, left = k;
+        if (pass == 1 && tx && lane == 0) mbar_expect_tx(mbar, tx);
+        while (left) {
+            const uint32_t a = H - (r & (H - 1)), b = kChunk - (c & (kChunk - 1));
+            const uint32_t L = left < a ? (left < b ? left : b) : (a < b ? a : b);
+            uint32_t head = 0, body = 0;
+            if (((r ^ c) & 1u) == 0) { head = r & 1u; if (head > L) head = L; body = (L - head) & ~1u; }
+            if (pass == 0) {
+                tx += body * 8u;
+            } else {
+                const uint32_t ch = ld_relaxed_u32(&tab[(c >> kChunkLog2) & tmask]);
+                const unsigned long long* gp = pool + ((size_t)ch << kChunkLog2) + (c & (kChunk - 1));
+                unsigned long long* sp = ring + (r & (H - 1));
+                if (body && lane == 0) bulk_g2s(sp + head, gp + head, body * 8u, mbar);
+                for (uint32_t q = lane; q < L; q += 32u)
+                    if (q < head || q >= head + body) sp[q] = ld_cg_u64(gp + q);
+            }
+            r += L; c += L; left -= L;
+        }
+    }
+    if (tx && lane == 0) {
+        mbar_wait(mbar, *phase);
+        *phase ^= 1u;
+    }
+    __syncwarp();
+}
+
 // ------------------------------------------------------------------------------------------
 // The persistent traversal kernel.
 //   H   = HotRing entries per warp (power of two, <= 2^15)
 //   VEC = neighbours per lane per window (1: 32-wide window; 4: 128-wide, 128-bit loads)
 //   WMAX = max warps per block (launch bounds: 32 -> 64 registers, 16 -> 128 registers)
 //   STATS = compile the diagnostic counters in
+//   BULK = flush/refill with cp.async.bulk (dfs_options.bulk_copy; the paper's TMA variant)
 //   CL  = compile the cluster (DSMEM) steal tier in: HotRing publication becomes cluster-visible
 //         and idle warps steal from the HotRings of the other CTAs of their thread-block cluster
 // Launched with blockDim.x = 32 * W (W <= WMAX) and dynamic shared memory
 // sizeof(SmemCtl) (16-byte padded) + W * H * 8 bytes.
 // ------------------------------------------------------------------------------------------
-template <int H, int VEC, int WMAX, bool STATS, bool CL>
+template <int H, int VEC, int WMAX, bool STATS, bool CL, bool BULK>
 __global__ void __launch_bounds__(32 * WMAX, 1) dfs_persistent_kernel(const KParams P) {
     static_assert((H & (H - 1)) == 0 && H >= 64 && H <= 32768, "H must be a power of two in [64, 2^15]");
     static_assert(VEC == 1 || VEC == 4, "VEC is 1 or 4");
@@ -405,8 +471,10 @@ __global__ void __launch_bounds__(32 * WMAX, 1) dfs_persistent_kernel(const KPar
     }
     unsigned long long* const cnt = S.cnt[w];     // lane 0 updates its warp's counters
     if (STATS && lane < kNumCounters) cnt[lane] = 0;
-    if (P.bulk_copy && lane == 0) { mbar_init(&S.mbar[w]); asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory"); }
-    uint32_t mbar_phase = 0;                      // parity of this warp's next refill wait
+    if (BULK && lane == 0) {
+        mbar_init(&S.mbar[w]); S.mbar_phase[w] = 0;
+        asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    }
     __syncthreads();
 
     // ---- per-warp state (warp-uniform registers) ----
@@ -515,28 +583,8 @@ __global__ void __launch_bounds__(32 * WMAX, 1) dfs_persistent_kernel(const KPar
             __syncwarp();
             return false;
         }
-        if (P.bulk_copy) {
-            // bulk variant: per contiguous piece (split at the ring wrap and at chunk ends) lane
-            // 0 issues one cp.async.bulk shared->global for the 16-byte-aligned middle when ring
-            // slot and ColdSeg position have equal parity; lanes store the rest
-            fence_proxy_async_smem();                 // generic ring writes -> async proxy
-            uint32_t r = t, c = my_top, left = kf;
-            bool any_bulk = false;
-            while (left) {
-                const uint32_t a = H - (r & (H - 1)), b = kChunk - (c & (kChunk - 1));
-                const uint32_t L = left < a ? (left < b ? left : b) : (a < b ? a : b);
-                const uint32_t ch = ld_relaxed_u32(&my_tab[(c >> kChunkLog2) & tmask]);
-                unsigned long long* gp = P.pool + ((size_t)ch << kChunkLog2) + (c & (kChunk - 1));
-                const unsigned long long* sp = ring + (r & (H - 1));
-                uint32_t head = 0, body = 0;
-                if (((r ^ c) & 1u) == 0) { head = r & 1u; if (head > L) head = L; body = (L - head) & ~1u; }
-                if (body && lane == 0) { bulk_s2g(gp + head, sp + head, body * 8u); any_bulk = true; }
-                for (uint32_t q = lane; q < L; q += 32u)
-                    if (q < head || q >= head + body) st_cg_u64(gp + q, sp[q]);
-                r += L; c += L; left -= L;
-            }
-            if (lane == 0 && any_bulk) { bulk_commit_wait(); fence_proxy_async_global(); }
-            __syncwarp();
+        if constexpr (BULK) {
+            bulk_flush_copy<H>(ring, t, my_top, kf, my_tab, tmask, P.pool, lane);
         } else {
             // warp copy, one 8-byte entry per lane per step
             for (uint32_t q = lane; q < kf; q += 32u) {
@@ -648,36 +696,8 @@ __global__ void __launch_bounds__(32 * WMAX, 1) dfs_persistent_kernel(const KPar
         if (k == 0) return 0;
         const uint32_t base = my_top - k;
         // ring is empty (my_head == tail); place entries oldest first
-        if (P.bulk_copy) {
-            // bulk variant: one cp.async.bulk global->shared per aligned piece, completion on the
-            // warp's mbarrier (expect_tx = the bulk bytes); lanes load the unaligned rest
-            uint32_t r = my_head, c = base, left = k, tx = 0;
-            for (int pass = 0; pass < 2; ++pass) {    // pass 0: count bytes, pass 1: issue
-                r = my_head; c = base; left = k;
-                if (pass == 1 && tx && lane == 0) mbar_expect_tx(&S.mbar[w], tx);
-                while (left) {
-                    const uint32_t a = H - (r & (H - 1)), b = kChunk - (c & (kChunk - 1));
-                    const uint32_t L = left < a ? (left < b ? left : b) : (a < b ? a : b);
-                    uint32_t head = 0, body = 0;
-                    if (((r ^ c) & 1u) == 0) { head = r & 1u; if (head > L) head = L; body = (L - head) & ~1u; }
-                    if (pass == 0) {
-                        tx += body * 8u;
-                    } else {
-                        const uint32_t ch = ld_relaxed_u32(&my_tab[(c >> kChunkLog2) & tmask]);
-                        const unsigned long long* gp = P.pool + ((size_t)ch << kChunkLog2) + (c & (kChunk - 1));
-                        unsigned long long* sp = ring + (r & (H - 1));
-                        if (body && lane == 0) bulk_g2s(sp + head, gp + head, body * 8u, &S.mbar[w]);
-                        for (uint32_t q = lane; q < L; q += 32u)
-                            if (q < head || q >= head + body) sp[q] = ld_cg_u64(gp + q);
-                    }
-                    r += L; c += L; left -= L;
-                }
-            }
-            if (tx) {
-                if (lane == 0) mbar_wait(&S.mbar[w], mbar_phase);
-                mbar_phase ^= 1u;
-            }
-            __syncwarp();
+        if constexpr (BULK) {
+            bulk_refill_copy<H>(ring, my_head, base, k, my_tab, tmask, P.pool, lane, &S.mbar[w], &S.mbar_phase[w]);
         } else {
             for (uint32_t q = lane; q < k; q += 32u) {
                 const uint32_t p = base + q;

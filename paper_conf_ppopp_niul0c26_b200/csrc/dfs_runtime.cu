@@ -39,18 +39,21 @@ bool is_device_ptr(const void* p) {
     return a.type == cudaMemoryTypeDevice || a.type == cudaMemoryTypeManaged;
 }
 
-// the 16 instantiations of the persistent kernel: [cluster tier][vec128][wmax16][stats]
-#define DFS_K(V, W, S, C) (const void*)dfs_persistent_kernel<kRing, V, W, S, C>
+// the 24 instantiations of the persistent kernel: [bulk][cluster tier][vec128][wmax16][stats]
+// (the bulk variants without the cluster tier)
+#define DFS_K(V, W, S, C, B) (const void*)dfs_persistent_kernel<kRing, V, W, S, C, B>
 const void* const* kernel_table() {
-    static const void* const t[16] = {
-        DFS_K(1, 32, false, false), DFS_K(1, 32, true, false), DFS_K(1, 16, false, false), DFS_K(1, 16, true, false),
-        DFS_K(4, 32, false, false), DFS_K(4, 32, true, false), DFS_K(4, 16, false, false), DFS_K(4, 16, true, false),
-        DFS_K(1, 32, false, true), DFS_K(1, 32, true, true), DFS_K(1, 16, false, true), DFS_K(1, 16, true, true),
-        DFS_K(4, 32, false, true), DFS_K(4, 32, true, true), DFS_K(4, 16, false, true), DFS_K(4, 16, true, true)};
+    static const void* const t[24] = {
+        DFS_K(1, 32, false, false, false), DFS_K(1, 32, true, false, false), DFS_K(1, 16, false, false, false), DFS_K(1, 16, true, false, false),
+        DFS_K(4, 32, false, false, false), DFS_K(4, 32, true, false, false), DFS_K(4, 16, false, false, false), DFS_K(4, 16, true, false, false),
+        DFS_K(1, 32, false, true, false), DFS_K(1, 32, true, true, false), DFS_K(1, 16, false, true, false), DFS_K(1, 16, true, true, false),
+        DFS_K(4, 32, false, true, false), DFS_K(4, 32, true, true, false), DFS_K(4, 16, false, true, false), DFS_K(4, 16, true, true, false),
+        DFS_K(1, 32, false, false, true), DFS_K(1, 32, true, false, true), DFS_K(1, 16, false, false, true), DFS_K(1, 16, true, false, true),
+        DFS_K(4, 32, false, false, true), DFS_K(4, 32, true, false, true), DFS_K(4, 16, false, false, true), DFS_K(4, 16, true, false, true)};
     return t;
 }
 #undef DFS_K
-constexpr int kNumKernels = 16;
+constexpr int kNumKernels = 24;
 
 size_t smem_bytes(int warps) {
     return ((sizeof(SmemCtl) + 15) & ~size_t(15)) + (size_t)warps * kRing * sizeof(unsigned long long);
@@ -226,7 +229,7 @@ dfs_graph* dfs_graph_create(const int64_t* row_ptr, const int32_t* col_idx, int6
     }
     if (!attr_ok) { cudaGetLastError(); delete g; fail(DFS_ECUDA); return nullptr; }
     int per_sm = 0;
-    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, dfs_persistent_kernel<kRing, 4, 32, false, false>, 1024, sm32) !=
+    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, dfs_persistent_kernel<kRing, 4, 32, false, false, false>, 1024, sm32) !=
             cudaSuccess || per_sm < 1) {
         cudaGetLastError(); per_sm = 1;
     }
@@ -394,8 +397,8 @@ static int launch_one(dfs_graph* g, Slot& sl, cudaStream_t s, int32_t root, int3
     P.seed = o.seed;
     void* args[] = {(void*)&P};
     const int cl = o.cluster > 1 ? o.cluster : 1;
-    const void* kfn = kernel_table()[(o.cluster >= 1 ? 8 : 0) + (o.window == 128 ? 4 : 0) + (warps <= 16 ? 2 : 0) +
-                                     (o.collect_stats ? 1 : 0)];
+    const void* kfn = kernel_table()[(o.bulk_copy ? 16 : o.cluster >= 1 ? 8 : 0) + (o.window == 128 ? 4 : 0) +
+                                     (warps <= 16 ? 2 : 0) + (o.collect_stats ? 1 : 0)];
     if (timed) cudaEventRecord(sl.evk0, s);
     cudaError_t e;
     if (o.cluster >= 1) {
@@ -460,6 +463,7 @@ static int resolve_options(dfs_graph* g, const dfs_options* in, int num_roots, d
     if (o.cold_cutoff < 1 || o.cold_cutoff / 2 > 64) return DFS_EINVAL;
     if (o.victim_policy != 0 && o.victim_policy != 1) return DFS_EINVAL;
     if (o.reserved0 != 0) return DFS_EINVAL;
+    if (o.bulk_copy && o.cluster >= 1) return DFS_EINVAL;     // no bulk + cluster instantiation
     if (o.spill_period < 0 || o.spill_period > 1024 || (o.spill_period & (o.spill_period - 1))) return DFS_EINVAL;
     if (o.cluster < 0 || o.cluster > 8 || (o.cluster > 1 && (o.cluster & (o.cluster - 1)))) return DFS_EINVAL;
     if (o.window == 0) o.window = (g->n > 0 && g->m >= 8 * g->n) ? 128 : 32;   // wide windows for dense lists

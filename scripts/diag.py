@@ -133,6 +133,7 @@ VARIANTS = {
     "bulk_copy": dict(bulk_copy=True),
     "bulk_copy_v1": dict(bulk_copy=True, ring_cap=2),
     "v1": dict(ring_cap=2),
+    "w0nointra": dict(collect_stats=2, intra_steal=False),
     "sp8": dict(spill_period=8),
     "sp16": dict(spill_period=16),
     "sp64": dict(spill_period=64),
@@ -208,7 +209,7 @@ def main():
                        total_ms=round(st.kernel_ms, 3), gteps=round(st.m_visited / st.traversal_ms / 1e6, 4),
                        n_visited=st.n_visited, util=round(util, 4), claims=st.claims,
                        failed=st.failed_claims, windows=st.windows, flushes=st.flushes,
-                       refills=st.refills, intra=st.intra_steals, inter=st.inter_steals, cl=st.cluster_steals, blocks=st.blocks,
+                       refills=st.refills, intra=st.intra_steals, inter=st.inter_steals, cl=getattr(st, "cluster_steals", 0), blocks=st.blocks,
                        attempts=st.steal_attempts, scans=st.inter_scans, spills=st.spills, chunks=st.chunks_allocated,
                        us_per_claim_per_warp=round(st.traversal_ms * 1e3 * warps * util / max(1, st.claims), 3),
                        windows_per_claim=round(st.windows / max(1, st.claims), 3),

@@ -1,0 +1,18 @@
+cd $GRAFT_REPO_ROOT
+mkdir -p gpurun_out/nb2
+timeout 900 python -m pytest tests/test_gpu_parity.py -x -q -m gpu -p no:cacheprovider > gpurun_out/nb2/parity.log 2>&1; echo "parity rc=$?" >> gpurun_out/nb2/parity.log
+tail -3 gpurun_out/nb2/parity.log
+for g in rmat:24 road:4900 path:1e8; do
+for rep in 1 2; do
+  (cd abtest/168b378 && timeout 600 python scripts/diag.py --graph $g --roots 3 --reps 1 --nostats --variants default | sed "s/\"variant\": \"default\"/\"variant\": \"168b378\"/" >> ../../gpurun_out/nb2/diag.jsonl 2>> ../../gpurun_out/nb2/err.log)
+  timeout 600 python scripts/diag.py --graph $g --roots 3 --reps 1 --nostats --variants default,bulk_copy >> gpurun_out/nb2/diag.jsonl 2>> gpurun_out/nb2/err.log
+done
+done
+python - <<'PY'
+import json, collections
+d=collections.defaultdict(list)
+for l in open('gpurun_out/nb2/diag.jsonl'):
+    r=json.loads(l); d[(r['graph'],r['variant'])].append(r['ms'])
+for k,v in sorted(d.items()): print(k, 'mean ms', round(sum(v)/len(v),3), v)
+PY
+tail -2 gpurun_out/nb2/err.log
