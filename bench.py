@@ -322,7 +322,7 @@ def batch_arm(a, world, rank, local):
     log(f"[rank {rank}] batch graph n={g.n} m={g.m} built in {time.time() - t0:.1f}s; {len(roots)} roots")
     G = Graph(g.row_ptr, g.col_idx)
     lo, hi = batch.partition(len(roots), world, rank)
-    conc = a.concurrency if a.concurrency > 0 else 4
+    conc = a.concurrency if a.concurrency > 0 else 8          # library auto (DESIGN §8 sweep)
     out_rows = torch.empty((max(conc, min(16, max(1, hi - lo))), g.n), dtype=torch.int32, device=dev)
     for s_ in range(a.warmup):                       # warm-up traversals (untimed)
         G.run(int(roots[(lo + s_) % len(roots)]), out=out_rows[0])

@@ -115,7 +115,7 @@ typedef struct dfs_options {
                                 as in Alg 3/4                                                       */
     int32_t concurrency;     /* batches: number of traversals run concurrently on the GPU, each on
                                 its own stream and a 1/concurrency share of the SMs (SURVEY
-                                §8(f)-2); 0 = auto (4, capped by the number of roots; a single
+                                §8(f)-2); 0 = auto (8, capped by the number of roots; a single
                                 dfs_run is always 1).  Slots beyond the first allocate their
                                 scratch on first use.                                              */
     int32_t ring_cap;        /* usable HotRing entries (0 = all 256); 2 makes every push spill: the
@@ -148,8 +148,8 @@ typedef struct dfs_options {
     int32_t bulk_copy;       /* 1: flush and refill move the 16-byte-aligned part of each piece with
                                 cp.async.bulk (shared->global, resp. global->shared completing on a
                                 per-warp mbarrier) — the paper's TMA variant;
-                                0 (default): warp-wide 8-byte copies.  Not combinable with
-                                cluster (DFS_EINVAL)                                               */
+                                0: warp-wide 8-byte copies.  Default 1.  Ignored when cluster >= 1
+                                (the cluster build has no bulk variant)                            */
     int32_t spill_period;    /* a busy warp checks the spill condition every spill_period expansion
                                 steps (power of two <= 1024; 0 = 32)                               */
     int32_t reserved[1];     /* zero                                                              */

@@ -70,7 +70,10 @@ enum CounterIdx {
 struct KParams {
     const uint32_t* __restrict__ rp;         // n+1 (narrowed row_ptr; m < 2^32)
     const int32_t* __restrict__ col;         // m (+8 padding)
-    uint32_t* bitmap;                        // ceil(n/32) visited words
+    uint32_t* bitmap;                        // visited words: word k covers vertices 32k..32k+31 at
+                                             // bitmap[k * stride]; 128-wide kernels use stride 2 with
+                                             // the leaf word of the same vertices at +1 (one 8-byte
+                                             // probe = one L2 sector gets both bits)
     const uint32_t* __restrict__ leafmap;    // ceil(n/32) leaf bits (create time), or null
     int32_t* parent;                         // n output
     unsigned long long* cold_tb;             // n_warps: (top << 32) | bottom
@@ -162,6 +165,12 @@ __device__ __forceinline__ uint32_t ld_cg_if(bool p, const uint32_t* a, uint32_t
     uint32_t r = dflt;
     asm volatile("{ .reg .pred q; setp.ne.u32 q, %1, 0; @q ld.global.cg.u32 %0, [%2]; }"
                  : "+r"(r) : "r"((uint32_t)p), "l"(a));
+    return r;
+}
+__device__ __forceinline__ uint2 ld_cg_u2_if(bool p, const uint32_t* a, uint32_t dx, uint32_t dy) {
+    uint2 r = make_uint2(dx, dy);
+    asm volatile("{ .reg .pred q; setp.ne.u32 q, %2, 0; @q ld.global.cg.v2.u32 {%0, %1}, [%3]; }"
+                 : "+r"(r.x), "+r"(r.y) : "r"((uint32_t)p), "l"(a));
     return r;
 }
 __device__ __forceinline__ uint32_t ld_nc_if(bool p, const void* a, uint32_t dflt) {
@@ -1019,7 +1028,7 @@ __global__ void __launch_bounds__(32 * WMAX, 1) dfs_persistent_kernel(const KPar
                     sv = (uint32_t)__shfl_sync(kFull, pick, sk);
                 }
             }
-            uint32_t s_old = atom_or_if(vb != 0 && lane == 0, P.bitmap + (sv >> 5), 1u << (sv & 31));
+            uint32_t s_old = atom_or_if(vb != 0 && lane == 0, P.bitmap + 2u * (sv >> 5), 1u << (sv & 31));
             const uint32_t s_rs = ld_nc_if(vb != 0, P.rp + sv, 0u), s_re = ld_nc_if(vb != 0, P.rp + sv + 1, 0u);
             // probe the visited bits; the lanes holding the first 8 positions also prefetch
             // their candidates' row_ptr pairs
@@ -1030,8 +1039,8 @@ __global__ void __launch_bounds__(32 * WMAX, 1) dfs_persistent_kernel(const KPar
             for (int e = 0; e < VEC; ++e) {
                 const bool ok = (vm >> e) & 1u;
                 const uint32_t x = (uint32_t)nbv[e];
-                const uint32_t word = ld_cg_if(ok, P.bitmap + (x >> 5), kFull);
-                const uint32_t lword = ld_nc_if(ok && P.leafmap != nullptr, P.leafmap + (x >> 5), 0u);
+                const uint2 wl = ld_cg_u2_if(ok, P.bitmap + 2u * (x >> 5), kFull, 0u);   // {visited, leaf}
+                const uint32_t word = wl.x, lword = wl.y;
                 const bool pf = ok && lane < kPfLanes;
                 prs[e] = ld_nc_if(pf, P.rp + x, 0u); pre[e] = ld_nc_if(pf, P.rp + x + 1, 0u);
                 if (ok && !((word >> (x & 31)) & 1u)) {
@@ -1046,7 +1055,7 @@ __global__ void __launch_bounds__(32 * WMAX, 1) dfs_persistent_kernel(const KPar
                 uint32_t lold[VEC];
 #pragma unroll
                 for (int e = 0; e < VEC; ++e)
-                    lold[e] = atom_or_if((lcm >> e) & 1u, P.bitmap + ((uint32_t)nbv[e] >> 5), 1u << (nbv[e] & 31));
+                    lold[e] = atom_or_if((lcm >> e) & 1u, P.bitmap + 2u * ((uint32_t)nbv[e] >> 5), 1u << (nbv[e] & 31));
                 uint32_t nl = 0;
 #pragma unroll
                 for (int e = 0; e < VEC; ++e) {
@@ -1107,7 +1116,7 @@ __global__ void __launch_bounds__(32 * WMAX, 1) dfs_persistent_kernel(const KPar
                 uint32_t cre = __shfl_sync(kFull, mine_re, k & (kPfLanes - 1));
                 if (k >= kPfLanes) { crs = __ldg(P.rp + cv); cre = __ldg(P.rp + cv + 1); }
                 const uint32_t bit = 1u << (cv & 31);
-                uint32_t old = atom_or_if(lane == 0, P.bitmap + (cv >> 5), bit);
+                uint32_t old = atom_or_if(lane == 0, P.bitmap + 2u * (cv >> 5), bit);
                 load_window(crs & ~(uint32_t)(VEC - 1), cre, 32, cnb);   // overlaps the claim
                 old = __shfl_sync(kFull, old, 0);
                 if (!(old & bit)) { won = true; v = cv; vrs = crs; vre = cre; kl = k; ke = e; continue; }
@@ -1449,7 +1458,10 @@ exit_loop:
 // ------------------------------------------------------------------------------------------
 // per-traversal reset (step a2) and finalize (step a9)
 // ------------------------------------------------------------------------------------------
-__global__ void dfs_reset_kernel(uint32_t* bitmap, uint32_t nwords, unsigned long long* cold_tb,
+// bitmap layout: bstride = 1 (32-wide kernels) or 2 (128-wide: {visited, leaf} word pairs; the
+// leaf words are copied from the graph's leaf map, or zero when bulk leaf claims are off)
+__global__ void dfs_reset_kernel(uint32_t* bitmap, uint32_t nwords, uint32_t bstride, const uint32_t* leaf,
+                                 unsigned long long* cold_tb,
                                  uint32_t n_warps, int* block_cold, uint32_t n_blocks, Ctl* ctl,
                                  int32_t* parent, int root, uint32_t* chunk_tab, size_t tab_words) {
     const size_t tid = blockIdx.x * (size_t)blockDim.x + threadIdx.x;
@@ -1457,7 +1469,11 @@ __global__ void dfs_reset_kernel(uint32_t* bitmap, uint32_t nwords, unsigned lon
     for (size_t k = tid; k < nwords; k += stride) {
         uint32_t v = 0;
         if (k == ((uint32_t)root >> 5)) v = 1u << (root & 31);    // Alg 1 l.1: visited[root]
-        bitmap[k] = v;
+        if (bstride == 2) {
+            reinterpret_cast<uint2*>(bitmap)[k] = make_uint2(v, leaf ? leaf[k] : 0u);
+        } else {
+            bitmap[k] = v;
+        }
     }
     for (size_t k = tid; k < n_warps; k += stride) cold_tb[k] = 0ull;
     for (size_t k = tid; k < n_blocks; k += stride) block_cold[k] = 0;
@@ -1474,23 +1490,23 @@ __global__ void dfs_reset_kernel(uint32_t* bitmap, uint32_t nwords, unsigned lon
     }
 }
 
-__global__ void dfs_finalize_kernel(const uint32_t* __restrict__ bitmap, int32_t* parent, uint32_t n,
+__global__ void dfs_finalize_kernel(const uint32_t* __restrict__ bitmap, uint32_t bstride, int32_t* parent, uint32_t n,
                                     const Ctl* ctl, int* status_acc) {
     const size_t stride = (size_t)gridDim.x * blockDim.x;
     if (blockIdx.x == 0 && threadIdx.x == 0 && ctl->status != 0) atomicMin(status_acc, ctl->status);
     for (size_t v = blockIdx.x * (size_t)blockDim.x + threadIdx.x; v < n; v += stride) {
-        const uint32_t word = __ldg(bitmap + (v >> 5));
+        const uint32_t word = __ldg(bitmap + bstride * (v >> 5));
         if (!((word >> (v & 31)) & 1u)) parent[v] = -2;            // DFS_UNREACHED (reading S2)
     }
 }
 
 // visited count and TEPS numerator (sum of out-degrees of visited vertices)
-__global__ void dfs_count_kernel(const uint32_t* __restrict__ bitmap, const uint32_t* __restrict__ rp,
+__global__ void dfs_count_kernel(const uint32_t* __restrict__ bitmap, uint32_t bstride, const uint32_t* __restrict__ rp,
                                  uint32_t n, unsigned long long* out2) {
     unsigned long long nv = 0, mv = 0;
     const size_t stride = (size_t)gridDim.x * blockDim.x;
     for (size_t v = blockIdx.x * (size_t)blockDim.x + threadIdx.x; v < n; v += stride) {
-        if ((__ldg(bitmap + (v >> 5)) >> (v & 31)) & 1u) { ++nv; mv += __ldg(rp + v + 1) - __ldg(rp + v); }
+        if ((__ldg(bitmap + bstride * (v >> 5)) >> (v & 31)) & 1u) { ++nv; mv += __ldg(rp + v + 1) - __ldg(rp + v); }
     }
     for (int o = 16; o > 0; o >>= 1) {
         nv += __shfl_down_sync(kFull, nv, o);

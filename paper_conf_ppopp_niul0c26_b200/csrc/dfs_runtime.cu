@@ -63,6 +63,7 @@ size_t smem_bytes(int warps) {
 struct Slot {
     bool ready = false;
     uint32_t* bitmap = nullptr;
+    uint32_t bstride = 1;                   // bitmap layout of the last launch (1, or 2 = {visited, leaf})
     int32_t* parent = nullptr;              // lazily allocated for host outputs
     unsigned long long* cold_tb = nullptr;
     uint32_t* tab = nullptr;
@@ -137,7 +138,7 @@ static int ensure_slot(dfs_graph* g, int k) {
     const size_t nwords = (size_t)((n + 31) / 32);
     bool ok = true;
     auto A = [&](void** p, size_t bytes) { if (ok && cudaMalloc(p, bytes ? bytes : 16) != cudaSuccess) ok = false; };
-    A((void**)&s.bitmap, nwords * sizeof(uint32_t));
+    A((void**)&s.bitmap, 2 * nwords * sizeof(uint32_t));      // room for the {visited, leaf} layout
     A((void**)&s.cold_tb, (size_t)n_warps * sizeof(unsigned long long));
     A((void**)&s.tab, s.tab_words * sizeof(uint32_t));
     A((void**)&s.pool, (size_t)s.n_chunks * kChunk * sizeof(unsigned long long));
@@ -191,6 +192,7 @@ void dfs_options_default(dfs_options* o) {
     o->max_pool_chunks = 0;
     o->leaf_skip = 2;            // A/B on B200: rmat22 5.20 -> 4.33 ms (bulk), others neutral
     o->steal_tries = 8;          // A/B on B200: road 16.8 -> 15.4 ms, grid -15%, others neutral
+    o->bulk_copy = 1;            // A/B on B200: rmat24 -11%, caterpillar -18%, road -2%, path -1%
 }
 
 int dfs_last_error(void) { return g_last_error; }
@@ -356,7 +358,10 @@ static int launch_one(dfs_graph* g, Slot& sl, cudaStream_t s, int32_t root, int3
     const uint32_t nwords = (uint32_t)((g->n + 31) / 32);
     const int rblocks = (int)std::min<int64_t>((std::max<int64_t>(nwords, sl.tab_dirty ? (int64_t)sl.tab_words : 0) + 255) / 256 + 1,
                                                (int64_t)g->sms * 8);
-    dfs_reset_kernel<<<rblocks, 256, 0, s>>>(sl.bitmap, nwords, sl.cold_tb, (uint32_t)(blocks * warps),
+    const uint32_t bstride = o.window == 128 ? 2u : 1u;
+    sl.bstride = bstride;
+    dfs_reset_kernel<<<rblocks, 256, 0, s>>>(sl.bitmap, nwords, bstride, o.leaf_skip >= 2 ? g->d_leaf : nullptr,
+                                            sl.cold_tb, (uint32_t)(blocks * warps),
                                             sl.block_cold, (uint32_t)blocks, sl.ctl, d_out, root,
                                             sl.tab, sl.tab_dirty ? sl.tab_words : 0);
     g->launches++;
@@ -365,6 +370,7 @@ static int launch_one(dfs_graph* g, Slot& sl, cudaStream_t s, int32_t root, int3
     KParams P;
     P.rp = g->d_rp; P.col = g->d_col; P.bitmap = sl.bitmap; P.parent = d_out;
     P.leafmap = o.leaf_skip >= 2 ? g->d_leaf : nullptr;     // 2: also claim leaf candidates in bulk
+                                                             // (128-wide: leaf words in the bitmap)
     P.cold_tb = sl.cold_tb; P.chunk_tab = sl.tab; P.pool = sl.pool;
     P.chunk_consumed = sl.consumed; P.chunk_next = sl.next; P.block_cold = sl.block_cold;
     P.ctl = sl.ctl;
@@ -397,7 +403,8 @@ static int launch_one(dfs_graph* g, Slot& sl, cudaStream_t s, int32_t root, int3
     P.seed = o.seed;
     void* args[] = {(void*)&P};
     const int cl = o.cluster > 1 ? o.cluster : 1;
-    const void* kfn = kernel_table()[(o.bulk_copy ? 16 : o.cluster >= 1 ? 8 : 0) + (o.window == 128 ? 4 : 0) +
+    // the cluster build has no bulk variant: cluster >= 1 takes precedence over bulk_copy
+    const void* kfn = kernel_table()[(o.cluster >= 1 ? 8 : o.bulk_copy ? 16 : 0) + (o.window == 128 ? 4 : 0) +
                                      (warps <= 16 ? 2 : 0) + (o.collect_stats ? 1 : 0)];
     if (timed) cudaEventRecord(sl.evk0, s);
     cudaError_t e;
@@ -425,7 +432,7 @@ static int launch_one(dfs_graph* g, Slot& sl, cudaStream_t s, int32_t root, int3
     if (timed) cudaEventRecord(sl.evk1, s);
     g->launches++;
     const int fblocks = (int)std::min<int64_t>((g->n + 255) / 256, (int64_t)g->sms * 16);
-    dfs_finalize_kernel<<<fblocks, 256, 0, s>>>(sl.bitmap, d_out, (uint32_t)g->n, sl.ctl, sl.status);
+    dfs_finalize_kernel<<<fblocks, 256, 0, s>>>(sl.bitmap, bstride, d_out, (uint32_t)g->n, sl.ctl, sl.status);
     g->launches++;
     return DFS_OK;
 }
@@ -463,7 +470,6 @@ static int resolve_options(dfs_graph* g, const dfs_options* in, int num_roots, d
     if (o.cold_cutoff < 1 || o.cold_cutoff / 2 > 64) return DFS_EINVAL;
     if (o.victim_policy != 0 && o.victim_policy != 1) return DFS_EINVAL;
     if (o.reserved0 != 0) return DFS_EINVAL;
-    if (o.bulk_copy && o.cluster >= 1) return DFS_EINVAL;     // no bulk + cluster instantiation
     if (o.spill_period < 0 || o.spill_period > 1024 || (o.spill_period & (o.spill_period - 1))) return DFS_EINVAL;
     if (o.cluster < 0 || o.cluster > 8 || (o.cluster > 1 && (o.cluster & (o.cluster - 1)))) return DFS_EINVAL;
     if (o.window == 0) o.window = (g->n > 0 && g->m >= 8 * g->n) ? 128 : 32;   // wide windows for dense lists
@@ -471,7 +477,7 @@ static int resolve_options(dfs_graph* g, const dfs_options* in, int num_roots, d
     if (o.concurrency < 0 || o.concurrency > kMaxSlots) return DFS_EINVAL;
     warps = o.warps_per_block <= 0 ? 32 : o.warps_per_block;
     if (warps > 32) return DFS_EINVAL;
-    conc = o.concurrency == 0 ? 4 : o.concurrency;       // auto: 4 in flight (B200 sweep)
+    conc = o.concurrency == 0 ? 8 : o.concurrency;       // auto: 8 in flight (B200 sweep)
     if (o.deterministic) conc = 1;
     if (conc > num_roots) conc = std::max(1, num_roots);
     const int share = std::max(1, g->max_blocks / conc);
@@ -589,7 +595,7 @@ static int run_sequential(dfs_graph* g, const int32_t* roots, int32_t k, int32_t
         if (rc != DFS_OK) return fail(rc);
         cudaEventRecord(sl.ev1, s);
         if (stats) {
-            dfs_count_kernel<<<g->sms * 4, 256, 0, s>>>(sl.bitmap, g->d_rp, (uint32_t)g->n, g->d_counts + 2 * q);
+            dfs_count_kernel<<<g->sms * 4, 256, 0, s>>>(sl.bitmap, sl.bstride, g->d_rp, (uint32_t)g->n, g->d_counts + 2 * q);
             g->launches++;
         }
         Ctl h;
@@ -672,7 +678,7 @@ static int run_concurrent(dfs_graph* g, const int32_t* roots, int32_t k, int32_t
         int rc = launch_one(g, sl, sl.stream, roots[q], d_out, o, blocks, warps, false, false);
         if (rc != DFS_OK) return fail(rc);
         if (stats) {
-            dfs_count_kernel<<<g->sms * 4, 256, 0, sl.stream>>>(sl.bitmap, g->d_rp, (uint32_t)g->n, g->d_counts + 2 * q);
+            dfs_count_kernel<<<g->sms * 4, 256, 0, sl.stream>>>(sl.bitmap, sl.bstride, g->d_rp, (uint32_t)g->n, g->d_counts + 2 * q);
             g->launches++;
         }
         if (!out_dev) {

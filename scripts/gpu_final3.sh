@@ -7,7 +7,7 @@ for c in road24m grid256 rmat24 path100m caterpillar; do
   timeout 900 python bench.py --config $c --steps 8 --warmup 3 --cpu-seconds 10 > gpurun_out/r01d/bench_$c.json 2> gpurun_out/r01d/bench_$c.err
   python -c "import json; d=json.load(open('gpurun_out/r01d/bench_$c.json')); print('$c', d['value'], d['ms_per_dfs'], 'cpu', d.get('cpu_baseline',{}).get('value'), 'e2e', d.get('e2e',{}).get('value'), 'roof', d['roofline']['frac'], 'traffic', d['roofline']['traffic'])" || tail -3 gpurun_out/r01d/bench_$c.err
 done
-for k in 0 2 6 8; do
+for k in 0 4; do
 timeout 900 python bench.py --config batch1024 --warmup 3 --concurrency $k > gpurun_out/r01d/bench_batch1024_k$k.json 2> gpurun_out/r01d/bench_batch1024_k$k.err
 python -c "import json; d=json.load(open('gpurun_out/r01d/bench_batch1024_k$k.json')); print('batch1024', d['value'], d['dfs_per_s'], d['concurrency'])"
 done
