@@ -152,7 +152,12 @@ typedef struct dfs_options {
                                 (the cluster build has no bulk variant)                            */
     int32_t spill_period;    /* a busy warp checks the spill condition every spill_period expansion
                                 steps (power of two <= 1024; 0 = 32)                               */
-    int32_t reserved[1];     /* zero                                                              */
+    int32_t l2_persist_mb;   /* > 0: set the device's persisting-L2 limit to this many MB (capped by
+                                cudaDevAttrMaxPersistingL2CacheSize; device-wide) and launch the
+                                traversal with an access-policy window that keeps row_ptr persisting
+                                in L2 while col_idx streams.  0 (default) = auto: 64 MB with
+                                128-wide windows (A/B on B200: RMAT-24 -4.8%, road/path neutral),
+                                else off; -1 = off.  The limit stays set after the handle is gone  */
 } dfs_options;
 
 typedef struct dfs_stats {

@@ -91,6 +91,8 @@ struct dfs_graph {
     int sms = 0;
     int max_blocks = 0;          // co-resident 32-warp blocks (allocation bound)
     int max_clusters[4] = {0, 0, 0, 0};   // co-resident clusters of 1/2/4/8 CTAs (lazy)
+    size_t persist_bytes = 0;    // persisting-L2 set-aside granted for l2_persist_mb (0 = none)
+    size_t max_window_bytes = 0; // cudaDevAttrMaxAccessPolicyWindowSize
     int tab_log2 = 0;
     uint32_t* d_rp = nullptr;
     int32_t* d_col = nullptr;    // col_idx (+8 padding for 128-bit window loads)
@@ -408,26 +410,38 @@ static int launch_one(dfs_graph* g, Slot& sl, cudaStream_t s, int32_t root, int3
                                      (warps <= 16 ? 2 : 0) + (o.collect_stats ? 1 : 0)];
     if (timed) cudaEventRecord(sl.evk0, s);
     cudaError_t e;
+    // launch attributes: cooperative (single traversals), cluster dimension (cluster tier,
+    // blocks is a multiple of cl and at most cl x the co-resident cluster count,
+    // resolve_options), and an L2 access-policy window that keeps row_ptr persisting in L2
+    // (l2_persist_mb; the window's hits are persisting, its misses streaming)
+    cudaLaunchConfig_t cfg = {};
+    cudaLaunchAttribute at[3];
+    int na = 0;
+    at[na].id = cudaLaunchAttributeCooperative;
+    at[na].val.cooperative = cooperative ? 1 : 0;
+    ++na;
     if (o.cluster >= 1) {
-        // cluster tier: clusters of `cl` CTAs; blocks is a multiple of cl and at
-        // most cl x the co-resident cluster count (resolve_options)
-        cudaLaunchConfig_t cfg = {};
-        cudaLaunchAttribute at[2];
-        at[0].id = cudaLaunchAttributeClusterDimension;
-        at[0].val.clusterDim.x = (unsigned)cl; at[0].val.clusterDim.y = 1; at[0].val.clusterDim.z = 1;
-        at[1].id = cudaLaunchAttributeCooperative;
-        at[1].val.cooperative = cooperative ? 1 : 0;
-        cfg.gridDim = dim3(blocks); cfg.blockDim = dim3(32 * warps);
-        cfg.dynamicSmemBytes = smem_bytes(warps); cfg.stream = s;
-        cfg.attrs = at; cfg.numAttrs = 2;
-        e = cudaLaunchKernelExC(&cfg, kfn, args);
-    } else if (cooperative) {
-        e = cudaLaunchCooperativeKernel(kfn, dim3(blocks), dim3(32 * warps), args, smem_bytes(warps), s);
-    } else {
-        // concurrent batch slots: co-residency is not required for progress — a block that starts
-        // late finds the traversal done or steals the remaining work
-        e = cudaLaunchKernel(kfn, dim3(blocks), dim3(32 * warps), args, smem_bytes(warps), s);
+        at[na].id = cudaLaunchAttributeClusterDimension;
+        at[na].val.clusterDim.x = (unsigned)cl; at[na].val.clusterDim.y = 1; at[na].val.clusterDim.z = 1;
+        ++na;
     }
+    if (o.l2_persist_mb > 0 && g->persist_bytes > 0) {
+        const size_t rp_bytes = (size_t)(g->n + 1) * sizeof(uint32_t);
+        const size_t win = std::min(rp_bytes, g->max_window_bytes);
+        at[na].id = cudaLaunchAttributeAccessPolicyWindow;
+        at[na].val.accessPolicyWindow.base_ptr = (void*)g->d_rp;
+        at[na].val.accessPolicyWindow.num_bytes = win;
+        at[na].val.accessPolicyWindow.hitRatio = std::min(1.0f, (float)g->persist_bytes / (float)win);
+        at[na].val.accessPolicyWindow.hitProp = cudaAccessPropertyPersisting;
+        at[na].val.accessPolicyWindow.missProp = cudaAccessPropertyStreaming;
+        ++na;
+    }
+    cfg.gridDim = dim3(blocks); cfg.blockDim = dim3(32 * warps);
+    cfg.dynamicSmemBytes = smem_bytes(warps); cfg.stream = s;
+    cfg.attrs = at; cfg.numAttrs = na;
+    // concurrent batch slots launch non-cooperatively: co-residency is not required for progress —
+    // a block that starts late finds the traversal done or steals the remaining work
+    e = cudaLaunchKernelExC(&cfg, kfn, args);
     if (e != cudaSuccess) { cudaGetLastError(); return DFS_ECUDA; }
     if (timed) cudaEventRecord(sl.evk1, s);
     g->launches++;
@@ -484,6 +498,24 @@ static int resolve_options(dfs_graph* g, const dfs_options* in, int num_roots, d
     blocks = o.blocks <= 0 ? share : o.blocks;
     if (blocks > g->max_blocks || (conc > 1 && blocks * conc > g->max_blocks)) return DFS_EINVAL;
     if (o.deterministic) { blocks = 1; warps = 1; o.intra_steal = 0; o.inter_steal = 0; o.cluster = 0; }
+    if (o.l2_persist_mb < -1) return DFS_EINVAL;
+    if (o.l2_persist_mb == 0) o.l2_persist_mb = o.window == 128 ? 64 : -1;   // auto (A/B: rmat24 -4.8%)
+    if (o.l2_persist_mb > 0) {
+        // device-wide persisting-L2 set-aside (capped by the device); done once per handle
+        const size_t want = (size_t)o.l2_persist_mb << 20;
+        if (g->persist_bytes != want) {
+            int maxp = 0, maxw = 0;
+            cudaDeviceGetAttribute(&maxp, cudaDevAttrMaxPersistingL2CacheSize, g->device);
+            cudaDeviceGetAttribute(&maxw, cudaDevAttrMaxAccessPolicyWindowSize, g->device);
+            const size_t bytes = std::min(want, (size_t)maxp);
+            if (bytes == 0 || maxw <= 0 || cudaDeviceSetLimit(cudaLimitPersistingL2CacheSize, bytes) != cudaSuccess) {
+                cudaGetLastError();
+                return DFS_ECUDA;
+            }
+            g->persist_bytes = want;
+            g->max_window_bytes = (size_t)maxw;
+        }
+    }
     if (o.cluster > 1) {
         // whole clusters only, no more than can be co-resident
         const int maxc = max_clusters(g, o.cluster, warps, o.window, o.collect_stats != 0);

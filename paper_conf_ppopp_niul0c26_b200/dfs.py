@@ -52,7 +52,7 @@ class _Options(ctypes.Structure):
                 ("leaf_skip", ctypes.c_int32), ("cluster", ctypes.c_int32),
                 ("cluster_late", ctypes.c_int32), ("steal_tries", ctypes.c_int32),
                 ("bulk_copy", ctypes.c_int32), ("spill_period", ctypes.c_int32),
-                ("reserved", ctypes.c_int32 * 1)]
+                ("l2_persist_mb", ctypes.c_int32)]
 
 
 class _Stats(ctypes.Structure):
@@ -103,6 +103,7 @@ class Options:
     steal_tries: Optional[int] = None
     bulk_copy: Optional[bool] = None
     spill_period: Optional[int] = None
+    l2_persist_mb: Optional[int] = None
 
     def to_c(self) -> _Options:
         o = _Options()

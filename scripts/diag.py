@@ -133,6 +133,10 @@ VARIANTS = {
     "bulk_copy": dict(bulk_copy=True),
     "bulk_copy_v1": dict(bulk_copy=True, ring_cap=2),
     "v1": dict(ring_cap=2),
+    "l2p32": dict(l2_persist_mb=32),
+    "l2off": dict(l2_persist_mb=-1),
+    "l2p64": dict(l2_persist_mb=64),
+    "l2p96": dict(l2_persist_mb=96),
     "w0nointra": dict(collect_stats=2, intra_steal=False),
     "sp8": dict(spill_period=8),
     "sp16": dict(spill_period=16),

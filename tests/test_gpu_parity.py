@@ -170,6 +170,7 @@ def test_parallel_directed_with_self_loops_and_duplicates():
     dict(steal_tries=8, warps_per_block=8, blocks=4, spill=False),
     dict(speculate=2 | 4 | 8),
     dict(bulk_copy=True),                                             # cp.async.bulk flush/refill
+    dict(bulk_copy=False, l2_persist_mb=16),                          # warp copies; L2 policy window
     dict(bulk_copy=True, ring_cap=3, hot_cutoff=2, cold_cutoff=2, window=128),
 ])
 def test_stress_options(opts):
