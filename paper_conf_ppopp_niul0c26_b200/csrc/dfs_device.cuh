@@ -70,10 +70,10 @@ enum CounterIdx {
 struct KParams {
     const uint32_t* __restrict__ rp;         // n+1 (narrowed row_ptr; m < 2^32)
     const int32_t* __restrict__ col;         // m (+8 padding)
-    uint32_t* bitmap;                        // visited words: word k covers vertices 32k..32k+31 at
-                                             // bitmap[k * stride]; 128-wide kernels use stride 2 with
-                                             // the leaf word of the same vertices at +1 (one 8-byte
-                                             // probe = one L2 sector gets both bits)
+    uint32_t* bitmap;                        // {visited, leaf} word pairs: bitmap[2k] holds the
+                                             // visited bits of vertices 32k..32k+31, bitmap[2k+1]
+                                             // their leaf bits (one 8-byte probe = one L2 sector
+                                             // returns both)
     const uint32_t* __restrict__ leafmap;    // ceil(n/32) leaf bits (create time), or null
     int32_t* parent;                         // n output
     unsigned long long* cold_tb;             // n_warps: (top << 32) | bottom
@@ -156,6 +156,10 @@ __device__ __forceinline__ uint32_t atom_or_if(bool p, uint32_t* a, uint32_t b) 
     asm volatile("{ .reg .pred q; setp.ne.u32 q, %1, 0; @q atom.global.or.b32 %0, [%2], %3; }"
                  : "+r"(r) : "r"((uint32_t)p), "l"(a), "r"(b) : "memory");
     return r;
+}
+__device__ __forceinline__ void red_or_if(bool p, uint32_t* a, uint32_t b) {
+    asm volatile("{ .reg .pred q; setp.ne.u32 q, %0, 0; @q red.global.or.b32 [%1], %2; }"
+                 ::"r"((uint32_t)p), "l"(a), "r"(b) : "memory");
 }
 __device__ __forceinline__ void st_global_if(bool p, int32_t* a, int32_t v) {
     asm volatile("{ .reg .pred q; setp.ne.u32 q, %0, 0; @q st.global.s32 [%1], %2; }"
@@ -879,17 +883,34 @@ __global__ void __launch_bounds__(32 * WMAX, 1) dfs_persistent_kernel(const KPar
             const uint32_t vb = __ballot_sync(kFull, spec_ok && valid && (uint32_t)nb != par);
             const int sk = __ffs(vb) - 1;
             const uint32_t sv = vb ? (uint32_t)__shfl_sync(kFull, nb, sk & 31) : u;
-            uint32_t s_old = atom_or_if(vb != 0 && lane == 0, P.bitmap + (sv >> 5), 1u << (sv & 31));
+            uint32_t s_old = atom_or_if(vb != 0 && lane == 0, P.bitmap + 2u * (sv >> 5), 1u << (sv & 31));
             const uint32_t s_rs = ld_nc_if(vb != 0, P.rp + sv, 0u), s_re = ld_nc_if(vb != 0, P.rp + sv + 1, 0u);
             // probe the visited bits; lanes holding the first 8 positions prefetch their
             // candidates' row_ptr pairs
-            const uint32_t word = ld_cg_if(valid, P.bitmap + ((uint32_t)nb >> 5), kFull);
+            const uint2 wl = ld_cg_u2_if(valid, P.bitmap + 2u * ((uint32_t)nb >> 5), kFull, 0u);   // {visited, leaf}
             const bool pf = valid && lane < kPfLanes;
             const uint32_t prs = ld_nc_if(pf, P.rp + nb, 0u), pre = ld_nc_if(pf, P.rp + nb + 1, 0u);
             // early child window (speculate & 4): issued once the row_ptr pair arrives, before
             // the claim returns (the probes are already in flight)
             int cnb = (int)ld_nc_if(spec_early && vb != 0 && s_rs + lane < s_re, P.col + s_rs + lane, kFull);
-            bool cand = valid && !((word >> (nb & 31)) & 1u) && lane != sk;   // sk is claimed either way
+            const bool unv = valid && !((wl.x >> (nb & 31)) & 1u) && lane != sk;   // sk is claimed either way
+            const bool lf = unv && ((wl.y >> (nb & 31)) & 1u);
+            bool cand = unv && !lf;
+            // bulk leaf claims (leaf_skip = 2): every unvisited leaf candidate of the window is
+            // claimed at once, in parallel with the claim of the next tree edge — each is exactly
+            // Alg 1's descend-and-pop-back (a leaf's only in-list is u's, reading S24)
+            // No other list holds a leaf and this warp is the only scanner of u's list, so the
+            // probe's "unvisited" cannot change before the claim: a fire-and-forget red.or sets
+            // the bit (the step does not wait for it) and the parent is u in every order.
+            if (__any_sync(kFull, lf)) {
+                red_or_if(lf, P.bitmap + 2u * ((uint32_t)nb >> 5), 1u << (nb & 31));
+                st_global_if(lf, P.parent + nb, (int32_t)u);                    // Alg 1 l.10
+                if (STATS || P.block_claims || P.timeline) {
+                    const uint32_t nl = __popc(__ballot_sync(kFull, lf));
+                    my_claims += nl;
+                    if (STATS && lane == 0) cnt[kCntClaims] += nl;
+                }
+            }
             s_old = __shfl_sync(kFull, s_old, 0);
             bool won = vb != 0 && !(s_old & (1u << (sv & 31)));
             uint32_t v = sv, vrs = s_rs, vre = s_re;
@@ -906,7 +927,7 @@ __global__ void __launch_bounds__(32 * WMAX, 1) dfs_persistent_kernel(const KPar
                     uint32_t crs = __shfl_sync(kFull, prs, k & (kPfLanes - 1)), cre = __shfl_sync(kFull, pre, k & (kPfLanes - 1));
                     if (k >= kPfLanes) { crs = __ldg(P.rp + cv); cre = __ldg(P.rp + cv + 1); }
                     const uint32_t bit = 1u << (cv & 31);
-                    uint32_t old = atom_or_if(lane == 0, P.bitmap + (cv >> 5), bit);
+                    uint32_t old = atom_or_if(lane == 0, P.bitmap + 2u * (cv >> 5), bit);
                     cnb = (int)ld_nc_if(crs + lane < cre, P.col + crs + lane, kFull);   // overlaps the claim
                     old = __shfl_sync(kFull, old, 0);
                     if (!(old & bit)) { won = true; v = cv; vrs = crs; vre = cre; kpos = k; break; }
@@ -1051,17 +1072,16 @@ __global__ void __launch_bounds__(32 * WMAX, 1) dfs_persistent_kernel(const KPar
             // bulk leaf claims (leaf_skip = 2, 128-wide windows): every unvisited leaf candidate
             // of the window is claimed at once — each is exactly Alg 1's descend-and-pop-back
             // (a leaf's only in-list is u's, so its parent is u in any order)
+            // (fire-and-forget red.or: no other list holds a leaf and this warp is the only
+            // scanner of u's list, so the probe's "unvisited" still holds — see the 32-wide step)
             if (__any_sync(kFull, lcm != 0)) {
-                uint32_t lold[VEC];
-#pragma unroll
-                for (int e = 0; e < VEC; ++e)
-                    lold[e] = atom_or_if((lcm >> e) & 1u, P.bitmap + 2u * ((uint32_t)nbv[e] >> 5), 1u << (nbv[e] & 31));
                 uint32_t nl = 0;
 #pragma unroll
                 for (int e = 0; e < VEC; ++e) {
-                    const bool lwon = ((lcm >> e) & 1u) && !(lold[e] & (1u << (nbv[e] & 31)));
-                    st_global_if(lwon, P.parent + nbv[e], (int32_t)u);           // Alg 1 l.10
-                    nl += lwon;
+                    const bool lf = (lcm >> e) & 1u;
+                    red_or_if(lf, P.bitmap + 2u * ((uint32_t)nbv[e] >> 5), 1u << (nbv[e] & 31));
+                    st_global_if(lf, P.parent + nbv[e], (int32_t)u);             // Alg 1 l.10
+                    nl += lf;
                 }
                 if (STATS || P.block_claims || P.timeline) {
                     nl = __reduce_add_sync(kFull, nl);

@@ -360,7 +360,7 @@ static int launch_one(dfs_graph* g, Slot& sl, cudaStream_t s, int32_t root, int3
     const uint32_t nwords = (uint32_t)((g->n + 31) / 32);
     const int rblocks = (int)std::min<int64_t>((std::max<int64_t>(nwords, sl.tab_dirty ? (int64_t)sl.tab_words : 0) + 255) / 256 + 1,
                                                (int64_t)g->sms * 8);
-    const uint32_t bstride = o.window == 128 ? 2u : 1u;
+    const uint32_t bstride = 2u;                              // {visited, leaf} pairs (both windows)
     sl.bstride = bstride;
     dfs_reset_kernel<<<rblocks, 256, 0, s>>>(sl.bitmap, nwords, bstride, o.leaf_skip >= 2 ? g->d_leaf : nullptr,
                                             sl.cold_tb, (uint32_t)(blocks * warps),
