@@ -128,9 +128,10 @@ typedef struct dfs_options {
     int32_t leaf_skip;       /* 1: a claimed child whose list is empty or holds only its parent is
                                 finished in place — Alg 1 would descend and pop straight back — so
                                 the parent's window scan continues without a push/pop round trip.
-                                2 (default): in addition, 128-wide windows claim every unvisited
-                                leaf candidate at once (leaf map built at create: out-degree 0, or
-                                1 whose only in-list is its neighbour's).  0: always descend       */
+                                2 (default): in addition, every window claims all its unvisited
+                                leaf candidates at once (leaf map built at create: all in-edges
+                                from one vertex w, out-list empty, [w] or [v]; S24).
+                                0: always descend                                                  */
     int32_t cluster;         /* cluster steal tier: 2, 4 or 8 = launch the persistent
                                 grid as thread-block clusters of that many CTAs; an idle warp that
                                 finds no Alg 3 victim in its own CTA steals from the HotRings of the

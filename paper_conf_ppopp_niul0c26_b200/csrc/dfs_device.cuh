@@ -74,7 +74,6 @@ struct KParams {
                                              // visited bits of vertices 32k..32k+31, bitmap[2k+1]
                                              // their leaf bits (one 8-byte probe = one L2 sector
                                              // returns both)
-    const uint32_t* __restrict__ leafmap;    // ceil(n/32) leaf bits (create time), or null
     int32_t* parent;                         // n output
     unsigned long long* cold_tb;             // n_warps: (top << 32) | bottom
     uint32_t* chunk_tab;                     // n_warps << tab_log2

@@ -371,8 +371,6 @@ static int launch_one(dfs_graph* g, Slot& sl, cudaStream_t s, int32_t root, int3
 
     KParams P;
     P.rp = g->d_rp; P.col = g->d_col; P.bitmap = sl.bitmap; P.parent = d_out;
-    P.leafmap = o.leaf_skip >= 2 ? g->d_leaf : nullptr;     // 2: also claim leaf candidates in bulk
-                                                             // (128-wide: leaf words in the bitmap)
     P.cold_tb = sl.cold_tb; P.chunk_tab = sl.tab; P.pool = sl.pool;
     P.chunk_consumed = sl.consumed; P.chunk_next = sl.next; P.block_cold = sl.block_cold;
     P.ctl = sl.ctl;
