@@ -20,6 +20,11 @@ METRICS = [
     "launch__registers_per_thread", "launch__grid_size", "launch__block_size",
     "lts__t_sectors_op_atom.sum", "lts__t_sectors_op_red.sum", "lts__t_sectors_op_read.sum",
     "lts__t_sectors_op_write.sum", "sm__pipe_tensor_cycles_active.avg.pct_of_peak_sustained_active",
+    # atomic throughput (claims: atom.or; leaf claims: red.or; stack control: atom.cas)
+    "lts__t_requests_srcunit_tex_op_atom_dot_alu.sum", "lts__t_requests_srcunit_tex_op_atom_dot_cas.sum",
+    "lts__t_requests_srcunit_tex_op_red.sum", "lts__t_sectors_srcunit_tex_op_atom_dot_alu.avg.per_cycle_elapsed",
+    "lts__t_sectors_srcunit_tex_op_atom_dot_alu.avg.peak_sustained",
+    "lts__t_sectors_srcunit_tex_op_atom_dot_alu_lookup_hit.sum",
 ]
 
 
