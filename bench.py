@@ -323,7 +323,8 @@ def batch_arm(a, world, rank, local):
     G = Graph(g.row_ptr, g.col_idx)
     lo, hi = batch.partition(len(roots), world, rank)
     conc = a.concurrency if a.concurrency > 0 else 8          # library auto (DESIGN §8 sweep)
-    out_rows = torch.empty((max(conc, min(16, max(1, hi - lo))), g.n), dtype=torch.int32, device=dev)
+    # chunks of 4 waves of `conc` traversals (device-resident parent rows, 96 MB each)
+    out_rows = torch.empty((max(1, min(4 * conc, hi - lo)), g.n), dtype=torch.int32, device=dev)
     for s_ in range(a.warmup):                       # warm-up traversals (untimed)
         G.run(int(roots[(lo + s_) % len(roots)]), out=out_rows[0])
     launches0 = G.launch_count()

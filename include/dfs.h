@@ -116,8 +116,8 @@ typedef struct dfs_options {
     int32_t concurrency;     /* batches: number of traversals run concurrently on the GPU, each on
                                 its own stream and a 1/concurrency share of the SMs (SURVEY
                                 §8(f)-2); 0 = auto (8, capped by the number of roots; a single
-                                dfs_run is always 1).  Slots beyond the first allocate their
-                                scratch on first use.                                              */
+                                dfs_run is always 1; at most 16).  Slots beyond the first allocate
+                                their scratch on first use.                                        */
     int32_t ring_cap;        /* usable HotRing entries (0 = all 256); 2 makes every push spill: the
                                 "one-level stack" of the paper's v1 (Fig 8)            */
     int32_t backoff_min_ns;  /* first __nanosleep of an idle warp's backoff; default 32           */

@@ -28,7 +28,7 @@ using namespace b200dfs;
 namespace {
 
 constexpr int kRing = DFS_KRING;            // HotRing entries per warp (P:367 uses 128)
-constexpr int kMaxSlots = 8;                 // concurrent traversals per handle (batches)
+constexpr int kMaxSlots = 16;                // concurrent traversals per handle (batches)
 thread_local int g_last_error = DFS_OK;
 
 int fail(int code) { g_last_error = code; return code; }
