@@ -185,6 +185,9 @@ typedef struct dfs_stats {
        claims (tree vertices discovered) per block — the task distribution of Fig 9 */
     int64_t *block_claims;
     int64_t cluster_steals;  /* steals through distributed shared memory (cluster tier)           */
+    int64_t pops;            /* 32-wide step: entries popped after a list was exhausted            */
+    int64_t dead_pops;       /* ... of which found nothing left to claim (every remaining target
+                                was claimed after the entry was pushed)                            */
 } dfs_stats;
 
 void dfs_options_default(dfs_options *opt);

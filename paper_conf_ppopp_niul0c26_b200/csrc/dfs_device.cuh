@@ -64,7 +64,8 @@ struct Ctl {
 enum CounterIdx {
     kCntClaims = 0, kCntFailedClaims, kCntFlushes, kCntRefills, kCntIntraSteals, kCntInterSteals,
     kCntStealAttempts, kCntChunks, kCntWindows, kCntIdleNs, kCntInterScans, kCntSpills,
-    kCntTWin, kCntTProbe, kCntTClaim, kCntTTail, kCntTOut, kCntOutIters, kCntClusterSteals, kNumCounters
+    kCntTWin, kCntTProbe, kCntTClaim, kCntTTail, kCntTOut, kCntOutIters, kCntClusterSteals,
+    kCntPops, kCntDeadPops, kNumCounters
 };
 
 struct KParams {
@@ -518,6 +519,8 @@ __global__ void __launch_bounds__(32 * WMAX, 1) dfs_persistent_kernel(const KPar
     unsigned long long t_idle0 = 0;
     uint32_t iter = 0;
     uint32_t my_claims = 0;                      // for P.block_claims (Fig 9 task distribution)
+    bool unproductive = false;                   // STATS: the top came from a pop and has not
+                                                 // claimed yet (dead-pop counter, 32-wide step)
     uint32_t tl_reported = 0;                    // timeline diagnostics
 
     if (blockIdx.x == 0 && w == 0) {
@@ -902,6 +905,7 @@ __global__ void __launch_bounds__(32 * WMAX, 1) dfs_persistent_kernel(const KPar
             // probe's "unvisited" cannot change before the claim: a fire-and-forget red.or sets
             // the bit (the step does not wait for it) and the parent is u in every order.
             if (__any_sync(kFull, lf)) {
+                if (STATS) unproductive = false;
                 red_or_if(lf, P.bitmap + 2u * ((uint32_t)nb >> 5), 1u << (nb & 31));
                 st_global_if(lf, P.parent + nb, (int32_t)u);                    // Alg 1 l.10
                 if (STATS || P.block_claims || P.timeline) {
@@ -938,6 +942,7 @@ __global__ void __launch_bounds__(32 * WMAX, 1) dfs_persistent_kernel(const KPar
             uint32_t next_i = i + 32u;                            // u's scan resumes here
             bool advance = !won;
             if (won) {
+                if (STATS) unproductive = false;
                 // descend (Alg 1 l.8-11): push <u, next candidate> unless u is exhausted —
                 // positions whose probe saw a claimed target stay claimed, so skipping them keeps
                 // Alg 1's order — then v becomes the register top with its first window loaded
@@ -974,7 +979,9 @@ __global__ void __launch_bounds__(32 * WMAX, 1) dfs_persistent_kernel(const KPar
                     spec_ok = false;
                 } else {
                     have_win = false;                             // i >= end: Alg 1 l.14: pop
+                    if (STATS && lane == 0) { ++cnt[kCntPops]; if (unproductive) ++cnt[kCntDeadPops]; }
                     has_top = pop(u, i);
+                    if (STATS) unproductive = true;
                     need_end = true;
                     spec_ok = spec_pop; par = kFull;
                 }

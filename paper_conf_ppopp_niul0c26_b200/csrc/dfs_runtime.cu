@@ -557,6 +557,8 @@ static void fill_stats(dfs_stats* stats, int blocks, int warps, float total_ms, 
     stats->cyc_tail = (int64_t)counters[kCntTTail];
     stats->cyc_outside = (int64_t)counters[kCntTOut];
     stats->cluster_steals = (int64_t)counters[kCntClusterSteals];
+    stats->pops = (int64_t)counters[kCntPops];
+    stats->dead_pops = (int64_t)counters[kCntDeadPops];
 }
 
 // per-root count buffer (2 x u64 per root) for stats calls

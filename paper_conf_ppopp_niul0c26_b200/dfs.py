@@ -68,7 +68,8 @@ class _Stats(ctypes.Structure):
                 ("cyc_window", ctypes.c_int64), ("cyc_probe", ctypes.c_int64),
                 ("cyc_claim", ctypes.c_int64), ("cyc_tail", ctypes.c_int64),
                 ("cyc_outside", ctypes.c_int64), ("root_counts", ctypes.c_void_p),
-                ("block_claims", ctypes.c_void_p), ("cluster_steals", ctypes.c_int64)]
+                ("block_claims", ctypes.c_void_p), ("cluster_steals", ctypes.c_int64),
+                ("pops", ctypes.c_int64), ("dead_pops", ctypes.c_int64)]
 
 
 @dataclass
@@ -141,6 +142,8 @@ class Stats:
     cyc_tail: int
     cyc_outside: int
     cluster_steals: int = 0
+    pops: int = 0
+    dead_pops: int = 0
     root_counts: Optional[np.ndarray] = None
     block_claims: Optional[np.ndarray] = None
 

@@ -214,6 +214,7 @@ def main():
                        n_visited=st.n_visited, util=round(util, 4), claims=st.claims,
                        failed=st.failed_claims, windows=st.windows, flushes=st.flushes,
                        refills=st.refills, intra=st.intra_steals, inter=st.inter_steals, cl=getattr(st, "cluster_steals", 0), blocks=st.blocks,
+                       pops=getattr(st, "pops", 0), dead_pops=getattr(st, "dead_pops", 0),
                        attempts=st.steal_attempts, scans=st.inter_scans, spills=st.spills, chunks=st.chunks_allocated,
                        us_per_claim_per_warp=round(st.traversal_ms * 1e3 * warps * util / max(1, st.claims), 3),
                        windows_per_claim=round(st.windows / max(1, st.claims), 3),
