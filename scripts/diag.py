@@ -135,6 +135,15 @@ VARIANTS = {
     "v1": dict(ring_cap=2),
     "l2p32": dict(l2_persist_mb=32),
     "l2off": dict(l2_persist_mb=-1),
+    "h2c1": dict(hot_cutoff=2, cold_cutoff=1),
+    "h1c4": dict(hot_cutoff=1, cold_cutoff=4),
+    "si64": dict(spill_idle=64),
+    "si256": dict(spill_idle=256),
+    "si8": dict(spill_idle=8),
+    "pb2": dict(pub_batch=2),
+    "bmin64": dict(backoff_min_ns=64),
+    "bmax1k": dict(backoff_max_ns=1024),
+    "bmax4k": dict(backoff_max_ns=4096),
     "l2p64": dict(l2_persist_mb=64),
     "l2p96": dict(l2_persist_mb=96),
     "w0nointra": dict(collect_stats=2, intra_steal=False),
