@@ -136,6 +136,9 @@ VARIANTS = {
     "l2p32": dict(l2_persist_mb=32),
     "l2off": dict(l2_persist_mb=-1),
     "h2c1": dict(hot_cutoff=2, cold_cutoff=1),
+    "w8": dict(warps_per_block=8),
+    "b32": dict(blocks=32),
+    "b74": dict(blocks=74),
     "h1c4": dict(hot_cutoff=1, cold_cutoff=4),
     "si64": dict(spill_idle=64),
     "si256": dict(spill_idle=256),
