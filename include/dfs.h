@@ -225,9 +225,10 @@ int dfs_graph_info(const dfs_graph *g, int64_t *n, int64_t *m, int32_t *device);
 int64_t dfs_launch_count(const dfs_graph *g);
 
 /* Diagnostics: busy-warp timeline.  dfs_debug_timeline(g, len, dt_ns, NULL) enables sampling
- * every dt_ns (block 0 / warp 0) into a device buffer of len entries for subsequent runs: entry
- * k < len/2 = busy warps + 1 (0 = no sample), entry len/2 + k = claims reported so far (busy warps
- * report every 32 windows); calling it again with the same len and a host buffer `out` copies the
+ * every dt_ns (block 0 / warp 0) into a device buffer of len entries for subsequent runs, in three
+ * regions of t = len/3 entries: entry k < t = busy blocks + 1 (0 = no sample), entry t + k = claims
+ * reported so far, entry 2t + k = expansion windows reported so far (collect_stats runs only; busy
+ * warps report every period); calling it again with the same len and a host buffer `out` copies the
  * last run's samples out and clears them; len = 0 disables. */
 int dfs_debug_timeline(dfs_graph *g, uint32_t len, uint32_t dt_ns, uint32_t *out);
 

@@ -59,6 +59,7 @@ struct Ctl {
     unsigned long long free_head;      // tagged free-stack head: (tag << 32) | chunk id
     unsigned long long counters[24];   // stats (collect_stats)
     unsigned long long claims_progress;// timeline diagnostics: claims reported so far
+    unsigned long long windows_progress;// ... and windows (STATS builds)
 };
 
 enum CounterIdx {
@@ -522,6 +523,7 @@ __global__ void __launch_bounds__(32 * WMAX, 1) dfs_persistent_kernel(const KPar
     bool unproductive = false;                   // STATS: the top came from a pop and has not
                                                  // claimed yet (dead-pop counter, 32-wide step)
     uint32_t tl_reported = 0;                    // timeline diagnostics
+    unsigned long long tl_win_reported = 0;
 
     if (blockIdx.x == 0 && w == 0) {
         // Alg 1 l.1-3: root claimed by the reset kernel; <root, row_ptr[root]> is our top
@@ -767,10 +769,14 @@ __global__ void __launch_bounds__(32 * WMAX, 1) dfs_persistent_kernel(const KPar
         if (P.timeline && blockIdx.x == 0 && w == 0 && lane == 0) {
             const unsigned long long now = globaltimer() - S.t_start;
             const unsigned int slot = (unsigned int)(now / P.timeline_dt_ns);
+            // timeline_len = 2 * (buffer length / 3): busy samples, claims, then (STATS) windows
             if (slot >= tl_next && slot < P.timeline_len / 2) {
                 P.timeline[slot] = *(volatile unsigned int*)&P.ctl->busy + 1u;   // 0 = no sample
                 P.timeline[P.timeline_len / 2 + slot] =
                     (unsigned int)*(volatile unsigned long long*)&P.ctl->claims_progress;
+                if (STATS)
+                    P.timeline[P.timeline_len + slot] =
+                        (unsigned int)*(volatile unsigned long long*)&P.ctl->windows_progress;
                 tl_next = slot + 1;
             }
         }
@@ -1195,6 +1201,10 @@ __global__ void __launch_bounds__(32 * WMAX, 1) dfs_persistent_kernel(const KPar
                 if (P.timeline && lane == 0) {                    // diagnostics: claim progress
                     atomicAdd(&P.ctl->claims_progress, (unsigned long long)(my_claims - tl_reported));
                     tl_reported = my_claims;
+                    if (STATS) {
+                        atomicAdd(&P.ctl->windows_progress, cnt[kCntWindows] - tl_win_reported);
+                        tl_win_reported = cnt[kCntWindows];
+                    }
                 }
                 sample();
                 if (P.spill) {
@@ -1512,6 +1522,7 @@ __global__ void dfs_reset_kernel(uint32_t* bitmap, uint32_t nwords, uint32_t bst
         ctl->pool_bump = 0u;
         ctl->free_head = (unsigned long long)kEmptySlot;
         ctl->claims_progress = 0ull;
+        ctl->windows_progress = 0ull;
         for (int k = 0; k < 24; ++k) ctl->counters[k] = 0ull;
     }
 }

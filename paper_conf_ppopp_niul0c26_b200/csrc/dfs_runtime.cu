@@ -397,7 +397,7 @@ static int launch_one(dfs_graph* g, Slot& sl, cudaStream_t s, int32_t root, int3
     P.period_mask = (uint32_t)(o.spill_period > 0 ? o.spill_period : 32) - 1u;
     const bool tl = g->d_timeline && &sl == &g->slots[0];
     P.timeline = tl ? g->d_timeline : nullptr;
-    P.timeline_len = tl ? g->timeline_len : 0;
+    P.timeline_len = tl ? (g->timeline_len / 3u) * 2u : 0;   // kernel: three regions of len/3
     P.timeline_dt_ns = tl ? g->timeline_dt_ns : 1;
     P.timeout_ns = (unsigned long long)o.timeout_ms * 1000000ull;
     P.seed = o.seed;

@@ -321,7 +321,8 @@ class Graph:
 
     def timeline(self, len_: int = 0, dt_ns: int = 10_000, fetch: bool = False):
         """Diagnostics (dfs_debug_timeline): enable with len_ > 0; fetch=True returns the last
-        run's (busy-warp samples (-1 = no sample), claims-so-far samples) as numpy arrays."""
+        run's (busy-block samples (-1 = no sample), claims-so-far, windows-so-far (collect_stats runs))
+        samples as numpy arrays."""
         if not fetch:
             rc = self._lib.dfs_debug_timeline(self._h, len_, dt_ns, None)
             if rc != 0:
@@ -331,8 +332,9 @@ class Graph:
         rc = self._lib.dfs_debug_timeline(self._h, len_, dt_ns, buf.ctypes.data)
         if rc != 0:
             raise DfsError(rc, "dfs_debug_timeline")
-        h = len_ // 2
-        return buf[:h].astype(np.int64) - 1, buf[h:].astype(np.int64)
+        t = len_ // 3
+        return (buf[:t].astype(np.int64) - 1, buf[t:2 * t].astype(np.int64),
+                buf[2 * t:3 * t].astype(np.int64))
 
     def launch_count(self) -> int:
         return int(self._lib.dfs_launch_count(self._h))

@@ -148,6 +148,7 @@ VARIANTS = {
     "bmax1k": dict(backoff_max_ns=1024),
     "bmax4k": dict(backoff_max_ns=4096),
     "l2p64": dict(l2_persist_mb=64),
+    "spec128": dict(speculate=1 | 4 | 8),
     "l2p96": dict(l2_persist_mb=96),
     "w0nointra": dict(collect_stats=2, intra_steal=False),
     "sp8": dict(spill_period=8),
@@ -234,12 +235,16 @@ def main():
                                        (st.cyc_window, st.cyc_probe, st.cyc_claim, st.cyc_tail, st.cyc_outside)])
             if a.timeline:
                 G.run(int(r), out=out, options=o)      # sampled run
-                tl, prog = G.timeline(TL, a.timeline * 1000, fetch=True)
+                tl, prog, wprog = G.timeline(TL, a.timeline * 1000, fetch=True)
                 k = int(np.nonzero(tl >= 0)[0].max()) + 1 if np.any(tl >= 0) else 0
                 tl = tl[:k]
                 prog = prog[:k]
+                wprog = wprog[:k]
                 if k >= 20:
                     rec["claims_by_5pct"] = [int(c[c > 0].max()) if np.any(c > 0) else 0 for c in np.array_split(prog, 20)]
+                    if np.any(wprog > 0):      # collect_stats runs: windows scanned so far
+                        rec["windows_by_5pct"] = [int(c[c > 0].max()) if np.any(c > 0) else 0
+                                                  for c in np.array_split(wprog, 20)]
                 valid = tl[tl >= 0]
                 dec = [int(np.mean(c[c >= 0])) if np.any(c >= 0) else -1 for c in np.array_split(tl, 20)] if k >= 20 else []
                 rec["timeline_us"] = a.timeline
