@@ -1116,9 +1116,9 @@ __global__ void __launch_bounds__(32 * WMAX, 1) dfs_persistent_kernel(const KPar
                     bool leaf = vre == vrs;
                     if (P.leaf_skip && vre == vrs + 1u) {
                         int first = cnb[0];
-                        if constexpr (VEC > 1) {
-#pragma unroll
-                            for (int f = 1; f < VEC; ++f) if ((int)(vrs & (VEC - 1)) == f) first = cnb[f];
+                        if constexpr (VEC == 4) {                // selects, not a local-memory index
+                            const uint32_t sel = vrs & 3u;
+                            first = sel == 0u ? cnb[0] : (sel == 1u ? cnb[1] : (sel == 2u ? cnb[2] : cnb[3]));
                         }
                         leaf = (uint32_t)__shfl_sync(kFull, first, 0) == u;
                     }
