@@ -1061,23 +1061,28 @@ __global__ void __launch_bounds__(32 * WMAX, 1) dfs_persistent_kernel(const KPar
                     sv = (uint32_t)__shfl_sync(kFull, pick, sk);
                 }
             }
-            uint32_t s_old = atom_or_if(vb != 0 && lane == 0, P.bitmap + 2u * (sv >> 5), 1u << (sv & 31));
-            const uint32_t s_rs = ld_nc_if(vb != 0, P.rp + sv, 0u), s_re = ld_nc_if(vb != 0, P.rp + sv + 1, 0u);
             // probe the visited bits; the lanes holding the first 8 positions also prefetch
-            // their candidates' row_ptr pairs
+            // their candidates' row_ptr pairs.  All loads are issued before the speculative
+            // claim: its result may be spilled, and a spill store waits for the atomic
             uint32_t cm = 0;                                      // unvisited candidates
             uint32_t lcm = 0;                                     // ... that are leaves
             uint32_t prs[VEC], pre[VEC];
+            uint2 wl[VEC];
 #pragma unroll
             for (int e = 0; e < VEC; ++e) {
                 const bool ok = (vm >> e) & 1u;
                 const uint32_t x = (uint32_t)nbv[e];
-                const uint2 wl = ld_cg_u2_if(ok, P.bitmap + 2u * (x >> 5), kFull, 0u);   // {visited, leaf}
-                const uint32_t word = wl.x, lword = wl.y;
+                wl[e] = ld_cg_u2_if(ok, P.bitmap + 2u * (x >> 5), kFull, 0u);   // {visited, leaf}
                 const bool pf = ok && lane < kPfLanes;
                 prs[e] = ld_nc_if(pf, P.rp + x, 0u); pre[e] = ld_nc_if(pf, P.rp + x + 1, 0u);
-                if (ok && !((word >> (x & 31)) & 1u)) {
-                    if ((lword >> (x & 31)) & 1u) lcm |= 1u << e; else cm |= 1u << e;
+            }
+            const uint32_t s_rs = ld_nc_if(vb != 0, P.rp + sv, 0u), s_re = ld_nc_if(vb != 0, P.rp + sv + 1, 0u);
+            uint32_t s_old = atom_or_if(vb != 0 && lane == 0, P.bitmap + 2u * (sv >> 5), 1u << (sv & 31));
+#pragma unroll
+            for (int e = 0; e < VEC; ++e) {
+                const uint32_t x = (uint32_t)nbv[e];
+                if (((vm >> e) & 1u) && !((wl[e].x >> (x & 31)) & 1u)) {
+                    if ((wl[e].y >> (x & 31)) & 1u) lcm |= 1u << e; else cm |= 1u << e;
                 }
             }
             if (lane == sk) { cm &= ~(1u << se); lcm &= ~(1u << se); }   // claimed either way
