@@ -451,7 +451,12 @@ __global__ void __launch_bounds__(32 * WMAX, 1) dfs_persistent_kernel(const KPar
     constexpr uint32_t kBatch = H / 2;              // flush batch (reading S10)
     constexpr uint32_t kWin = 32u * VEC;            // positions per window
     constexpr int kHeadLanes = VEC == 1 ? 8 : 16;   // lanes fetched before a window's end is known
-    constexpr int kPfLanes = 8 / VEC;               // lanes covering the first 8 positions
+#ifndef DFS_PF_LANES128
+#define DFS_PF_LANES128 2
+#endif
+    // lanes whose candidates' row_ptr pairs are loaded with the probes: the first 8 positions
+    // (128-wide: DFS_PF_LANES128 lanes of 4 positions; A/B builds only)
+    constexpr int kPfLanes = VEC == 1 ? 8 : DFS_PF_LANES128;
     extern __shared__ __align__(16) unsigned char smem_raw[];
     SmemCtl& S = *reinterpret_cast<SmemCtl*>(smem_raw);
     constexpr int kCtlBytes = (sizeof(SmemCtl) + 15) & ~15;
