@@ -6,14 +6,22 @@ One step = one full unordered DFS (reset + persistent traversal + finalize, SURV
 over the resident graph, from the step's root.  Roots follow the paper's methodology (64 sources,
 average TEPS, P:1523-1526): the config's headline root followed by 63 seeded roots with degree > 0;
 step s of rank r uses root (r + s*N) mod 64.  With N > 1 every rank holds a replica of the graph
-and runs its own roots (weak scaling, no data-path collective); the single exchange step is an
-NCCL all_gather of the per-root summaries at the end.
+and runs its own roots (weak scaling, no data-path collective).
 
-value  = whole-job GTEPS = sum over ranks and steps of m_r (out-degree sum of the visited set,
-         reading S6) / max over ranks of the sum of per-step device times (CUDA events).
-e2e    = same metric through the public C ABI with HOST buffers: dfs_graph_create (host CSR ->
-         device) + dfs_run (host parent_out) + dfs_graph_destroy per step.
+The JSON line (rank 0) carries, besides the contract keys:
+  roofline      dominant kernel (persistent traversal): algorithmic bytes per launch
+                over its CUDA-event time, against MEASURED_PEAKS.json hbm_gbs; `step` adds
+                SURVEY §8(d)'s B_min (with the 4n reset term) over the whole step
+  cpu_baseline  the oracle (Alg 1) pinned to one host core, median over whole traversals
+  e2e           the public C ABI with host buffers (dfs_run into pinned host memory)
+  batch1024     C5 (configs[4]): 1,024 seeded roots on the road graph partitioned contiguously
+                across the N ranks (strong scaling), DFS/s without and with the NCCL gather of
+                the parent arrays to rank 0, roofline, all-core oracle baseline, I1-I6 checks
+  rmat24        C3 (configs[2], N = 1): GTEPS, ms, roofline of the 128-wide kernel
 --impl reference = the CPU oracle (Alg 1, oracle/) timed on the host cores, same workload.
+
+`python bench.py --gpus N` without torchrun re-launches itself under torch.distributed.run
+with N ranks (one per GPU, NCCL).
 
 Usage: python bench.py [--gpus N] [--steps K] [--warmup W] [--config road24m] [--impl b200|reference]
 """
@@ -22,7 +30,7 @@ from __future__ import annotations
 import argparse
 import json
 import os
-import platform
+import socket
 import subprocess
 import sys
 import threading
@@ -41,7 +49,7 @@ def log(*a):
     print(*a, file=sys.stderr, flush=True)
 
 
-def parse():
+def parse(argv=None):
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
     ap.add_argument("--steps", type=int, default=10)
@@ -50,20 +58,44 @@ def parse():
                     choices=["road24m", "grid256", "rmat24", "path100m", "caterpillar", "batch1024"])
     ap.add_argument("--batch-roots", type=int, default=1024)
     ap.add_argument("--concurrency", type=int, default=0,
-                    help="batch1024: traversals in flight per GPU (0 = auto)")
+                    help="batch: traversals in flight per GPU (0 = library auto)")
     ap.add_argument("--impl", default="b200", choices=["b200", "reference"])
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-validate", action="store_true")
+    ap.add_argument("--no-batch", action="store_true", help="skip the batch1024 sub-record")
+    ap.add_argument("--no-rmat", action="store_true", help="skip the rmat24 sub-record")
+    ap.add_argument("--no-gather", action="store_true", help="batch: skip the with-gather pass")
     ap.add_argument("--cpu-seconds", type=float, default=12.0)
     ap.add_argument("--nroots", type=int, default=64)
-    return ap.parse_args()
+    ap.add_argument("--set", action="append", default=[], metavar="KEY=VALUE",
+                    help="dfs_options field for the timed runs (A/B experiments)")
+    return ap.parse_args(argv)
 
 
 def roots_for(g, root0, k):
     import graphgen
     rs = [int(root0)] + [int(x) for x in graphgen.random_roots(g, k - 1, seed=0x6A7)]
     return rs[:k]
+
+
+def cpu_model():
+    try:
+        with open("/proc/cpuinfo") as f:
+            for ln in f:
+                if ln.startswith("model name"):
+                    return ln.split(":", 1)[1].strip()
+    except OSError:
+        pass
+    import platform
+    return platform.processor() or "cpu"
+
+
+def host_cores():
+    try:
+        return len(os.sched_getaffinity(0))
+    except AttributeError:  # pragma: no cover
+        return os.cpu_count() or 1
 
 
 # ------------------------------------------------------------------------------ clocks
@@ -88,6 +120,7 @@ class ClockSampler:
         except Exception as e:  # pragma: no cover
             log("clock sampler unavailable:", e)
             self.proc = None
+        return self
 
     def _read(self):
         for line in self.proc.stdout:
@@ -124,105 +157,214 @@ def measured_peaks():
     if os.path.exists(p):
         with open(p) as f:
             d = json.load(f)
-        return float(d["hbm_gbs"]), "measured"
+        return float(d["hbm_gbs"]), "measured (MEASURED_PEAKS.json hbm_gbs)"
     return 6650.0, "fallback (B200_PROFILING.md)"
 
 
 def traffic_from_profile(workload):
+    """ncu dram__bytes_read.sum + dram__bytes_write.sum of one traversal-kernel launch
+    (profiles/ncu_traffic.json, written from the committed `ncu --set full` captures)."""
     p = os.path.join(ROOT, "profiles", "ncu_traffic.json")
     if os.path.exists(p):
         with open(p) as f:
             d = json.load(f)
-        return d.get(workload)
+        v = d.get(workload)
+        return v.get("bytes") if isinstance(v, dict) else v
     return None
 
 
+def parse_sets(sets):
+    opts = {}
+    for kv in sets:
+        k, _, v = kv.partition("=")
+        opts[k] = int(v)
+    return opts
+
+
 # ------------------------------------------------------------------------------ oracle (CPU)
-def cpu_oracle(g, roots, seconds, steps=None):
-    """Time oracle.dfs (Alg 1, one host core) over whole traversals; bounded by `seconds`."""
+def cpu_oracle_pinned(g, roots, seconds, steps=None):
+    """oracle.dfs (Alg 1) on ONE host core (sched_setaffinity), whole traversals, bounded by
+    `seconds` (or exactly `steps` traversals); returns (GTEPS of the median traversal, median ms,
+    count, core)."""
     import oracle
-    tot_t, tot_e, done = 0.0, 0, 0
-    for q in range(10**9):
-        r = roots[q % len(roots)]
-        t0 = time.perf_counter()
-        p = oracle.dfs(g.row_ptr, g.col_idx, r)
-        dt = time.perf_counter() - t0
-        vis = p != -2
-        tot_t += dt
-        tot_e += int(np.diff(g.row_ptr)[vis].sum())
-        done += 1
-        if (steps is not None and done >= steps) or (steps is None and tot_t >= seconds):
-            break
-    return tot_e / tot_t / 1e9, tot_t / done * 1e3, done
+    deg = np.diff(g.row_ptr)
+    old = os.sched_getaffinity(0)
+    core = min(old)
+    os.sched_setaffinity(0, {core})
+    ms, gteps = [], []
+    try:
+        t_all = 0.0
+        for q in range(10**9):
+            r = roots[q % len(roots)]
+            t0 = time.perf_counter()
+            p = oracle.dfs(g.row_ptr, g.col_idx, r)
+            dt = time.perf_counter() - t0
+            t_all += dt
+            ms.append(dt * 1e3)
+            gteps.append(int(deg[p != -2].sum()) / dt / 1e9)
+            if (steps is not None and len(ms) >= steps) or (steps is None and t_all >= seconds):
+                break
+    finally:
+        os.sched_setaffinity(0, old)
+    return float(np.median(gteps)), float(np.median(ms)), len(ms), core
 
 
-# ------------------------------------------------------------------------------ main
+def cpu_oracle_pool(g, roots, seconds):
+    """C5 CPU baseline: a pool of threads over ALL host cores, one root per task (oracle.dfs
+    releases the GIL in C); bounded by `seconds`.  Returns (DFS/s, completed, threads)."""
+    import oracle
+    nthreads = host_cores()
+    lock = threading.Lock()
+    state = {"next": 0, "done": 0}
+    t0 = time.perf_counter()
+
+    def worker():
+        while True:
+            with lock:
+                if time.perf_counter() - t0 >= seconds:
+                    return
+                q = state["next"]
+                state["next"] += 1
+            oracle.dfs(g.row_ptr, g.col_idx, int(roots[q % len(roots)]))
+            with lock:
+                state["done"] += 1
+
+    th = [threading.Thread(target=worker) for _ in range(nthreads)]
+    for t in th:
+        t.start()
+    for t in th:
+        t.join()
+    el = time.perf_counter() - t0
+    return state["done"] / el, state["done"], nthreads, el
+
+
+# ------------------------------------------------------------------------------ launch
+def free_port():
+    s = socket.socket()
+    s.bind(("127.0.0.1", 0))
+    p = s.getsockname()[1]
+    s.close()
+    return p
+
+
+def relaunch(a):
+    """`--gpus N` without torchrun: re-execute this script under torch.distributed.run, one rank
+    per GPU (the driver's own N > 1 launch goes straight to main())."""
+    cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", f"--nproc-per-node={a.gpus}",
+           "--master-addr", "127.0.0.1", "--master-port", str(free_port()),
+           os.path.abspath(__file__), *sys.argv[1:]]
+    log("relaunch:", " ".join(cmd))
+    return subprocess.call(cmd)
+
+
 def main():
     a = parse()
+    if "WORLD_SIZE" not in os.environ and a.gpus > 1:
+        sys.exit(relaunch(a))
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
     local = int(os.environ.get("LOCAL_RANK", "0"))
-    import graphgen
-
     if a.impl == "reference":
         return reference_arm(a, world, rank)
-    if a.config == "batch1024":
-        return batch_arm(a, world, rank, local)
 
     import torch
     import torch.distributed as dist
-    from paper_conf_ppopp_niul0c26_b200 import Graph, Options
-    from paper_conf_ppopp_niul0c26_b200 import dfs as dfsmod
-
     torch.cuda.set_device(local)
     if world > 1:
         dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    dev = torch.device("cuda", local)
+    import graphgen
+
+    if a.config == "batch1024":
+        g = graphgen.road(4900, 4900)
+        rec = {"metric": METRIC, "n_gpus": world}
+        b = batch_leg(a, g, world, rank, local, dev)
+        if rank == 0:
+            rec.update({"value": b["dfs_per_s"], "unit": "DFS/s", "steps": b["roots"], "warmup": a.warmup,
+                        "ms_per_step": b["ms_per_dfs"], "higher_is_better": True, "scaling": "strong",
+                        "vs_baseline": None, "dtype": "int32", "data": "synthetic",
+                        "config": {"workload": "batch1024", "n": g.n, "m": g.m},
+                        "batch1024": b})
+            print(json.dumps(rec), flush=True)
+        if world > 1:
+            dist.destroy_process_group()
+        return
 
     t0 = time.time()
     g, root0, undirected, desc = graphgen.config_graph(a.config)
     log(f"[rank {rank}] graph {a.config}: n={g.n} m={g.m} built in {time.time() - t0:.1f}s")
+    rec = single_root_leg(a, a.config, g, root0, undirected, desc, world, rank, local, headline=True)
+
+    if not a.no_batch and a.config in ("road24m",):
+        b = batch_leg(a, g, world, rank, local, dev)
+        if rank == 0:
+            rec["batch1024"] = b
+    if rank == 0 and world == 1 and not a.no_rmat and a.config != "rmat24":
+        del g
+        t0 = time.time()
+        gr, rr, und, desc_r = graphgen.config_graph("rmat24")
+        log(f"[rank {rank}] graph rmat24: n={gr.n} m={gr.m} built in {time.time() - t0:.1f}s")
+        sub = single_root_leg(a, "rmat24", gr, rr, und, desc_r, 1, 0, local, headline=False)
+        rec["rmat24"] = sub
+    if rank == 0:
+        print(json.dumps(rec), flush=True)
+    if world > 1:
+        dist.destroy_process_group()
+
+
+# ------------------------------------------------------------------------------ single root
+def single_root_leg(a, workload, g, root0, undirected, desc, world, rank, local, headline):
+    """Single-root traversals on one GPU per rank (weak-scaled replicas for N > 1).  Returns the
+    full JSON record (headline) or the sub-record (rmat24) on rank 0."""
+    import torch
+    import torch.distributed as dist
+
+    import oracle
+    from paper_conf_ppopp_niul0c26_b200 import Graph, Options
+    from paper_conf_ppopp_niul0c26_b200 import dfs as dfsmod
+
     roots = roots_for(g, root0, a.nroots)
     deg = np.diff(g.row_ptr)
-
     G = Graph(g.row_ptr, g.col_idx)
     out = torch.empty(g.n, dtype=torch.int32, device="cuda")
     stream = torch.cuda.current_stream()
     ws_bytes = (g.n + 1) * 4 + g.m * 4 + g.n * 4
     flush_l2 = ws_bytes < 2 * L2_BYTES
     scratch = torch.empty(2 * L2_BYTES // 4, dtype=torch.int32, device="cuda") if flush_l2 else None
+    opts = parse_sets(a.set)
+    timed_opts = Options(**opts)
 
-    my_roots = [roots[(rank + s * world) % len(roots)] for s in range(a.steps)]
-    # m_r per root is fixed (the reach set is unique): computed once, outside timing, from a
-    # validated run; the first run of each root is also checked against the oracle (I1-I6)
-    m_r, valid = {}, {}
-    import oracle
+    steps = a.steps if headline else max(5, min(a.steps, 10))
+    my_roots = [roots[(rank + s * world) % len(roots)] for s in range(steps)]
+    # m_r / n_r per root are fixed (the reach set is unique): computed once, outside timing, from
+    # a validated run; the first runs are also checked against the oracle (I1-I6 exact)
+    m_r, n_r, valid = {}, {}, {}
     for q, r in enumerate(sorted(set(my_roots))):
-        p = G.run(r, out=out)
+        p = G.run(r, out=out, options=timed_opts)
         vis = (p != -2).cpu().numpy()
         m_r[r] = int(deg[vis].sum())
+        n_r[r] = int(vis.sum())
         if not a.no_validate and q < 2:
             res = oracle.check_tree(g.row_ptr, g.col_idx, r, p.cpu().numpy(), i7=True, undirected=undirected)
             valid[r] = {k: getattr(res, k) for k in ("i1", "i2", "i3", "i4", "i5", "i6", "i7")}
             valid[r]["n_cross_I7"] = res.n_cross
             assert res.ok or res.failed() == ["i7"], (r, res)
-    for s in range(a.warmup):
-        G.run(my_roots[s % len(my_roots)], out=out)
+    for s in range(max(3, a.warmup)):
+        G.run(my_roots[s % len(my_roots)], out=out, options=timed_opts)
     torch.cuda.synchronize()
 
-    ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(a.steps)]
-    opt_stats = Options()
+    ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(steps)]
     trav_ms = []
-    clocks = ClockSampler(local)
-    clocks.start()
+    clocks = ClockSampler(local).start()
     launches0 = G.launch_count()
     if world > 1:
         dist.barrier()
     torch.cuda.synchronize()
-    for s in range(a.steps):
+    for s in range(steps):
         if flush_l2:
             scratch.fill_(s)
         ev[s][0].record(stream)
-        _, st = G.run(my_roots[s], out=out, options=opt_stats, stats=True)
+        _, st = G.run(my_roots[s], out=out, options=timed_opts, stats=True)
         ev[s][1].record(stream)
         trav_ms.append(st.traversal_ms)
     torch.cuda.synchronize()
@@ -233,139 +375,171 @@ def main():
     step_ms = [e0.elapsed_time(e1) for e0, e1 in ev]
     my_time = sum(step_ms) / 1e3
     my_edges = sum(m_r[r] for r in my_roots)
+    # roofline of the dominant kernel (persistent traversal, launched on `stream`; its duration
+    # is the library's CUDA-event pair around the launch, dfs_stats.traversal_ms): algorithmic
+    # bytes per launch = 12 B per reached vertex (uint32 row_ptr pair + parent write) + 8 B per
+    # scanned edge (col_idx entry + one visited probe); the step-level figure adds
+    # SURVEY §8(d)'s 4n reset term over the whole step time
+    kbytes = sum(12.0 * n_r[r] + 8.0 * m_r[r] for r in my_roots)
+    sbytes = kbytes + 4.0 * g.n * steps
+    my_trav = sum(trav_ms) / 1e3
 
-    # exchange step: per-root summaries gathered over NCCL (roots, m_r, ms)
-    summ = torch.tensor([[float(r), float(m_r[r]), float(t)] for r, t in zip(my_roots, step_ms)],
-                        dtype=torch.float64, device="cuda")
-    if world > 1:
-        allsum = torch.empty((world * a.steps, 3), dtype=torch.float64, device="cuda")
-        dist.all_gather_into_tensor(allsum, summ)
-        tmax = torch.tensor([my_time], dtype=torch.float64, device="cuda")
-        dist.all_reduce(tmax, op=dist.ReduceOp.MAX)
-        t_job = float(tmax.item())
-        edges = float(allsum[:, 1].sum().item())
-    else:
-        t_job = my_time
-        edges = float(my_edges)
+    from paper_conf_ppopp_niul0c26_b200 import batch
+    (t_job, _), (edges,) = batch.reduce_max_sum([my_time, my_trav], [float(my_edges)], world,
+                                                device=torch.device("cuda", local))
     if rank != 0:
-        if world > 1:
-            dist.destroy_process_group()
-        return
+        G.close()
+        return None
 
-    gteps = edges / t_job / 1e9
-    ms_per_dfs = t_job * 1e3 / a.steps
-    # roofline of the dominant kernel (persistent traversal): algorithmic bytes per launch =
-    # 12 B per reached vertex (uint32 row_ptr pair + parent write) + 8 B per scanned edge
-    # (col_idx + one visited probe)  (DESIGN.md §"Roofline")
-    byte_sum, trav_sum = 0.0, 0.0
     peak, peak_src = measured_peaks()
-    # n_r per root (visited count)
-    n_r = {}
-    for r in set(my_roots):
-        p = G.run(r, out=out)
-        n_r[r] = int((p != -2).sum().item())
-    for r, tm in zip(my_roots, trav_ms):
-        byte_sum += 12.0 * n_r[r] + 8.0 * m_r[r]
-        trav_sum += tm / 1e3
-    achieved = byte_sum / trav_sum / 1e9
+    achieved = kbytes / my_trav / 1e9            # rank 0's own launches (per-GPU kernel figure)
     roof = {"bound": "hbm", "achieved": round(achieved, 3), "peak": peak, "unit": "GB/s",
-            "frac": round(achieved / peak, 6), "traffic": traffic_from_profile(a.config),
-            "kernel": "b200dfs::dfs_persistent_kernel<256>", "peak_source": peak_src,
-            "kernel_share_of_step": round(trav_sum / t_job, 4),
-            "bytes_per_launch_avg": round(byte_sum / len(my_roots), 1)}
-
+            "frac": round(achieved / peak, 6), "traffic": traffic_from_profile(workload),
+            "kernel": "b200dfs::dfs_persistent_kernel", "peak_source": peak_src,
+            "bytes_per_launch_avg": round(kbytes / steps, 1),
+            "launch_ms_avg": round(my_trav * 1e3 / steps, 4),
+            "kernel_share_of_step": round(my_trav / my_time, 4),
+            "step": {"bytes_B_min_avg": round(sbytes / steps, 1),
+                     "achieved": round(sbytes / my_time / 1e9, 3),
+                     "frac": round(sbytes / my_time / 1e9 / peak, 6),
+                     "what": "SURVEY 8(d) B_min = 4n + 12 n_r + 8 m_r over the whole step (reset + traversal + finalize)"}}
+    gteps = edges / t_job / 1e9
+    ms_per_dfs = t_job * 1e3 / steps
     rec = {"metric": METRIC, "value": round(gteps, 6), "unit": "GTEPS", "n_gpus": world,
-           "steps": a.steps, "warmup": a.warmup, "ms_per_step": round(ms_per_dfs, 4),
+           "steps": steps, "warmup": a.warmup, "ms_per_step": round(ms_per_dfs, 4),
            "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "int32",
            "data": "synthetic",
-           "config": {"workload": a.config, "desc": desc, "n": g.n, "m": g.m, "roots": len(set(my_roots)),
+           "config": {"workload": workload, "desc": desc, "n": g.n, "m": g.m, "roots": len(set(my_roots)),
                       "root_policy": "headline root + 63 seeded degree>0 roots, round robin (P:1523-1526)",
                       "l2": ("flushed between steps (2x L2 write)" if flush_l2 else
                              f"inputs larger than L2 ({ws_bytes / 1e6:.0f} MB CSR+parent)"),
                       "parallelism": f"replicas x{world}" if world > 1 else "single GPU",
-                      "blocks": st.blocks, "warps_per_block": st.warps_per_block},
-           "ms_per_dfs": round(ms_per_dfs, 4), "dfs_per_s": round(a.steps * world / t_job, 3),
+                      "blocks": st.blocks, "warps_per_block": st.warps_per_block,
+                      "options": opts or "library defaults"},
+           "ms_per_dfs": round(ms_per_dfs, 4), "dfs_per_s": round(steps * world / t_job, 3),
            "ms_per_dfs_median": round(float(np.median(step_ms)), 4),
            "gpu_launches": int(launches), "clocks": clk, "roofline": roof, "validation": valid}
-
-    if not a.no_cpu_baseline and world == 1:
-        v, ms, cnt = cpu_oracle(g, roots, a.cpu_seconds)
+    if headline and not a.no_cpu_baseline and world == 1:
+        v, ms, cnt, core = cpu_oracle_pinned(g, roots, a.cpu_seconds)
         rec["cpu_baseline"] = {"value": round(v, 6), "unit": "GTEPS", "cores": 1, "kind": "oracle",
-                               "sample": f"{cnt} full Alg-1 traversals of {a.config} (round-robin roots), "
-                                         f"{ms:.1f} ms each, 1 host thread ({platform.processor() or 'cpu'}, "
-                                         f"{os.cpu_count()} host cores)"}
-    if not a.no_e2e:
+                               "sample": f"{cnt} whole Alg-1 traversals of {workload} (round-robin roots), "
+                                         f"median {ms:.1f} ms; pinned to host core {core} "
+                                         f"(sched_setaffinity) of {host_cores()}; {cpu_model()}",
+                               "statistic": "median GTEPS over traversals"}
+    if headline and not a.no_e2e:
         rec["e2e"] = e2e_leg(a, g, my_roots, m_r, dfsmod, G)
-    print(json.dumps(rec), flush=True)
     G.close()
-    if world > 1:
-        dist.destroy_process_group()
+    return rec
 
 
-def batch_arm(a, world, rank, local):
-    """C5 (BASELINE.json configs[4]): 1,024 seeded roots on the replicated road graph, partitioned
-    contiguously across ranks (strong scaling); one NCCL all_gather of per-root summaries."""
+# ------------------------------------------------------------------------------ C5 batch
+def batch_leg(a, g, world, rank, local, dev):
+    """C5 (BASELINE.json configs[4]): `--batch-roots` seeded roots on the replicated road graph,
+    partitioned contiguously across ranks (strong scaling).  Pass 1: traversals only
+    (dfs_run_batch_ex, chunks of device-resident parent rows, K traversals in flight per GPU).
+    Pass 2: the same with every chunk's parent rows gathered to rank 0 over NCCL (bounded
+    sub-chunks into a reused rank-0 device buffer: the result sink).  Times are device events,
+    max over ranks.  After timing, 4 rows of the last chunk per rank are checked against the
+    oracle (I1-I6 exact); the all-core CPU baseline runs on rank 0 at N = 1."""
     import torch
     import torch.distributed as dist
 
     import graphgen
-    from paper_conf_ppopp_niul0c26_b200 import Graph
+    import oracle
+    from paper_conf_ppopp_niul0c26_b200 import Graph, Options
     from paper_conf_ppopp_niul0c26_b200 import batch
 
-    torch.cuda.set_device(local)
-    if world > 1:
-        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
-    dev = torch.device("cuda", local)
-    t0 = time.time()
-    g = graphgen.road(4900, 4900)
     roots = graphgen.random_roots(g, a.batch_roots, seed=0xC5)
-    log(f"[rank {rank}] batch graph n={g.n} m={g.m} built in {time.time() - t0:.1f}s; {len(roots)} roots")
+    k = len(roots)
+    lo, hi = batch.partition(k, world, rank)
+    mine = [int(r) for r in roots[lo:hi]]
     G = Graph(g.row_ptr, g.col_idx)
-    lo, hi = batch.partition(len(roots), world, rank)
-    conc = a.concurrency if a.concurrency > 0 else 8          # library auto (DESIGN §8 sweep)
-    # chunks of 4 waves of `conc` traversals (device-resident parent rows, 96 MB each)
-    out_rows = torch.empty((max(1, min(4 * conc, hi - lo)), g.n), dtype=torch.int32, device=dev)
-    for s_ in range(a.warmup):                       # warm-up traversals (untimed)
-        G.run(int(roots[(lo + s_) % len(roots)]), out=out_rows[0])
-    launches0 = G.launch_count()
-    clocks = ClockSampler(local)
-    clocks.start()
-    if world > 1:
-        dist.barrier()
+    opts = parse_sets(a.set)
+    if a.concurrency > 0:
+        opts["concurrency"] = a.concurrency
+    o = Options(**opts)
+    cap = max(b - a_ for a_, b in (batch.partition(k, world, p) for p in range(world)))
+    rows = max(1, min(128, cap))                              # same on every rank
+    out_rows = torch.empty((rows, g.n), dtype=torch.int32, device=dev)
+    G.run_batch(mine[:min(rows, 8)], out=out_rows[:min(rows, 8)], options=o)      # warm-up
     torch.cuda.synchronize()
-    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-    e0.record()
-    res = batch.run_batch_chunked(G, out_rows, roots, world=world, rank=rank, device=dev, concurrency=conc)
-    e1.record()
-    torch.cuda.synchronize()
-    if world > 1:
-        dist.barrier()
+    sub = 8                                                   # rows per gather round
+    sink = None
+    if world > 1 and rank == 0 and not a.no_gather:
+        sink = [torch.empty((sub, g.n), dtype=torch.int32, device=dev) for _ in range(world)]
+
+    def one_pass(gather):
+        counts = []
+        launches0 = G.launch_count()
+        if world > 1:
+            dist.barrier()
+        torch.cuda.synchronize()
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record()
+        for c0 in range(0, cap, rows):
+            chunk = mine[c0:c0 + rows]
+            if chunk:
+                _, st = G.run_batch(chunk, out=out_rows[:len(chunk)], options=o, stats=True)
+                counts.append(st.root_counts.copy())
+            if gather and world > 1:
+                batch.gather_chunk_to_rank0(out_rows, len(chunk), min(rows, cap - c0), sub, sink, world, rank)
+        e1.record()
+        torch.cuda.synchronize()
+        ms = e0.elapsed_time(e1)
+        launches = G.launch_count() - launches0
+        (t_max,), _ = batch.reduce_max_sum([ms], [], world, device=dev)
+        return t_max, ms, np.concatenate(counts) if counts else np.zeros((0, 2)), launches
+
+    clocks = ClockSampler(local).start()
+    t_trav, my_ms, counts, launches = one_pass(False)
+    t_gath = None
+    if not a.no_gather and world > 1:
+        t_gath, _, _, _ = one_pass(True)
     clk = clocks.stop()
-    region_ms = e0.elapsed_time(e1)
-    if world > 1:
-        t = torch.tensor([region_ms], dtype=torch.float64, device=dev)
-        dist.all_reduce(t, op=dist.ReduceOp.MAX)
-        region_ms = float(t.item())
-    launches = G.launch_count() - launches0
-    if rank == 0:
-        k = len(roots)
-        rec = {"metric": METRIC, "value": round(res.gteps(), 6), "unit": "GTEPS", "n_gpus": world,
-               "steps": k, "warmup": a.warmup, "ms_per_step": round(res.max_ms / max(1, hi - lo), 4),
-               "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "int32",
-               "data": "synthetic",
-               "config": {"workload": "batch1024", "desc": "C5: road-maze 4900x4900, 1024 seeded roots "
-                          "partitioned contiguously across ranks, NCCL all_gather of per-root summaries",
-                          "n": g.n, "m": g.m, "roots": k, "parallelism": f"replicas x{world}",
-                          "l2": f"inputs larger than L2 ({((g.n + 1) * 4 + g.m * 8 + g.n * 4) / 1e6:.0f} MB)"},
-               "dfs_per_s": round(res.dfs_per_s(), 3),
-               "dfs_per_s_region": round(k / (region_ms * 1e-3), 3),
-               "region_ms": round(region_ms, 3), "gpu_launches": int(launches), "clocks": clk,
-               "exchange": "all_gather_into_tensor of (k x 5) float64 summaries",
-               "concurrency": conc}
-        print(json.dumps(rec), flush=True)
+    # algorithmic bytes of this rank's traversals (SURVEY 8(d) B_min per traversal)
+    my_bytes = float(sum(4.0 * g.n + 12.0 * nv + 8.0 * mv for nv, mv in counts))
+    my_edges = float(counts[:, 1].sum()) if len(counts) else 0.0
+    # validation of rows produced by the timed run (the last chunk), outside timing
+    vals = []
+    if not a.no_validate and mine:
+        last0 = ((len(mine) - 1) // rows) * rows
+        for q in range(min(4, len(mine) - last0)):
+            r = mine[last0 + q]
+            res = oracle.check_tree(g.row_ptr, g.col_idx, r, out_rows[q].cpu().numpy(), i7=False, undirected=True)
+            assert res.ok, (r, res)
+            vals.append(int(res.ok))
+    _, (tot_bytes, tot_edges, nval, nok) = batch.reduce_max_sum(
+        [], [my_bytes, my_edges, float(len(vals)), float(sum(vals))], world, device=dev)
     G.close()
-    if world > 1:
-        dist.destroy_process_group()
+    if rank != 0:
+        return None
+    peak, peak_src = measured_peaks()
+    conc = opts.get("concurrency", 0) or "auto (8)"
+    b = {"roots": k, "dfs_per_s": round(k / (t_trav * 1e-3), 3), "ms_per_dfs": round(t_trav / k, 4),
+         "region_ms": round(t_trav, 3), "gteps": round(tot_edges / (t_trav * 1e-3) / 1e9, 4),
+         "partition": f"contiguous slices of {k} seeded roots over {world} rank(s) (strong scaling)",
+         "concurrency": conc, "rows_per_call": rows, "gpu_launches": int(launches), "clocks": clk,
+         "roofline": {"bound": "hbm", "achieved": round(my_bytes / (my_ms * 1e-3) / 1e9, 3), "peak": peak,
+                      "unit": "GB/s", "frac": round(my_bytes / (my_ms * 1e-3) / 1e9 / peak, 6),
+                      "peak_source": peak_src,
+                      "what": "rank 0: SURVEY 8(d) B_min (4n + 12 n_r + 8 m_r) x its roots / its batch region time "
+                              "(concurrent traversal kernels overlap, so the region is the kernel time)"},
+         "validation": {"rows_checked": int(nval), "rows_ok_I1_I6": int(nok),
+                        "what": "4 rows of the last timed chunk per rank, oracle.check_tree I1-I6 exact"}}
+    if world == 1:
+        b["with_gather"] = {"dfs_per_s": b["dfs_per_s"], "region_ms": b["region_ms"], "bytes_to_rank0": 0,
+                            "what": "N=1: the parent rows are already on rank 0 (no exchange step)"}
+    elif t_gath is not None:
+        b["with_gather"] = {"dfs_per_s": round(k / (t_gath * 1e-3), 3), "region_ms": round(t_gath, 3),
+                            "bytes_to_rank0": int((k - (hi - lo)) * g.n * 4),
+                            "what": f"each chunk's parent rows gathered to rank 0 (NCCL gather, {sub}-row rounds "
+                                    "into a reused rank-0 device buffer)"}
+    if world == 1 and not a.no_cpu_baseline:
+        v, done, nth, el = cpu_oracle_pool(g, roots, a.cpu_seconds)
+        b["cpu_baseline"] = {"value": round(v, 4), "unit": "DFS/s", "cores": nth, "kind": "oracle",
+                             "sample": f"{done} whole Alg-1 traversals of the batch roots in {el:.1f} s, "
+                                       f"a pool of {nth} threads (one root per task) on {cpu_model()}"}
+    return b
 
 
 def e2e_leg(a, g, my_roots, m_r, dfsmod, G):
@@ -427,21 +601,24 @@ def e2e_leg(a, g, my_roots, m_r, dfsmod, G):
 
 
 def reference_arm(a, world, rank):
-    """The CPU oracle (Alg 1, oracle/dfs_oracle.c) as the reference implementation."""
+    """The CPU oracle (Alg 1, oracle/dfs_oracle.c) as the reference implementation: rank 0 only
+    (the other ranks exit without work), one pinned host core, each step one whole traversal."""
     import graphgen
     if world > 1 and rank != 0:
         return
-    g, root0, undirected, desc = graphgen.config_graph(a.config)
+    g, root0, undirected, desc = graphgen.config_graph(a.config if a.config != "batch1024" else "road24m")
     roots = roots_for(g, root0, a.nroots)
-    cpu_oracle(g, roots, 0, steps=a.warmup) if a.warmup > 0 else None
-    v, ms, cnt = cpu_oracle(g, roots, 0, steps=a.steps)
+    if a.warmup > 0:
+        cpu_oracle_pinned(g, roots, 0, steps=min(a.warmup, 3))
+    v, ms, cnt, core = cpu_oracle_pinned(g, roots, 0, steps=a.steps)
     rec = {"metric": METRIC, "value": round(v, 6), "unit": "GTEPS", "impl": "reference",
            "n_gpus": world, "steps": a.steps, "warmup": a.warmup, "ms_per_step": round(ms, 3),
            "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "int32",
            "data": "synthetic",
            "config": {"workload": a.config, "desc": desc, "n": g.n, "m": g.m},
            "cpu_baseline": {"value": round(v, 6), "unit": "GTEPS", "cores": 1, "kind": "oracle",
-                            "sample": f"{cnt} full Alg-1 traversals of {a.config}, 1 host thread"},
+                            "sample": f"{cnt} whole Alg-1 traversals of {a.config}, median; pinned to host "
+                                      f"core {core} of {host_cores()}; {cpu_model()}"},
            "e2e": {"value": round(v, 6), "unit": "GTEPS", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
     print(json.dumps(rec), flush=True)
 

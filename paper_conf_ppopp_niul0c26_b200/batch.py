@@ -150,3 +150,45 @@ def run_batch_chunked(G, out_rows, roots, world: int = 1, rank: int = 0, group=N
             results.append((int(st.root_counts[q, 0]), int(st.root_counts[q, 1]), share))
     it = iter(results)
     return run_batch(lambda root, q: next(it), roots, world=world, rank=rank, group=group, device=device)
+
+
+def reduce_max_sum(maxvals: Sequence[float], sumvals: Sequence[float], world: int, device=None,
+                   group=None) -> Tuple[List[float], List[float]]:
+    """Job-level reduction of per-rank figures (bench.py): element-wise MAX over ranks of
+    ``maxvals`` (device times: the job takes as long as its slowest rank) and SUM of ``sumvals``
+    (edges, bytes, counts).  One all_reduce each; identity for world == 1."""
+    if world == 1:
+        return [float(x) for x in maxvals], [float(x) for x in sumvals]
+    import torch
+    import torch.distributed as dist
+    dev = device if device is not None else torch.device("cpu")
+    tm = torch.tensor([float(x) for x in maxvals], dtype=torch.float64, device=dev)
+    ts = torch.tensor([float(x) for x in sumvals], dtype=torch.float64, device=dev)
+    dist.all_reduce(tm, op=dist.ReduceOp.MAX, group=group)
+    dist.all_reduce(ts, op=dist.ReduceOp.SUM, group=group)
+    return tm.cpu().tolist(), ts.cpu().tolist()
+
+
+def gather_chunk_to_rank0(rows, have: int, nrows: int, sub: int, sink, world: int, rank: int,
+                          group=None, dst: int = 0) -> int:
+    """The C5 exchange step for one chunk of parent rows (bench.py batch pass 2): every rank
+    sends rows [0, nrows) of ``rows`` (a (>= nrows, n) int32 tensor whose first ``have`` rows are
+    valid; the rest are sent as -3 padding so every rank makes the same calls) to ``dst`` in
+    rounds of ``sub`` rows; ``dst`` receives each round into ``sink`` (world tensors of
+    (sub, n) — a reused buffer: the result sink).  Returns the number of rounds (the same on
+    every rank).  Tensors live on the process group's device (CUDA for NCCL, CPU for gloo)."""
+    import torch
+    import torch.distributed as dist
+    rounds = 0
+    n = rows.shape[1]
+    for s0 in range(0, nrows, sub):
+        take = max(0, min(sub, have - s0))
+        if take == sub:
+            src = rows[s0:s0 + sub]
+        else:
+            src = torch.full((sub, n), -3, dtype=rows.dtype, device=rows.device)
+            if take > 0:
+                src[:take] = rows[s0:s0 + take]
+        dist.gather(src.contiguous(), gather_list=sink if rank == dst else None, dst=dst, group=group)
+        rounds += 1
+    return rounds

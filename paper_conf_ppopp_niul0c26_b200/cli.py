@@ -27,6 +27,8 @@ def main(argv=None) -> int:
     ap.add_argument("--root", type=int, action="append", help="explicit source vertex (repeatable)")
     ap.add_argument("--seed", type=int, default=0x6A7)
     ap.add_argument("--csv", help="write per-source results here")
+    ap.add_argument("--save-parents", metavar="NPY",
+                    help="also save the (sources x n) int32 parent arrays (numpy .npy) for checking")
     ap.add_argument("--set", action="append", default=[], metavar="KEY=VALUE",
                     help="dfs_options field, e.g. --set hot_cutoff=32 --set cold_cutoff=64")
     a = ap.parse_args(argv)
@@ -53,11 +55,19 @@ def main(argv=None) -> int:
     out = torch.empty(g.n, dtype=torch.int32, device="cuda")
     G.run(roots[0], out=out, options=options)                 # warm-up
     rows = []
-    for r in roots:
+    saved = None
+    if a.save_parents:
+        import numpy as np
+        saved = np.empty((len(roots), g.n), dtype=np.int32)
+    for q, r in enumerate(roots):
         _, st = G.run(r, out=out, options=options, stats=True)
+        if saved is not None:
+            saved[q] = out.cpu().numpy()
         rows.append(dict(root=r, n_visited=st.n_visited, m_visited=st.m_visited,
                          ms=round(st.kernel_ms, 4), mteps=round(st.m_visited / st.kernel_ms / 1e3, 2)))
     G.close()
+    if saved is not None:
+        np.save(a.save_parents, saved)
     if a.csv:
         with open(a.csv, "w", newline="") as f:
             w = csv.DictWriter(f, fieldnames=list(rows[0]))

@@ -139,6 +139,20 @@ __device__ __forceinline__ unsigned long long globaltimer() {
     asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
     return t;
 }
+__device__ __forceinline__ unsigned long long ld_acquire_u64(const unsigned long long* p) {
+    unsigned long long v;
+    asm volatile("ld.acquire.gpu.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
+    return v;
+}
+// acquire side of a GPU-scope release (pairs with fence_release_gpu + the publishing atomic):
+// SASS CCTL.IVALL — used only on cold paths (after a successful ColdSeg steal reservation)
+__device__ __forceinline__ void fence_acquire_gpu() { asm volatile("fence.acquire.gpu;" ::: "memory"); }
+__device__ __forceinline__ unsigned long long atom_cas_acquire_u64(unsigned long long* p, unsigned long long cmp,
+                                                                   unsigned long long v) {
+    unsigned long long r;
+    asm volatile("atom.acquire.gpu.global.cas.b64 %0, [%1], %2, %3;" : "=l"(r) : "l"(p), "l"(cmp), "l"(v) : "memory");
+    return r;
+}
 __device__ __forceinline__ unsigned long long ld_cg_u64(const unsigned long long* p) {
     unsigned long long v;
     asm volatile("ld.global.cg.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
@@ -334,15 +348,18 @@ __device__ __forceinline__ void smem_unlock(uint32_t* l) { st_release_cta(l, 0u)
 // ------------------------------------------------------------------------------------------
 // chunk pool: tagged lock-free free stack + bump allocator
 // ------------------------------------------------------------------------------------------
+// pool_alloc reads the link chunk_next[idx] written by the pool_free that pushed idx: the head
+// is read with acquire semantics (pairs with pool_free's fence.release + CAS), so the link read
+// is ordered after it; a failed CAS returns the new head, also with acquire semantics.
 __device__ __forceinline__ uint32_t pool_alloc(const KParams& P) {
     Ctl* c = P.ctl;
-    unsigned long long old = ld_relaxed_u64(&c->free_head);
+    unsigned long long old = ld_acquire_u64(&c->free_head);
     for (;;) {
         uint32_t idx = (uint32_t)old;
         if (idx == kEmptySlot) break;
         uint32_t nxt = ld_relaxed_u32(&P.chunk_next[idx]);
         unsigned long long nw = ((unsigned long long)((uint32_t)(old >> 32) + 1u) << 32) | nxt;
-        unsigned long long got = atomicCAS(&c->free_head, old, nw);
+        unsigned long long got = atom_cas_acquire_u64(&c->free_head, old, nw);
         if (got == old) return idx;
         old = got;
     }
@@ -1417,19 +1434,29 @@ __global__ void __launch_bounds__(32 * WMAX, 1) dfs_persistent_kernel(const KPar
                                 if (got == old) { ok = 1; bot = b; break; }
                                 old = got;
                             }
-                            if (!ok) deregister();
+                            // Alg 4 l.20 threadfence: acquire after the reservation, pairing with
+                            // the owner's fence.release before it published `top` (its entries
+                            // and chunk-table slots are visible before we read them)
+                            if (ok) fence_acquire_gpu();
+                            else deregister();
                         }
                         ok = __shfl_sync(kFull, ok, 0);
                         if (ok) {
                             bot = __shfl_sync(kFull, bot, 0);
                             kst = __shfl_sync(kFull, kst, 0);
+                            __syncwarp();                                // lane 0's acquire -> all lanes
                             // remote transfer (Alg 4 l.21-22): L2 loads, addresses from the CAS;
-                            // the range [bot, bot+kst) may straddle two ColdSeg chunks
+                            // the range [bot, bot+kst) may straddle two ColdSeg chunks.  A slot
+                            // that is not a pool chunk (only after an error exit of its owner)
+                            // is never dereferenced.
                             uint32_t* vtab = P.chunk_tab + ((size_t)vwg << P.tab_log2);
                             for (uint32_t q = lane; q < kst; q += 32u) {
                                 const uint32_t p = bot + q;
                                 const uint32_t c = ld_relaxed_u32(&vtab[(p >> kChunkLog2) & tmask]);
-                                ring[(my_head + q) & (H - 1)] = ld_cg_u64(P.pool + ((size_t)c << kChunkLog2) + (p & (kChunk - 1)));
+                                if (c < P.n_chunks)
+                                    ring[(my_head + q) & (H - 1)] = ld_cg_u64(P.pool + ((size_t)c << kChunkLog2) + (p & (kChunk - 1)));
+                                else
+                                    ring[(my_head + q) & (H - 1)] = pack_entry((uint32_t)P.root, P.m);   // exhausted entry
                             }
                             __syncwarp();
                             if (lane == 0) {
@@ -1441,10 +1468,12 @@ __global__ void __launch_bounds__(32 * WMAX, 1) dfs_persistent_kernel(const KPar
                                     const uint32_t part = left < in_chunk ? left : in_chunk;
                                     uint32_t* slot = &vtab[(p >> kChunkLog2) & tmask];
                                     const uint32_t c = ld_relaxed_u32(slot);
-                                    const uint32_t before = atomicAdd(&P.chunk_consumed[c], part);
-                                    if (before + part == kChunk) {             // chunk fully consumed
-                                        st_relaxed_u32(slot, kEmptySlot);
-                                        pool_free(P, c);
+                                    if (c < P.n_chunks) {
+                                        const uint32_t before = atomicAdd(&P.chunk_consumed[c], part);
+                                        if (before + part == kChunk) {         // chunk fully consumed
+                                            st_relaxed_u32(slot, kEmptySlot);
+                                            pool_free(P, c);
+                                        }
                                     }
                                     p += part; left -= part;
                                 }
@@ -1480,8 +1509,11 @@ exit_loop:
     __syncwarp();
     if (STATS && !active && t_idle0 && lane == 0) cnt[kCntIdleNs] += globaltimer() - t_idle0;
     // release the ColdSeg chunks still mapped by this warp so the chunk table is all-empty
-    // for the next run (thieves free the chunks they fully consume)
-    {
+    // for the next run (thieves free the chunks they fully consume).  Only after a clean
+    // termination (every ColdSeg is then empty): after an error exit other warps may still
+    // steal from this warp's ColdSeg, so its table stays as it is and the host re-initialises
+    // the whole table before the next run (Slot::tab_dirty)
+    if (__shfl_sync(kFull, lane == 0 ? (fence_acquire_gpu(), ld_relaxed_s32(&P.ctl->status)) : 0, 0) == 0) {
         const unsigned long long word = ld_relaxed_u64(&P.cold_tb[gw]);
         const uint32_t bot = (uint32_t)word;
         const uint32_t lo = bot >> kChunkLog2;     // chunks below were freed by the thieves

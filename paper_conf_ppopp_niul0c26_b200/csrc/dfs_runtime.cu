@@ -76,6 +76,7 @@ struct Slot {
     int* status = nullptr;                  // worst status over the slot's traversals in a batch
     unsigned long long* block_claims = nullptr;   // per-block claim counts (stats), else null
     size_t tab_words = 0;
+    int64_t n_warps_cap = 0;                // warps (blocks x warps per block) the scratch is sized for
     uint32_t n_chunks = 0;
     bool tab_dirty = false;
     cudaStream_t stream = nullptr;          // own stream (slots >= 1 of a concurrent batch)
@@ -91,7 +92,8 @@ struct dfs_graph {
     int sms = 0;
     int max_blocks = 0;          // co-resident 32-warp blocks (allocation bound)
     int max_clusters[4] = {0, 0, 0, 0};   // co-resident clusters of 1/2/4/8 CTAs (lazy)
-    size_t persist_bytes = 0;    // persisting-L2 set-aside granted for l2_persist_mb (0 = none)
+    size_t persist_req = 0;      // l2_persist_mb requested last (bytes)
+    size_t persist_bytes = 0;    // persisting-L2 set-aside granted for it (0 = none)
     size_t max_window_bytes = 0; // cudaDevAttrMaxAccessPolicyWindowSize
     int tab_log2 = 0;
     uint32_t* d_rp = nullptr;
@@ -128,12 +130,15 @@ static void free_graph(dfs_graph* g) {
     delete g;
 }
 
-// allocate scratch slot k (sized for every warp of the device, so any block split fits)
-static int ensure_slot(dfs_graph* g, int k) {
+// allocate scratch slot k for traversals on up to `n_warps` warps (slot 0: every warp of the
+// device; the slots of a concurrent batch: their block share).  A slot that is too small is
+// reallocated.
+static int ensure_slot(dfs_graph* g, int k, int64_t n_warps) {
     Slot& s = g->slots[k];
-    if (s.ready) return DFS_OK;
+    if (s.ready && s.n_warps_cap >= n_warps) return DFS_OK;
+    if (s.ready) { cudaStreamSynchronize(s.stream ? s.stream : g->stream); free_slot(s); }
     const int64_t n = g->n;
-    const int64_t n_warps = (int64_t)g->max_blocks * kMaxWarps;
+    s.n_warps_cap = n_warps;
     s.tab_words = (size_t)n_warps << g->tab_log2;
     // pool: sum of live spans <= n, plus <= 4 partially used chunks per warp (reading S9)
     s.n_chunks = (uint32_t)(n / kChunk + 4 * n_warps + 16);
@@ -248,7 +253,7 @@ dfs_graph* dfs_graph_create(const int64_t* row_ptr, const int32_t* col_idx, int6
         cudaMalloc(&g->d_col, (size_t)(m + 8) * sizeof(int32_t)) != cudaSuccess) {   // padded for 128-bit loads
         cudaGetLastError(); free_graph(g); fail(DFS_ENOMEM); return nullptr;
     }
-    const int rc = ensure_slot(g, 0);
+    const int rc = ensure_slot(g, 0, (int64_t)g->max_blocks * kMaxWarps);
     if (rc != DFS_OK) { free_graph(g); fail(rc); return nullptr; }
 
     // ---- copy + validate + narrow (step a1) ----
@@ -497,21 +502,28 @@ static int resolve_options(dfs_graph* g, const dfs_options* in, int num_roots, d
     if (blocks > g->max_blocks || (conc > 1 && blocks * conc > g->max_blocks)) return DFS_EINVAL;
     if (o.deterministic) { blocks = 1; warps = 1; o.intra_steal = 0; o.inter_steal = 0; o.cluster = 0; }
     if (o.l2_persist_mb < -1) return DFS_EINVAL;
-    if (o.l2_persist_mb == 0) o.l2_persist_mb = o.window == 128 ? 64 : -1;   // auto (A/B: rmat24 -4.8%)
+    const bool persist_auto = o.l2_persist_mb == 0;
+    if (persist_auto) o.l2_persist_mb = o.window == 128 ? 64 : -1;   // auto (A/B: rmat24 -4.8%)
     if (o.l2_persist_mb > 0) {
-        // device-wide persisting-L2 set-aside (capped by the device); done once per handle
+        // device-wide persisting-L2 set-aside (capped by the device); done once per handle.
+        // Where it cannot be granted (MIG: max 0; MPS: the limit is not settable) an explicit
+        // request fails with DFS_ECUDA and the auto setting quietly runs without it.
         const size_t want = (size_t)o.l2_persist_mb << 20;
-        if (g->persist_bytes != want) {
+        if (g->persist_req != want) {
             int maxp = 0, maxw = 0;
             cudaDeviceGetAttribute(&maxp, cudaDevAttrMaxPersistingL2CacheSize, g->device);
             cudaDeviceGetAttribute(&maxw, cudaDevAttrMaxAccessPolicyWindowSize, g->device);
-            const size_t bytes = std::min(want, (size_t)maxp);
+            cudaGetLastError();
+            const size_t bytes = std::min(want, (size_t)std::max(maxp, 0));
             if (bytes == 0 || maxw <= 0 || cudaDeviceSetLimit(cudaLimitPersistingL2CacheSize, bytes) != cudaSuccess) {
                 cudaGetLastError();
-                return DFS_ECUDA;
+                if (!persist_auto) return DFS_ECUDA;
+                o.l2_persist_mb = -1;
+            } else {
+                g->persist_req = want;
+                g->persist_bytes = bytes;                 // granted (hitRatio uses this)
+                g->max_window_bytes = (size_t)maxw;
             }
-            g->persist_bytes = want;
-            g->max_window_bytes = (size_t)maxw;
         }
     }
     if (o.cluster > 1) {
@@ -674,8 +686,6 @@ static int run_sequential(dfs_graph* g, const int32_t* roots, int32_t k, int32_t
 static int run_concurrent(dfs_graph* g, const int32_t* roots, int32_t k, int32_t* out, bool out_dev,
                           const dfs_options& o, int blocks, int warps, int conc, dfs_stats* stats) {
     for (int c = 0; c < conc; ++c) {
-        int rc = ensure_slot(g, c);
-        if (rc != DFS_OK) return fail(rc);
         Slot& sl = g->slots[c];
         if (sl.block_claims) { cudaFree(sl.block_claims); sl.block_claims = nullptr; }
         if (!out_dev && !sl.parent) {
@@ -750,6 +760,12 @@ static int run_concurrent(dfs_graph* g, const int32_t* roots, int32_t k, int32_t
     return DFS_OK;
 }
 
+static bool is_pinned_host(const void* p) {
+    cudaPointerAttributes a;
+    if (cudaPointerGetAttributes(&a, p) != cudaSuccess) { cudaGetLastError(); return false; }
+    return a.type == cudaMemoryTypeHost;
+}
+
 static int run_many(dfs_graph* g, const int32_t* roots_host, int32_t k, int32_t* out, bool out_dev,
                     const dfs_options* opt, dfs_stats* stats) {
     dfs_options o;
@@ -758,8 +774,39 @@ static int run_many(dfs_graph* g, const int32_t* roots_host, int32_t k, int32_t*
     if (rc != DFS_OK) return fail(rc);
     for (int32_t q = 0; q < k; ++q)
         if (roots_host[q] < 0 || roots_host[q] >= g->n) return fail(DFS_EINVAL);
+    // concurrent slots: scratch sized for their block share; when the device cannot hold
+    // `conc` slots, fewer traversals run concurrently (each on a larger share)
+    const bool auto_blocks = o.blocks <= 0;
+    while (conc > 1) {
+        int c = 1;
+        rc = DFS_OK;
+        for (; c < conc; ++c) {
+            rc = ensure_slot(g, c, (int64_t)blocks * warps);
+            if (rc != DFS_OK) break;
+        }
+        if (rc == DFS_OK) break;
+        if (rc != DFS_ENOMEM) return fail(rc);
+        for (int q = c; q < kMaxSlots; ++q) free_slot(g->slots[q]);
+        conc = c;
+        if (auto_blocks) blocks = std::max(1, g->max_blocks / conc);
+        if (conc == 1) blocks = auto_blocks ? g->max_blocks : blocks;
+    }
     if (conc <= 1) return run_sequential(g, roots_host, k, out, out_dev, o, blocks, warps, stats);
-    return run_concurrent(g, roots_host, k, out, out_dev, o, blocks, warps, conc, stats);
+    // a device->pageable-host copy is synchronous, which would serialise the concurrent
+    // traversals: the output range is page-locked for the call (or the batch runs sequentially
+    // on the whole GPU when it cannot be)
+    bool registered = false;
+    if (!out_dev && !is_pinned_host(out)) {
+        if (cudaHostRegister(out, (size_t)k * (size_t)g->n * sizeof(int32_t), cudaHostRegisterDefault) != cudaSuccess) {
+            cudaGetLastError();
+            if (auto_blocks) blocks = g->max_blocks;
+            return run_sequential(g, roots_host, k, out, out_dev, o, blocks, warps, stats);
+        }
+        registered = true;
+    }
+    rc = run_concurrent(g, roots_host, k, out, out_dev, o, blocks, warps, conc, stats);
+    if (registered) { cudaHostUnregister(out); cudaGetLastError(); }
+    return rc;
 }
 
 extern "C" {

@@ -16,7 +16,8 @@ from typing import Optional
 import numpy as np
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-_SO = os.path.join(_HERE, "libdfs.so")
+# DFS_LIB: an alternative build of the same library (A/B experiments, scripts/ab_libs.py)
+_SO = os.environ.get("DFS_LIB") or os.path.join(_HERE, "libdfs.so")
 
 DFS_ROOT_PARENT = -1
 DFS_UNREACHED = -2
@@ -155,14 +156,16 @@ def lib_path() -> str:
     return _SO
 
 
-def load_library():
-    """Load libdfs.so; raises if it is missing (no fallback path exists)."""
+def load_library(path: Optional[str] = None):
+    """Load libdfs.so; raises if it is missing (no fallback path exists).  ``path`` loads another
+    build of the same library without caching it (A/B experiments)."""
     global _lib
-    if _lib is None:
-        if not os.path.exists(_SO):
-            raise ImportError(f"{_SO} is missing: run `python __graft_entry__.py` (build()) first; "
+    if path is not None or _lib is None:
+        so = path or _SO
+        if not os.path.exists(so):
+            raise ImportError(f"{so} is missing: run `python __graft_entry__.py` (build()) first; "
                               "there is no CPU fallback")
-        lib = ctypes.CDLL(_SO)
+        lib = ctypes.CDLL(so)
         P, I32, I64 = ctypes.c_void_p, ctypes.c_int32, ctypes.c_int64
         lib.dfs_options_default.argtypes = [ctypes.POINTER(_Options)]
         lib.dfs_options_default.restype = None
@@ -190,6 +193,8 @@ def load_library():
         lib.dfs_last_error.restype = ctypes.c_int
         lib.dfs_strerror.argtypes = [ctypes.c_int]
         lib.dfs_strerror.restype = ctypes.c_char_p
+        if path is not None:
+            return lib
         _lib = lib
     return _lib
 
@@ -239,9 +244,9 @@ class Graph:
     the CPU or on the current GPU; they are copied, so the caller may drop them afterwards.
     """
 
-    def __init__(self, row_ptr, col_idx):
+    def __init__(self, row_ptr, col_idx, lib=None):
         import torch
-        self._lib = load_library()
+        self._lib = lib if lib is not None else load_library()
         rp = _as(row_ptr, np.int64, torch.int64)
         ci = _as(col_idx, np.int32, torch.int32)
         n = int(rp.shape[0]) - 1

@@ -47,3 +47,10 @@ def test_product_arm_json_line():
     assert e["d2h_bytes_per_step"] >= 4 * d["config"]["n"]          # the parent array comes back
     assert {"sm_mhz", "sm_max_mhz", "reasons"} <= d["clocks"].keys()
     assert d["validation"] and all(v["i6"] == 1 for v in d["validation"].values())
+
+
+def test_gpus_flag_relaunches_under_torchrun():
+    """`bench.py --gpus 2` without torchrun re-launches itself with 2 ranks (torch.distributed.run);
+    the reference arm runs on rank 0 only, the other rank exits 0 without work: one JSON line."""
+    d = _run(["--impl", "reference", "--gpus", "2", "--config", "grid256", "--steps", "1", "--warmup", "0"], 600)
+    assert d["impl"] == "reference" and d["n_gpus"] == 2 and d["value"] > 0

@@ -1,6 +1,6 @@
 """Pin the oracle's acceptance checker by set equality with brute force.
 
-For tiny graphs (<= 7 vertices), over EVERY candidate parent array (tests/bruteforce.py):
+For tiny graphs (<= 8 vertices), over EVERY candidate parent array (tests/bruteforce.py):
   * {checker I1-I6 accepts} == async in-order-scan outcome set   (I6 is exactly that model)
   * {checker I1-I5 + I7 accepts} == classical DFS trees over all adjacency permutations
   * Alg 1 oracle tree ∈ both; k-agent work-stealing outcomes ⊆ I6 set.
@@ -123,3 +123,26 @@ def test_i6_rejects_out_of_order_claim():
     assert oracle.check_tree(rp, ci, 0, np.array([-1, 0, 0], dtype=np.int32)).ok
     r = oracle.check_tree(rp, ci, 0, np.array([-1, 2, 0], dtype=np.int32))
     assert r.failed() == ["i6"]
+
+
+def _graphs_p(n_graphs, seed, n, p_lo, p_hi, directed_frac):
+    rng = np.random.default_rng(seed)
+    for k in range(n_graphs):
+        directed = rng.random() < directed_frac
+        p = float(rng.uniform(p_lo, p_hi))
+        rp, col = bf.random_tiny_graph(rng, n, p, directed, self_loops=directed and k % 2 == 0)
+        root = int(rng.integers(0, n))
+        yield rp, col, root, not directed
+
+
+def test_eight_vertex_graphs():
+    """north_star / SURVEY T2: brute force on graphs of 8 vertices (the largest size named),
+    undirected and directed (with self loops), sparse enough that the enumerations finish."""
+    seen = 0
+    for rp, col, root, undirected in _graphs_p(6, 8, 8, 0.25, 0.4, 0.5):
+        adj, classical, scan, acc6, acc7 = _sets_for(rp, col, root, undirected)
+        assert acc6 == scan and acc7 == classical, (adj, root)
+        lex = tuple(oracle.dfs(rp, col, root).tolist())
+        assert lex in classical and lex in scan
+        seen += len(bf.reach_set(adj, root)) == 8
+    assert seen >= 2          # at least two cases reach all 8 vertices

@@ -100,3 +100,57 @@ def test_run_batch_gloo_world2():
             assert parents is None
     res0 = batch.BatchResult(out[0][1], (0, 5), out[0][2], out[0][3])
     assert res0.dfs_per_s() == pytest.approx(len(roots) / (out[0][3] * 1e-3))
+
+
+def _worker_bench_exchange(rank, world, port, q):
+    """bench.py's exchange helpers: reduce_max_sum (job time = max over ranks, totals = sums)
+    and gather_chunk_to_rank0 (the C5 gather of parent rows into a reused rank-0 sink), with
+    uneven slices (rank 1 holds one row fewer) so the padding path runs."""
+    os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    try:
+        mx, sm = batch.reduce_max_sum([1.0 + rank, 10.0 - rank], [2.0 * rank + 1, 5.0], world)
+        n, nrows, sub = 17, 7, 3
+        have = nrows - rank                                    # rank 0: 7 rows, rank 1: 6
+        rows = torch.arange(nrows * n, dtype=torch.int32).reshape(nrows, n) + 1000 * rank
+        sink = [torch.empty((sub, n), dtype=torch.int32) for _ in range(world)] if rank == 0 else None
+        received = []
+        rounds = 0
+        for s0 in range(0, nrows, sub):
+            # one round at a time so the test can copy out what the sink received
+            rounds += batch.gather_chunk_to_rank0(rows[s0:], max(0, have - s0), min(sub, nrows - s0), sub,
+                                                  sink, world, rank)
+            if rank == 0:
+                received.append([t.clone() for t in sink])
+        q.put((rank, mx, sm, rounds, received))
+    finally:
+        dist.destroy_process_group()
+
+
+def test_bench_exchange_gloo_world2():
+    world, port = 2, _free_port()
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    procs = [ctx.Process(target=_worker_bench_exchange, args=(r, world, port, q)) for r in range(world)]
+    for p in procs:
+        p.start()
+    out = sorted([q.get(timeout=240) for _ in range(world)], key=lambda t: t[0])
+    for p in procs:
+        p.join(timeout=60)
+        assert p.exitcode == 0
+    n, nrows, sub = 17, 7, 3
+    for rank, mx, sm, rounds, received in out:
+        assert mx == [2.0, 10.0] and sm == [4.0, 10.0]
+        assert rounds == 3
+    received = out[0][4]
+    for r_i, s0 in enumerate(range(0, nrows, sub)):
+        for src in range(world):
+            have = nrows - src
+            want = torch.arange(nrows * n, dtype=torch.int32).reshape(nrows, n) + 1000 * src
+            got = received[r_i][src]
+            for j in range(sub):
+                row = s0 + j
+                if row < have and row < nrows:
+                    assert torch.equal(got[j], want[row]), (r_i, src, j)
+                else:
+                    assert bool((got[j] == -3).all()), (r_i, src, j)

@@ -356,12 +356,31 @@ def test_cli_on_matrix_market(tmp_path, capsys):
     p = tmp_path / "road.mtx"
     graphgen.write_mtx(g, str(p))
     out_csv = tmp_path / "perf.csv"
-    assert cli.main(["--mtx", str(p), "--roots", "4", "--csv", str(out_csv), "--set", "hot_cutoff=4"]) == 0
+    npy = tmp_path / "parents.npy"
+    assert cli.main(["--mtx", str(p), "--roots", "4", "--csv", str(out_csv), "--set", "hot_cutoff=4",
+                     "--save-parents", str(npy)]) == 0
     summary = _json.loads(capsys.readouterr().out.strip().splitlines()[-1])
     assert summary["sources"] == 4 and summary["n"] == g.n and summary["m"] == g.m
     rows = out_csv.read_text().strip().splitlines()
     assert len(rows) == 5 and rows[0].startswith("root,n_visited")
     assert all(int(r.split(",")[1]) == g.n for r in rows[1:])          # connected: all reached
+    # every tree the CLI produced from the .mtx path is a valid DFS tree of the file's graph
+    gm = graphgen.read_mtx(str(p))
+    assert np.array_equal(gm.row_ptr, g.row_ptr) and np.array_equal(gm.col_idx, g.col_idx)
+    parents = np.load(npy)
+    assert parents.shape == (4, g.n)
+    for q, line in enumerate(rows[1:]):
+        _valid(gm, int(line.split(",")[0]), parents[q])
+    # a directed file written from shuffled lists (not symmetrised; the reader sorts rows)
+    gd = graphgen.shuffle_lists(graphgen.random_graph(3000, 9000, seed=8, symmetric=False), 3)
+    pd = tmp_path / "dir.mtx"
+    graphgen.write_mtx(gd, str(pd))
+    gdm = graphgen.read_mtx(str(pd))
+    assert cli.main(["--mtx", str(pd), "--root", "0", "--root", "17", "--save-parents", str(npy)]) == 0
+    capsys.readouterr()
+    parents = np.load(npy)
+    for q, r in enumerate((0, 17)):
+        _valid(gdm, r, parents[q], undirected=False)
 
 
 @pytest.mark.parametrize("cl", [2, 4])
