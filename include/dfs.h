@@ -159,6 +159,14 @@ typedef struct dfs_options {
                                 in L2 while col_idx streams.  0 (default) = auto: 64 MB with
                                 128-wide windows (A/B on B200: RMAT-24 -4.8%, road/path neutral),
                                 else off; -1 = off.  The limit stays set after the handle is gone  */
+    int32_t walker_lanes;    /* lanes per walker: 32 = the warp kernel (one walker per warp, windows of
+                                `window` positions); 16, 8 or 4 = the sub-warp walker kernel (32/L
+                                independent walkers per warp, each with its own HotRing/ColdSeg and
+                                an L-position window); 0 = auto.
+                                deterministic, cluster >= 1 and window = 128 use the warp kernel   */
+    int32_t steal_period;    /* walker kernel: an idle walker in a warp that still has busy walkers
+                                tries one Alg 3 steal every steal_period steps (power of two <= 1024;
+                                0 = 1)                                                             */
 } dfs_options;
 
 typedef struct dfs_stats {

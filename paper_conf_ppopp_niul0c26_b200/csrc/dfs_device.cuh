@@ -111,6 +111,7 @@ struct KParams {
     int steal_tries;                         // Alg 3 victims tried per idle round (best first)
     int bulk_copy;                           // flush/refill with cp.async.bulk (TMA ablation)
     uint32_t period_mask;                    // spill_period - 1
+    uint32_t steal_period_mask;              // walker kernel: steal_period - 1
 };
 
 // ------------------------------------------------------------------------------------------

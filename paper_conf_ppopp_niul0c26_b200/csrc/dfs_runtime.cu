@@ -18,6 +18,7 @@
 
 #include "../../include/dfs.h"
 #include "dfs_device.cuh"
+#include "dfs_walker.cuh"
 
 using namespace b200dfs;
 
@@ -55,8 +56,23 @@ const void* const* kernel_table() {
 #undef DFS_K
 constexpr int kNumKernels = 24;
 
+// sub-warp walker kernels (dfs_walker.cuh): [G = 16, 8, 4][stats]; HotRing H = 16 * G entries
+// per walker, so a 32-warp CTA holds 128 KB of rings for every G
+#define DFS_WK(G, S) (const void*)dfs_walker_kernel<G, 16 * G, S>
+const void* const* walker_table() {
+    static const void* const t[6] = {DFS_WK(16, false), DFS_WK(16, true), DFS_WK(8, false), DFS_WK(8, true),
+                                     DFS_WK(4, false), DFS_WK(4, true)};
+    return t;
+}
+#undef DFS_WK
+constexpr int kNumWalkerKernels = 6;
+int walker_index(int lanes) { return lanes == 16 ? 0 : lanes == 8 ? 2 : 4; }
+
 size_t smem_bytes(int warps) {
     return ((sizeof(SmemCtl) + 15) & ~size_t(15)) + (size_t)warps * kRing * sizeof(unsigned long long);
+}
+size_t walker_smem_bytes(int warps, int lanes) {
+    return ((sizeof(SmemW) + 15) & ~size_t(15)) + (size_t)warps * (32 / lanes) * (16 * lanes) * sizeof(unsigned long long);
 }
 
 // per-traversal scratch set
@@ -236,6 +252,12 @@ dfs_graph* dfs_graph_create(const int64_t* row_ptr, const int32_t* col_idx, int6
         if (cudaFuncSetAttribute(kernel_table()[kf], cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm32) != cudaSuccess)
             attr_ok = false;
     }
+    for (int kf = 0; kf < kNumWalkerKernels; ++kf) {
+        const int lanes = kf < 2 ? 16 : kf < 4 ? 8 : 4;
+        if (cudaFuncSetAttribute(walker_table()[kf], cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                 (int)walker_smem_bytes(32, lanes)) != cudaSuccess)
+            attr_ok = false;
+    }
     if (!attr_ok) { cudaGetLastError(); delete g; fail(DFS_ECUDA); return nullptr; }
     int per_sm = 0;
     if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, dfs_persistent_kernel<kRing, 4, 32, false, false, false>, 1024, sm32) !=
@@ -367,8 +389,11 @@ static int launch_one(dfs_graph* g, Slot& sl, cudaStream_t s, int32_t root, int3
                                                (int64_t)g->sms * 8);
     const uint32_t bstride = 2u;                              // {visited, leaf} pairs (both windows)
     sl.bstride = bstride;
+    const int wl = o.walker_lanes;                            // resolved: 32 = warp kernel
+    const int owners = blocks * warps * (wl == 32 ? 1 : 32 / wl);   // stack owners (warps or walkers)
+    if (owners > sl.n_warps_cap) return DFS_EINTERNAL;
     dfs_reset_kernel<<<rblocks, 256, 0, s>>>(sl.bitmap, nwords, bstride, o.leaf_skip >= 2 ? g->d_leaf : nullptr,
-                                            sl.cold_tb, (uint32_t)(blocks * warps),
+                                            sl.cold_tb, (uint32_t)owners,
                                             sl.block_cold, (uint32_t)blocks, sl.ctl, d_out, root,
                                             sl.tab, sl.tab_dirty ? sl.tab_words : 0);
     g->launches++;
@@ -400,6 +425,7 @@ static int launch_one(dfs_graph* g, Slot& sl, cudaStream_t s, int32_t root, int3
     P.steal_tries = o.steal_tries > 0 ? o.steal_tries : 1;
     P.bulk_copy = o.bulk_copy;
     P.period_mask = (uint32_t)(o.spill_period > 0 ? o.spill_period : 32) - 1u;
+    P.steal_period_mask = (uint32_t)(o.steal_period > 0 ? o.steal_period : 1) - 1u;
     const bool tl = g->d_timeline && &sl == &g->slots[0];
     P.timeline = tl ? g->d_timeline : nullptr;
     P.timeline_len = tl ? (g->timeline_len / 3u) * 2u : 0;   // kernel: three regions of len/3
@@ -409,8 +435,9 @@ static int launch_one(dfs_graph* g, Slot& sl, cudaStream_t s, int32_t root, int3
     void* args[] = {(void*)&P};
     const int cl = o.cluster > 1 ? o.cluster : 1;
     // the cluster build has no bulk variant: cluster >= 1 takes precedence over bulk_copy
-    const void* kfn = kernel_table()[(o.cluster >= 1 ? 8 : o.bulk_copy ? 16 : 0) + (o.window == 128 ? 4 : 0) +
-                                     (warps <= 16 ? 2 : 0) + (o.collect_stats ? 1 : 0)];
+    const void* kfn = wl != 32 ? walker_table()[walker_index(wl) + (o.collect_stats ? 1 : 0)]
+                               : kernel_table()[(o.cluster >= 1 ? 8 : o.bulk_copy ? 16 : 0) + (o.window == 128 ? 4 : 0) +
+                                                (warps <= 16 ? 2 : 0) + (o.collect_stats ? 1 : 0)];
     if (timed) cudaEventRecord(sl.evk0, s);
     cudaError_t e;
     // launch attributes: cooperative (single traversals), cluster dimension (cluster tier,
@@ -440,7 +467,7 @@ static int launch_one(dfs_graph* g, Slot& sl, cudaStream_t s, int32_t root, int3
         ++na;
     }
     cfg.gridDim = dim3(blocks); cfg.blockDim = dim3(32 * warps);
-    cfg.dynamicSmemBytes = smem_bytes(warps); cfg.stream = s;
+    cfg.dynamicSmemBytes = wl != 32 ? walker_smem_bytes(warps, wl) : smem_bytes(warps); cfg.stream = s;
     cfg.attrs = at; cfg.numAttrs = na;
     // concurrent batch slots launch non-cooperatively: co-residency is not required for progress —
     // a block that starts late finds the traversal done or steals the remaining work
@@ -489,7 +516,15 @@ static int resolve_options(dfs_graph* g, const dfs_options* in, int num_roots, d
     if (o.reserved0 != 0) return DFS_EINVAL;
     if (o.spill_period < 0 || o.spill_period > 1024 || (o.spill_period & (o.spill_period - 1))) return DFS_EINVAL;
     if (o.cluster < 0 || o.cluster > 8 || (o.cluster > 1 && (o.cluster & (o.cluster - 1)))) return DFS_EINVAL;
+    if (o.walker_lanes != 0 && o.walker_lanes != 32 && o.walker_lanes != 16 && o.walker_lanes != 8 && o.walker_lanes != 4)
+        return DFS_EINVAL;
+    if (o.steal_period < 0 || o.steal_period > 1024 || (o.steal_period & (o.steal_period - 1))) return DFS_EINVAL;
+    const bool window_auto = o.window == 0;
     if (o.window == 0) o.window = (g->n > 0 && g->m >= 8 * g->n) ? 128 : 32;   // wide windows for dense lists
+    // kernel: the warp kernel (one walker per warp) or sub-warp walkers; auto = warp kernel
+    if (o.walker_lanes == 0) o.walker_lanes = 32;
+    if (o.deterministic || o.cluster >= 1 || (o.window == 128 && !window_auto)) o.walker_lanes = 32;
+    if (o.walker_lanes != 32) o.window = 32;
     if (o.window != 32 && o.window != 128) return DFS_EINVAL;
     if (o.concurrency < 0 || o.concurrency > kMaxSlots) return DFS_EINVAL;
     warps = o.warps_per_block <= 0 ? 32 : o.warps_per_block;
@@ -605,6 +640,11 @@ static int finish_counts(dfs_graph* g, int32_t k, dfs_stats* stats, int64_t& nv,
 static int run_sequential(dfs_graph* g, const int32_t* roots, int32_t k, int32_t* out, bool out_dev,
                           const dfs_options& o, int blocks, int warps, dfs_stats* stats) {
     Slot& sl = g->slots[0];
+    {
+        const int64_t owners = (int64_t)blocks * warps * (o.walker_lanes == 32 ? 1 : 32 / o.walker_lanes);
+        const int rc = ensure_slot(g, 0, std::max<int64_t>(owners, (int64_t)g->max_blocks * kMaxWarps));
+        if (rc != DFS_OK) return fail(rc);
+    }
     if (!out_dev && !sl.parent) {
         if (cudaMalloc(&sl.parent, (size_t)g->n * sizeof(int32_t)) != cudaSuccess) {
             cudaGetLastError();
@@ -778,14 +818,15 @@ static int run_many(dfs_graph* g, const int32_t* roots_host, int32_t k, int32_t*
     // `conc` slots, fewer traversals run concurrently (each on a larger share)
     const bool auto_blocks = o.blocks <= 0;
     while (conc > 1) {
-        int c = 1;
+        int c = 0;
         rc = DFS_OK;
+        const int64_t owners = (int64_t)blocks * warps * (o.walker_lanes == 32 ? 1 : 32 / o.walker_lanes);
         for (; c < conc; ++c) {
-            rc = ensure_slot(g, c, (int64_t)blocks * warps);
+            rc = ensure_slot(g, c, c == 0 ? std::max<int64_t>(owners, (int64_t)g->max_blocks * kMaxWarps) : owners);
             if (rc != DFS_OK) break;
         }
         if (rc == DFS_OK) break;
-        if (rc != DFS_ENOMEM) return fail(rc);
+        if (rc != DFS_ENOMEM || c == 0) return fail(rc);
         for (int q = c; q < kMaxSlots; ++q) free_slot(g->slots[q]);
         conc = c;
         if (auto_blocks) blocks = std::max(1, g->max_blocks / conc);

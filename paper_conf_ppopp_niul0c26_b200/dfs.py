@@ -53,7 +53,8 @@ class _Options(ctypes.Structure):
                 ("leaf_skip", ctypes.c_int32), ("cluster", ctypes.c_int32),
                 ("cluster_late", ctypes.c_int32), ("steal_tries", ctypes.c_int32),
                 ("bulk_copy", ctypes.c_int32), ("spill_period", ctypes.c_int32),
-                ("l2_persist_mb", ctypes.c_int32)]
+                ("l2_persist_mb", ctypes.c_int32), ("walker_lanes", ctypes.c_int32),
+                ("steal_period", ctypes.c_int32)]
 
 
 class _Stats(ctypes.Structure):
@@ -106,6 +107,8 @@ class Options:
     bulk_copy: Optional[bool] = None
     spill_period: Optional[int] = None
     l2_persist_mb: Optional[int] = None
+    walker_lanes: Optional[int] = None
+    steal_period: Optional[int] = None
 
     def to_c(self) -> _Options:
         o = _Options()

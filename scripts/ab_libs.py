@@ -34,6 +34,8 @@ def main():
     ap.add_argument("--steps", type=int, default=8)
     ap.add_argument("--nroots", type=int, default=16)
     ap.add_argument("--set", action="append", default=[], help="dfs_options KEY=VALUE (all builds)")
+    ap.add_argument("--variant", action="append", default=[],
+                    help="comma-separated dfs_options KEY=VALUE list; every build x variant is timed")
     ap.add_argument("--batch", type=int, default=0, help="time dfs_run_batch of this many roots instead")
     ap.add_argument("--validate", type=int, default=1)
     ap.add_argument("--out")
@@ -54,25 +56,36 @@ def main():
     for kv in a.set:
         k, _, v = kv.partition("=")
         opts[k] = int(v)
-    o = Options(**opts) if opts else None
+    variants = []
+    for v in (a.variant or [""]):
+        d = dict(opts)
+        for kv in filter(None, v.split(",")):
+            k, _, x = kv.partition("=")
+            d[k] = int(x)
+        variants.append((v, Options(**d) if d else None))
     libs = [dfsmod.load_library(os.path.abspath(p)) for p in a.libs]
-    Gs = [Graph(g.row_ptr, g.col_idx, lib=lib) for lib in libs]
+    Gs0 = [Graph(g.row_ptr, g.col_idx, lib=lib) for lib in libs]
+    # one timed arm per (build, variant); arms of one build share its graph handle
+    arms = [(Gs0[li], f"{p}" + (f" [{vn}]" if vn else ""), vo) for li, p in enumerate(a.libs) for vn, vo in variants]
+    Gs = [x[0] for x in arms]
+    names = [x[1] for x in arms]
+    opts_of = [x[2] for x in arms]
     out = torch.empty(g.n, dtype=torch.int32, device="cuda")
     bout = torch.empty((a.batch, g.n), dtype=torch.int32, device="cuda") if a.batch else None
     broots = graphgen.random_roots(g, a.batch, seed=0xC5) if a.batch else None
     deg = np.diff(g.row_ptr)
-    for G, p in zip(Gs, a.libs):
+    for G, p, o in zip(Gs, names, opts_of):
         for r in roots[:a.validate]:
             par = G.run(r, out=out, options=o).cpu().numpy()
             res = oracle.check_tree(g.row_ptr, g.col_idx, r, par, undirected=undirected)
             assert res.ok, (p, r, res)
         G.run(roots[0], out=out, options=o)
-    res = {p: {"step_ms": [], "trav_ms": [], "gteps": []} for p in a.libs}
+    res = {p: {"step_ms": [], "trav_ms": [], "gteps": []} for p in names}
     s = 0
     for rep in range(a.reps):
         order = list(range(len(Gs))) if rep % 2 == 0 else list(reversed(range(len(Gs))))
         for i in order:
-            G, p = Gs[i], a.libs[i]
+            G, p, o = Gs[i], names[i], opts_of[i]
             if a.batch:
                 torch.cuda.synchronize()
                 _, st = G.run_batch(broots, out=bout, options=o, stats=True)
@@ -92,7 +105,7 @@ def main():
             res[p]["gteps"].append(ed / km / 1e6)
         s += a.steps
     lines = []
-    for p in a.libs:
+    for p in names:
         d = res[p]
         rec = {"lib": p, "config": a.config, "set": opts, "batch": a.batch,
                "step_ms_median": round(float(np.median(d["step_ms"])), 4),
@@ -104,7 +117,7 @@ def main():
     if a.out:
         with open(a.out, "a") as f:
             f.write("\n".join(lines) + "\n")
-    for G in Gs:
+    for G in Gs0:
         G.close()
 
 
