@@ -167,6 +167,9 @@ typedef struct dfs_options {
     int32_t steal_period;    /* walker kernel: an idle walker in a warp that still has busy walkers
                                 tries one Alg 3 steal every steal_period steps (power of two <= 1024;
                                 0 = 1)                                                             */
+    int32_t donate;          /* walker kernel: 1 (default) = a walker about to push an entry while a
+                                sibling walker of its warp holds nothing hands the entry to that
+                                sibling instead; 0 = always push                    */
 } dfs_options;
 
 typedef struct dfs_stats {
@@ -196,6 +199,7 @@ typedef struct dfs_stats {
     int64_t pops;            /* 32-wide step: entries popped after a list was exhausted            */
     int64_t dead_pops;       /* ... of which found nothing left to claim (every remaining target
                                 was claimed after the entry was pushed)                            */
+    int64_t donations;       /* walker kernel: entries handed to idle sibling walkers             */
 } dfs_stats;
 
 void dfs_options_default(dfs_options *opt);

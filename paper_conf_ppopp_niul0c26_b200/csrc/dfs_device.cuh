@@ -112,6 +112,7 @@ struct KParams {
     int bulk_copy;                           // flush/refill with cp.async.bulk (TMA ablation)
     uint32_t period_mask;                    // spill_period - 1
     uint32_t steal_period_mask;              // walker kernel: steal_period - 1
+    int donate;                              // walker kernel: hand pushed entries to idle siblings
 };
 
 // ------------------------------------------------------------------------------------------

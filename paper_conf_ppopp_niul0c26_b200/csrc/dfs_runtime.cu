@@ -216,6 +216,7 @@ void dfs_options_default(dfs_options* o) {
     o->leaf_skip = 2;            // A/B on B200: rmat22 5.20 -> 4.33 ms (bulk), others neutral
     o->steal_tries = 8;          // A/B on B200: road 16.8 -> 15.4 ms, grid -15%, others neutral
     o->bulk_copy = 1;            // A/B on B200: rmat24 -11%, caterpillar -18%, road -2%, path -1%
+    o->donate = 1;               // walker kernel: hand pushed entries to idle sibling walkers
 }
 
 int dfs_last_error(void) { return g_last_error; }
@@ -426,6 +427,7 @@ static int launch_one(dfs_graph* g, Slot& sl, cudaStream_t s, int32_t root, int3
     P.bulk_copy = o.bulk_copy;
     P.period_mask = (uint32_t)(o.spill_period > 0 ? o.spill_period : 32) - 1u;
     P.steal_period_mask = (uint32_t)(o.steal_period > 0 ? o.steal_period : 1) - 1u;
+    P.donate = o.donate;
     const bool tl = g->d_timeline && &sl == &g->slots[0];
     P.timeline = tl ? g->d_timeline : nullptr;
     P.timeline_len = tl ? (g->timeline_len / 3u) * 2u : 0;   // kernel: three regions of len/3
@@ -606,6 +608,7 @@ static void fill_stats(dfs_stats* stats, int blocks, int warps, float total_ms, 
     stats->cluster_steals = (int64_t)counters[kCntClusterSteals];
     stats->pops = (int64_t)counters[kCntPops];
     stats->dead_pops = (int64_t)counters[kCntDeadPops];
+    stats->donations = (int64_t)counters[kCntDonations];
 }
 
 // per-root count buffer (2 x u64 per root) for stats calls
@@ -651,7 +654,7 @@ static int run_sequential(dfs_graph* g, const int32_t* roots, int32_t k, int32_t
             return fail(DFS_ENOMEM);
         }
     }
-    unsigned long long counters[kNumCounters] = {0};
+    unsigned long long counters[kNumWCounters] = {0};
     float total_ms = 0.f, trav_ms = 0.f;
     int64_t nv = 0, mv = 0;
     cudaStream_t s = g->stream;
@@ -702,7 +705,7 @@ static int run_sequential(dfs_graph* g, const int32_t* roots, int32_t k, int32_t
             cudaEventElapsedTime(&kms, sl.evk0, sl.evk1);
             total_ms += ms;
             trav_ms += kms;
-            for (int c = 0; c < kNumCounters; ++c) counters[c] += h.counters[c];
+            for (int c = 0; c < kNumWCounters; ++c) counters[c] += h.counters[c];
         }
     }
     if (cudaStreamSynchronize(s) != cudaSuccess) { cudaGetLastError(); return fail(DFS_ECUDA); }
@@ -794,7 +797,7 @@ static int run_concurrent(dfs_graph* g, const int32_t* roots, int32_t k, int32_t
         if (rc != DFS_OK) return fail(rc);
         float ms = 0.f;
         cudaEventElapsedTime(&ms, s0.ev0, s0.evk1);
-        unsigned long long counters[kNumCounters] = {0};
+        unsigned long long counters[kNumWCounters] = {0};
         fill_stats(stats, blocks, warps, ms, ms, nv, mv, counters);
     }
     return DFS_OK;

@@ -25,6 +25,8 @@
 namespace b200dfs {
 
 constexpr int kMaxWalkersPerCta = 256;
+constexpr int kCntDonations = kNumCounters;         // walker kernel only (Ctl::counters has 24)
+constexpr int kNumWCounters = kNumCounters + 1;
 
 struct SmemW {
     uint32_t ht[kMaxWalkersPerCta];                 // HotRing (head << 16) | tail per walker
@@ -34,7 +36,7 @@ struct SmemW {
     volatile int done;
     uint32_t inter_token;                           // one Alg 4 scan per CTA at a time
     unsigned long long t_start;
-    unsigned long long cnt[kMaxWarps][kNumCounters];
+    unsigned long long cnt[kMaxWarps][kNumWCounters];
 };
 
 __device__ __forceinline__ uint32_t atom_add_relaxed_cta_if_ret(bool p, uint32_t* a, uint32_t v) {
@@ -98,7 +100,7 @@ __global__ void __launch_bounds__(1024, 1) dfs_walker_kernel(const KParams P) {
         S.t_start = globaltimer();
     }
     unsigned long long* const cnt = S.cnt[w];
-    if (STATS && lane < kNumCounters) cnt[lane] = 0;
+    if (STATS && lane < kNumWCounters) cnt[lane] = 0;
     __syncthreads();
 
     auto seg = [&](uint32_t b) -> uint32_t { return (b >> base) & GM; };
@@ -590,8 +592,35 @@ __global__ void __launch_bounds__(1024, 1) dfs_walker_kernel(const KParams P) {
                 else { exhausted = true; have_win = false; }
             }
             // push <u, ni> unless u is exhausted (positions whose probe saw a claimed target stay
-            // claimed, so skipping them keeps Alg 1's order), publish at once (CTA-scope release)
-            const bool do_push = descend && ni < end;
+            // claimed, so skipping them keeps Alg 1's order), publish at once (CTA-scope release).
+            // Donation (B200 addition): while a sibling walker of this warp holds
+            // nothing, the entry goes to that sibling as its top instead — a register move, no
+            // ring or atomic; <u, ni> is still scanned in order by exactly one walker.  The
+            // donor is registered, so the block count is >= 1 and the receiver's registration
+            // needs no global update.
+            bool do_push = descend && ni < end;
+            if (P.donate) {
+                const uint32_t pm = __ballot_sync(kFull, do_push && sl == 0);
+                const uint32_t im = __ballot_sync(kFull, !act && sl == 0);
+                if (pm && im) {
+                    const uint32_t below = (1u << base) - 1u;
+                    const int rp_ = __popc(pm & below), ri_ = __popc(im & below);
+                    const bool give = do_push && rp_ < __popc(im);
+                    const bool recv = !act && ri_ < __popc(pm);
+                    const int srcl = recv ? (int)__fns(pm, 0, ri_ + 1) : lane;
+                    const uint32_t du = __shfl_sync(kFull, u, srcl);
+                    const uint32_t dni = __shfl_sync(kFull, ni, srcl);
+                    const uint32_t dend = __shfl_sync(kFull, end, srcl);
+                    atom_add_relaxed_cta_if(recv && !active && sl == 0, &S.lbusy, 1u);
+                    count(kCntDonations, recv && sl == 0);
+                    if (recv) {
+                        has_top = true; active = true;
+                        u = du; i = dni; end = dend;
+                        have_win = false; need_end = false; spec_ok = spec_pop; par = kFull;
+                    }
+                    if (give) do_push = false;
+                }
+            }
             st_shared_u64_if(do_push && sl == 0, ring + (my_head & (H - 1)), pack_entry(u, ni));
             atom_add_release_cta_if(do_push && sl == 0, &S.ht[bk], 0x10000u);
             if (do_push) { ++my_head; pub = my_head; }
@@ -644,9 +673,11 @@ __global__ void __launch_bounds__(1024, 1) dfs_walker_kernel(const KParams P) {
             }
             if (gotw) pop_if(((gotw >> lane) & 1u) != 0);
         }
-        // newly idle walkers leave the busy count
+        // newly idle walkers leave the busy count — only once their ColdSeg is empty (the refill
+        // above found nothing: cold_lo == my_top); a walker whose refilled entries were all
+        // stolen before its pop keeps its registration and refills again
         {
-            const bool dereg = !has_top && active;
+            const bool dereg = !has_top && active && my_top == cold_lo;
             if (dereg && sl == 0) deregister();
             if (dereg) active = false;
             __syncwarp();
@@ -666,7 +697,7 @@ __global__ void __launch_bounds__(1024, 1) dfs_walker_kernel(const KParams P) {
         {
             uint32_t backoff = P.backoff_min_ns;
             uint32_t idle_iter = 0;
-            int thief = 0;
+            uint32_t got = 0;                                 // walkers that got work
             for (;;) {
                 if (__shfl_sync(kFull, S.done, 0)) goto exit_loop;
                 if (w == 0 && __shfl_sync(kFull, (int)(*(volatile unsigned int*)&P.ctl->done), 0)) {
@@ -678,13 +709,17 @@ __global__ void __launch_bounds__(1024, 1) dfs_walker_kernel(const KParams P) {
                     if (lane == 0) { raise_error(P, kStatusETIMEOUT); S.done = 1; }
                     goto exit_loop;
                 }
-                if (P.intra && steal_intra(thief)) break;
-                if (P.inter && gridDim.x > 1 && steal_inter(thief)) break;
+                // every walker of the warp tries Alg 3, then Alg 4, until one finds no victim
+                for (int k = 0; k < WPW; ++k) {
+                    if (P.intra && steal_intra(k)) { got |= 1u << k; continue; }
+                    if (P.inter && gridDim.x > 1 && steal_inter(k)) { got |= 1u << k; continue; }
+                    break;
+                }
+                if (got) break;
                 __nanosleep(backoff);
                 if (backoff < P.backoff_max_ns) backoff <<= 1;
-                thief = (thief + 1) & (WPW - 1);
             }
-            pop_if(wk == thief);
+            pop_if(((got >> wk) & 1u) != 0);
         }
     }
 exit_loop:
@@ -702,7 +737,7 @@ exit_loop:
     if (P.block_claims && sl == 0 && my_claims) atomicAdd(&P.block_claims[blockIdx.x], (unsigned long long)my_claims);
     if (STATS && (P.collect_stats != 2 || gk == 0)) {
 #pragma unroll
-        for (int k = 0; k < kNumCounters; ++k)
+        for (int k = 0; k < kNumWCounters; ++k)
             if (lane == 0 && cnt[k]) atomicAdd(&P.ctl->counters[k], cnt[k]);
         __syncwarp();
     }

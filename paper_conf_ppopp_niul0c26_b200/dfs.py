@@ -54,7 +54,7 @@ class _Options(ctypes.Structure):
                 ("cluster_late", ctypes.c_int32), ("steal_tries", ctypes.c_int32),
                 ("bulk_copy", ctypes.c_int32), ("spill_period", ctypes.c_int32),
                 ("l2_persist_mb", ctypes.c_int32), ("walker_lanes", ctypes.c_int32),
-                ("steal_period", ctypes.c_int32)]
+                ("steal_period", ctypes.c_int32), ("donate", ctypes.c_int32)]
 
 
 class _Stats(ctypes.Structure):
@@ -71,7 +71,7 @@ class _Stats(ctypes.Structure):
                 ("cyc_claim", ctypes.c_int64), ("cyc_tail", ctypes.c_int64),
                 ("cyc_outside", ctypes.c_int64), ("root_counts", ctypes.c_void_p),
                 ("block_claims", ctypes.c_void_p), ("cluster_steals", ctypes.c_int64),
-                ("pops", ctypes.c_int64), ("dead_pops", ctypes.c_int64)]
+                ("pops", ctypes.c_int64), ("dead_pops", ctypes.c_int64), ("donations", ctypes.c_int64)]
 
 
 @dataclass
@@ -109,6 +109,7 @@ class Options:
     l2_persist_mb: Optional[int] = None
     walker_lanes: Optional[int] = None
     steal_period: Optional[int] = None
+    donate: Optional[bool] = None
 
     def to_c(self) -> _Options:
         o = _Options()
@@ -148,6 +149,7 @@ class Stats:
     cluster_steals: int = 0
     pops: int = 0
     dead_pops: int = 0
+    donations: int = 0
     root_counts: Optional[np.ndarray] = None
     block_claims: Optional[np.ndarray] = None
 
