@@ -682,7 +682,10 @@ __global__ void __launch_bounds__(1024, 1) dfs_walker_kernel(const KParams P) {
             if (dereg) active = false;
             __syncwarp();
         }
-        const uint32_t idle_mask = __ballot_sync(kFull, !has_top && sl == 0);
+        // idle = no top and deregistered (a walker whose ColdSeg may still hold entries stays
+        // registered and retries its refill on the next pass; it never steals: a thief
+        // registers before it reserves, so only deregistered walkers may steal)
+        const uint32_t idle_mask = __ballot_sync(kFull, !has_top && !active && sl == 0);
         if (idle_mask == 0) continue;
         if (idle_mask != __ballot_sync(kFull, sl == 0)) {
             // some walkers of this warp are busy: one Alg 3 attempt for the first idle walker
