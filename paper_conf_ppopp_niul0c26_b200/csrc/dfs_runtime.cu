@@ -177,7 +177,10 @@ static int ensure_slot(dfs_graph* g, int k, int64_t n_warps) {
         (k > 0 && cudaStreamCreateWithFlags(&s.stream, cudaStreamNonBlocking) != cudaSuccess)) {
         cudaGetLastError(); free_slot(s); return DFS_ECUDA;
     }
-    if (cudaMemset(s.tab, 0xFF, s.tab_words * sizeof(uint32_t)) != cudaSuccess) {   // all chunk slots empty
+    // all chunk slots empty; complete before any stream (the slot streams are non-blocking, so
+    // they do not wait for work on the legacy default stream) can launch on this slot
+    if (cudaMemset(s.tab, 0xFF, s.tab_words * sizeof(uint32_t)) != cudaSuccess ||
+        cudaDeviceSynchronize() != cudaSuccess) {
         cudaGetLastError(); free_slot(s); return DFS_ECUDA;
     }
     s.ready = true;
