@@ -346,7 +346,8 @@ __global__ void __launch_bounds__(1024, 1) dfs_walker_kernel(const KParams P) {
             const uint32_t k_head = __shfl_sync(kFull, my_head, k * G);
             const unsigned long long* vring = rings + (size_t)vj * H;
             unsigned long long* const kring = rings + (size_t)kb * H;
-            if (lane < (int)kst) kring[(k_head + lane) & (H - 1)] = vring[(t + lane) & (H - 1)];
+            for (uint32_t q = lane; q < kst; q += 32u)       // kst <= kStealMax (64 for G = 16)
+                kring[(k_head + q) & (H - 1)] = vring[(t + q) & (H - 1)];
             __syncwarp();
             if (lane == 0) {
                 S.tailf[vj] = (t + kst) & 0xFFFFu;           // slots reusable by the owner
