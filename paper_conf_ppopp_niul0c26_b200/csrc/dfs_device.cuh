@@ -113,7 +113,26 @@ struct KParams {
     uint32_t period_mask;                    // spill_period - 1
     uint32_t steal_period_mask;              // walker kernel: steal_period - 1
     int donate;                              // walker kernel: hand pushed entries to idle siblings
+    const uint32_t* __restrict__ rec;        // vertex records (8 words per vertex: col[rp[v] .. +6),
+                                             // rp[v], rp[v+1]; padding kFull), or null
 };
+
+// vertex records (create time, on first use): record v = 8 words = one 32-byte
+// sector: the first 6 entries of v's adjacency list (kFull past its end), then row_ptr[v] and
+// row_ptr[v+1].  A walker of >= 8 lanes loads a claimed child's record with one coalesced request,
+// so a list of <= 6 entries needs no dependent row_ptr -> col_idx round trip.
+__global__ void dfs_records_kernel(const uint32_t* __restrict__ rp, const int32_t* __restrict__ col, uint32_t n,
+                                   uint4* __restrict__ rec) {
+    const size_t stride = (size_t)gridDim.x * blockDim.x;
+    for (size_t v = blockIdx.x * (size_t)blockDim.x + threadIdx.x; v < n; v += stride) {
+        const uint32_t s = rp[v], e = rp[v + 1];
+        uint32_t w[6];
+#pragma unroll
+        for (int k = 0; k < 6; ++k) w[k] = s + k < e ? (uint32_t)col[s + k] : kFull;
+        rec[2 * v] = make_uint4(w[0], w[1], w[2], w[3]);
+        rec[2 * v + 1] = make_uint4(w[4], w[5], s, e);
+    }
+}
 
 // ------------------------------------------------------------------------------------------
 // small PTX helpers

@@ -56,17 +56,24 @@ const void* const* kernel_table() {
 #undef DFS_K
 constexpr int kNumKernels = 24;
 
-// sub-warp walker kernels (dfs_walker.cuh): [G = 16, 8, 4][stats]; HotRing H = 16 * G entries
-// per walker, so a 32-warp CTA holds 128 KB of rings for every G
-#define DFS_WK(G, S) (const void*)dfs_walker_kernel<G, 16 * G, S>
+// sub-warp walker kernels (dfs_walker.cuh): [G = 16, 8, 4][stats], then the vertex-record
+// variants [G = 16, 8][stats]; HotRing H = 16 * G entries per walker, so a 32-warp CTA holds
+// 128 KB of rings for every G
+#define DFS_WK(G, S, R) (const void*)dfs_walker_kernel<G, 16 * G, S, R>
 const void* const* walker_table() {
-    static const void* const t[6] = {DFS_WK(16, false), DFS_WK(16, true), DFS_WK(8, false), DFS_WK(8, true),
-                                     DFS_WK(4, false), DFS_WK(4, true)};
+    static const void* const t[10] = {DFS_WK(16, false, false), DFS_WK(16, true, false), DFS_WK(8, false, false),
+                                      DFS_WK(8, true, false), DFS_WK(4, false, false), DFS_WK(4, true, false),
+                                      DFS_WK(16, false, true), DFS_WK(16, true, true), DFS_WK(8, false, true),
+                                      DFS_WK(8, true, true)};
     return t;
 }
 #undef DFS_WK
-constexpr int kNumWalkerKernels = 6;
-int walker_index(int lanes) { return lanes == 16 ? 0 : lanes == 8 ? 2 : 4; }
+constexpr int kNumWalkerKernels = 10;
+int walker_lanes_of(int kf) { return (kf % 6) < 2 ? 16 : (kf % 6) < 4 ? 8 : 4; }
+int walker_index(int lanes, bool rec) {
+    if (rec && lanes >= 8) return lanes == 16 ? 6 : 8;
+    return lanes == 16 ? 0 : lanes == 8 ? 2 : 4;
+}
 
 size_t smem_bytes(int warps) {
     return ((sizeof(SmemCtl) + 15) & ~size_t(15)) + (size_t)warps * kRing * sizeof(unsigned long long);
@@ -115,6 +122,7 @@ struct dfs_graph {
     uint32_t* d_rp = nullptr;
     int32_t* d_col = nullptr;    // col_idx (+8 padding for 128-bit window loads)
     uint32_t* d_leaf = nullptr;  // leaf map: ceil(n/32) words (dfs_leaf_*_kernel)
+    uint32_t* d_rec = nullptr;   // vertex records: 8 words per vertex (built on first use)
     Slot slots[kMaxSlots];
     int64_t launches = 0;
     unsigned int* d_timeline = nullptr;   // diagnostics (dfs_debug_timeline)
@@ -140,7 +148,7 @@ static void free_graph(dfs_graph* g) {
     int cur = 0;
     cudaGetDevice(&cur);
     cudaSetDevice(g->device);
-    cudaFree(g->d_rp); cudaFree(g->d_col); cudaFree(g->d_leaf); cudaFree(g->d_timeline); cudaFree(g->d_counts);
+    cudaFree(g->d_rp); cudaFree(g->d_col); cudaFree(g->d_leaf); cudaFree(g->d_rec); cudaFree(g->d_timeline); cudaFree(g->d_counts);
     for (int k = 0; k < kMaxSlots; ++k) free_slot(g->slots[k]);
     cudaSetDevice(cur);
     delete g;
@@ -220,6 +228,7 @@ void dfs_options_default(dfs_options* o) {
     o->steal_tries = 8;          // A/B on B200: road 16.8 -> 15.4 ms, grid -15%, others neutral
     o->bulk_copy = 1;            // A/B on B200: rmat24 -11%, caterpillar -18%, road -2%, path -1%
     o->donate = 1;               // walker kernel: hand pushed entries to idle sibling walkers
+    o->records = 1;              // walker kernel (>= 8 lanes): vertex records
 }
 
 int dfs_last_error(void) { return g_last_error; }
@@ -257,7 +266,7 @@ dfs_graph* dfs_graph_create(const int64_t* row_ptr, const int32_t* col_idx, int6
             attr_ok = false;
     }
     for (int kf = 0; kf < kNumWalkerKernels; ++kf) {
-        const int lanes = kf < 2 ? 16 : kf < 4 ? 8 : 4;
+        const int lanes = walker_lanes_of(kf);
         if (cudaFuncSetAttribute(walker_table()[kf], cudaFuncAttributeMaxDynamicSharedMemorySize,
                                  (int)walker_smem_bytes(32, lanes)) != cudaSuccess)
             attr_ok = false;
@@ -440,7 +449,9 @@ static int launch_one(dfs_graph* g, Slot& sl, cudaStream_t s, int32_t root, int3
     void* args[] = {(void*)&P};
     const int cl = o.cluster > 1 ? o.cluster : 1;
     // the cluster build has no bulk variant: cluster >= 1 takes precedence over bulk_copy
-    const void* kfn = wl != 32 ? walker_table()[walker_index(wl) + (o.collect_stats ? 1 : 0)]
+    P.rec = g->d_rec;
+    const bool rec = wl != 32 && wl >= 8 && o.records && g->d_rec;
+    const void* kfn = wl != 32 ? walker_table()[walker_index(wl, rec) + (o.collect_stats ? 1 : 0)]
                                : kernel_table()[(o.cluster >= 1 ? 8 : o.bulk_copy ? 16 : 0) + (o.window == 128 ? 4 : 0) +
                                                 (warps <= 16 ? 2 : 0) + (o.collect_stats ? 1 : 0)];
     if (timed) cudaEventRecord(sl.evk0, s);
@@ -530,6 +541,14 @@ static int resolve_options(dfs_graph* g, const dfs_options* in, int num_roots, d
     if (o.walker_lanes == 0) o.walker_lanes = 32;
     if (o.deterministic || o.cluster >= 1 || (o.window == 128 && !window_auto)) o.walker_lanes = 32;
     if (o.walker_lanes != 32) o.window = 32;
+    if (o.records && o.walker_lanes != 32 && o.walker_lanes >= 8 && !g->d_rec) {
+        // vertex records (8 words per vertex), built once per handle on first use
+        if (cudaMalloc(&g->d_rec, (size_t)g->n * 32) != cudaSuccess) { cudaGetLastError(); g->d_rec = nullptr; return DFS_ENOMEM; }
+        const int blocks_r = (int)std::min<int64_t>((g->n + 255) / 256, (int64_t)g->sms * 16);
+        dfs_records_kernel<<<blocks_r, 256>>>(g->d_rp, g->d_col, (uint32_t)g->n, reinterpret_cast<uint4*>(g->d_rec));
+        g->launches++;
+        if (cudaDeviceSynchronize() != cudaSuccess) { cudaGetLastError(); cudaFree(g->d_rec); g->d_rec = nullptr; return DFS_ECUDA; }
+    }
     if (o.window != 32 && o.window != 128) return DFS_EINVAL;
     if (o.concurrency < 0 || o.concurrency > kMaxSlots) return DFS_EINVAL;
     warps = o.warps_per_block <= 0 ? 32 : o.warps_per_block;

@@ -63,9 +63,10 @@ __device__ __forceinline__ unsigned long long ld_shared_u64_if(bool p, const uns
 // Stack owners are walkers: cold_tb / chunk_tab are indexed by the global walker id
 // blockIdx.x * (W * 32 / G) + warp * (32 / G) + walker.
 // ------------------------------------------------------------------------------------------
-template <int G, int H, bool STATS>
+template <int G, int H, bool STATS, bool REC>
 __global__ void __launch_bounds__(1024, 1) dfs_walker_kernel(const KParams P) {
     static_assert(G == 4 || G == 8 || G == 16, "G is 4, 8 or 16");
+    static_assert(!REC || G >= 8, "a vertex record spans 8 lanes");
     static_assert((H & (H - 1)) == 0 && H >= 32 && H <= 1024, "H is a power of two in [32, 1024]");
     constexpr int WPW = 32 / G;                       // walkers per warp
     constexpr uint32_t GM = (1u << G) - 1u;
@@ -520,13 +521,25 @@ __global__ void __launch_bounds__(1024, 1) dfs_walker_kernel(const KParams P) {
             const uint32_t svx = (uint32_t)__shfl_sync(kFull, nb, sk & (G - 1), G);
             const uint32_t sv = vbs ? svx : u;
             uint32_t s_old = atom_or_if(vbs != 0 && sl == 0, P.bitmap + 2u * (sv >> 5), 1u << (sv & 31));
-            const uint32_t s_rs = ld_nc_if(vbs != 0, P.rp + sv, 0u), s_re = ld_nc_if(vbs != 0, P.rp + sv + 1, 0u);
-            // probes of the visited bits ({visited, leaf} pair: one 8-byte L2 load); the first
-            // kPf lanes also load their candidates' row_ptr pairs
+            // the claimed child's list: with vertex records (REC) one 32-byte load gives its
+            // first 6 neighbours and its row_ptr pair — no dependent col load for
+            // lists of <= 6 entries; else the row_ptr pair, then the window
+            uint32_t s_rs, s_re;
+            int cnb;
+            if constexpr (REC) {
+                const uint32_t rw = ld_nc_if(vbs != 0 && sl < 8, P.rec + 8u * sv + sl, kFull);
+                s_rs = __shfl_sync(kFull, rw, 6, G); s_re = __shfl_sync(kFull, rw, 7, G);
+                const int cx = (int)ld_nc_if(vbs != 0 && sl >= 6 && s_rs + sl < s_re, P.col + s_rs + sl, kFull);
+                cnb = sl < 6 ? (int)rw : cx;
+            } else {
+                s_rs = ld_nc_if(vbs != 0, P.rp + sv, 0u); s_re = ld_nc_if(vbs != 0, P.rp + sv + 1, 0u);
+            }
+            // probes of the visited bits ({visited, leaf} pair: one 8-byte L2 load); without
+            // records the first kPf lanes also load their candidates' row_ptr pairs
             const uint2 wl = ld_cg_u2_if(valid, P.bitmap + 2u * ((uint32_t)nb >> 5), kFull, 0u);
-            const bool pf = valid && sl < kPf;
+            const bool pf = !REC && valid && sl < kPf;
             const uint32_t prs = ld_nc_if(pf, P.rp + nb, 0u), pre = ld_nc_if(pf, P.rp + nb + 1, 0u);
-            int cnb = (int)ld_nc_if(spec_early && vbs != 0 && s_rs + sl < s_re, P.col + s_rs + sl, kFull);
+            if constexpr (!REC) cnb = (int)ld_nc_if(spec_early && vbs != 0 && s_rs + sl < s_re, P.col + s_rs + sl, kFull);
             const bool unv = valid && !((wl.x >> (nb & 31)) & 1u) && sl != sk;   // sk is claimed either way
             const bool lf = unv && ((wl.y >> (nb & 31)) & 1u);
             bool cand = unv && !lf;
@@ -543,7 +556,7 @@ __global__ void __launch_bounds__(1024, 1) dfs_walker_kernel(const KParams P) {
             count(kCntFailedClaims, vbs != 0 && !won && sl == 0);
             uint32_t v = sv, vrs = s_rs, vre = s_re;
             int kpos = sk;
-            if (!spec_early) cnb = (int)ld_nc_if(won && vrs + sl < vre, P.col + vrs + sl, kFull);
+            if (!REC && !spec_early) cnb = (int)ld_nc_if(won && vrs + sl < vre, P.col + vrs + sl, kFull);
             // claim the first unvisited candidate in CSR order; on a lost race try the next (all
             // walkers that still search advance together)
             bool need = act && !won;
@@ -553,12 +566,22 @@ __global__ void __launch_bounds__(1024, 1) dfs_walker_kernel(const KParams P) {
                 if (!__any_sync(kFull, tr)) break;
                 const int k = anyc ? __ffs(anyc) - 1 : 0;
                 const uint32_t cv = (uint32_t)__shfl_sync(kFull, nb, k, G);
-                uint32_t crs = __shfl_sync(kFull, prs, k & (kPf - 1), G), cre = __shfl_sync(kFull, pre, k & (kPf - 1), G);
-                crs = ld_nc_if(tr && k >= kPf, P.rp + cv, crs);
-                cre = ld_nc_if(tr && k >= kPf, P.rp + cv + 1, cre);
                 const uint32_t bit = 1u << (cv & 31);
-                uint32_t old = atom_or_if(tr && sl == 0, P.bitmap + 2u * (cv >> 5), bit);
-                const int cw = (int)ld_nc_if(tr && crs + sl < cre, P.col + crs + sl, kFull);   // overlaps the claim
+                uint32_t crs, cre, old;
+                int cw;
+                if constexpr (REC) {                         // the record load overlaps the claim
+                    old = atom_or_if(tr && sl == 0, P.bitmap + 2u * (cv >> 5), bit);
+                    const uint32_t rw = ld_nc_if(tr && sl < 8, P.rec + 8u * cv + sl, kFull);
+                    crs = __shfl_sync(kFull, rw, 6, G); cre = __shfl_sync(kFull, rw, 7, G);
+                    const int cx = (int)ld_nc_if(tr && sl >= 6 && crs + sl < cre, P.col + crs + sl, kFull);
+                    cw = sl < 6 ? (int)rw : cx;
+                } else {
+                    crs = __shfl_sync(kFull, prs, k & (kPf - 1), G); cre = __shfl_sync(kFull, pre, k & (kPf - 1), G);
+                    crs = ld_nc_if(tr && k >= kPf, P.rp + cv, crs);
+                    cre = ld_nc_if(tr && k >= kPf, P.rp + cv + 1, cre);
+                    old = atom_or_if(tr && sl == 0, P.bitmap + 2u * (cv >> 5), bit);
+                    cw = (int)ld_nc_if(tr && crs + sl < cre, P.col + crs + sl, kFull);   // overlaps the claim
+                }
                 old = __shfl_sync(kFull, old, 0, G);
                 const bool ok = tr && !(old & bit);
                 if (ok) { won = true; v = cv; vrs = crs; vre = cre; kpos = k; cnb = cw; need = false; }

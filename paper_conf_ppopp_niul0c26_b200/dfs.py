@@ -54,7 +54,8 @@ class _Options(ctypes.Structure):
                 ("cluster_late", ctypes.c_int32), ("steal_tries", ctypes.c_int32),
                 ("bulk_copy", ctypes.c_int32), ("spill_period", ctypes.c_int32),
                 ("l2_persist_mb", ctypes.c_int32), ("walker_lanes", ctypes.c_int32),
-                ("steal_period", ctypes.c_int32), ("donate", ctypes.c_int32)]
+                ("steal_period", ctypes.c_int32), ("donate", ctypes.c_int32),
+                ("records", ctypes.c_int32)]
 
 
 class _Stats(ctypes.Structure):
@@ -110,6 +111,7 @@ class Options:
     walker_lanes: Optional[int] = None
     steal_period: Optional[int] = None
     donate: Optional[bool] = None
+    records: Optional[bool] = None
 
     def to_c(self) -> _Options:
         o = _Options()

@@ -75,6 +75,7 @@ def test_walker_tree_inputs_bit_exact(lanes, name, build, roots):
     dict(inter_steal=False), dict(intra_steal=False), dict(blocks=3, warps_per_block=2),
     dict(blocks=1), dict(warps_per_block=1, blocks=5), dict(victim_policy=0), dict(speculate=0),
     dict(speculate=1), dict(leaf_skip=0), dict(leaf_skip=1), dict(pub_batch=4), dict(spill_period=1),
+    dict(records=0), dict(records=0, ring_cap=3), dict(donate=0), dict(donate=0, steal_period=1024),
 ])
 def test_walker_stress(lanes, opts):
     g = graphgen.road(300, 200, seed=7)
@@ -98,6 +99,18 @@ def test_walker_counters_and_steals(lanes):
         p, st = G.run(0, options=Options(walker_lanes=lanes, collect_stats=True, inter_steal=False), stats=True)
         _valid(g, 0, p)
         assert st.inter_steals == 0 and st.intra_steals > 0
+
+
+@pytest.mark.parametrize("lanes", LANES)
+@pytest.mark.parametrize("records", [0, 1])
+def test_walker_records_directed_long_lists(lanes, records):
+    """Vertex records hold the first 6 neighbours: lists of 0..40 entries (directed, self loops,
+    duplicates, unsorted) take both the record path and the col_idx path of the same list."""
+    g = graphgen.shuffle_lists(graphgen.random_graph(20_000, 200_000, seed=12, symmetric=False,
+                                                     allow_self=True, allow_dup=True), 4)
+    with Graph(g.row_ptr, g.col_idx) as G:
+        for r in (0, 999):
+            _valid(g, r, G.run(r, options=Options(walker_lanes=lanes, records=records)), undirected=False)
 
 
 @pytest.mark.parametrize("lanes", LANES)
