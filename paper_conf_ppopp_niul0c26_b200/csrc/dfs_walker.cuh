@@ -301,13 +301,40 @@ __global__ void __launch_bounds__(1024, 1) dfs_walker_kernel(const KParams P) {
         return take;
     };
 
-    // Alg 3 for thief walker k: the walker of this CTA with max hot_rest >= hot_cutoff (siblings
-    // in this warp included); reserve from its tail under its lock, copy SMEM -> SMEM
-    auto steal_intra = [&](int k) -> bool {
-        const int kb = w * WPW + k;
+    // deliver kst stolen entries to the thief walkers tb (bit k = walker k of this warp; all idle,
+    // deregistered, with empty rings): entry q (oldest first) goes to the (q mod nt)-th thief, so
+    // one steal can feed every idle walker of the warp.  Each receiver publishes its entries
+    // (CTA-scope release) and becomes active; the thief registration made before the reservation
+    // counts the first receiver, the others are added to the block count (>= 1, no global update).
+    // Returns the receivers.
+    auto deliver = [&](uint32_t tb, uint32_t kst, auto&& load_entry) -> uint32_t {
+        const int nt = __popc(tb);
+        for (uint32_t it = 0; it < (kst + 31u) / 32u; ++it) {
+            const uint32_t q = lane + 32u * it;
+            const int tw = (int)__fns(tb, 0, (int)(q % (uint32_t)nt) + 1);
+            const uint32_t th = __shfl_sync(kFull, my_head, (tw & (WPW - 1)) * G);
+            if (q < kst) rings[(size_t)(w * WPW + tw) * H + ((th + q / (uint32_t)nt) & (H - 1))] = load_entry(q);
+        }
+        __syncwarp();
+        const int rank = __popc(tb & ((1u << wk) - 1u));
+        const uint32_t cntw = (((tb >> wk) & 1u) && kst > (uint32_t)rank) ? (kst - (uint32_t)rank + (uint32_t)nt - 1u) / (uint32_t)nt : 0u;
+        atom_add_release_cta_if(cntw != 0 && sl == 0, &S.ht[bk], cntw << 16);
+        const uint32_t nr = kst < (uint32_t)nt ? kst : (uint32_t)nt;
+        if (lane == 0 && nr > 1) atomicAdd(&S.lbusy, nr - 1);
+        if (cntw) { my_head += cntw; pub = my_head; active = true; }
+        __syncwarp();
+        uint32_t got = 0;
+#pragma unroll
+        for (int k = 0; k < WPW; ++k) got |= (__ballot_sync(kFull, cntw != 0) >> (k * G) & 1u) << k;
+        return got;
+    };
+
+    // Alg 3 for the thief walkers tb: the walker of this CTA with max hot_rest >= hot_cutoff
+    // (siblings in this warp included); reserve from its tail under its lock, copy SMEM -> SMEM
+    auto steal_intra = [&](uint32_t tb) -> uint32_t {
         int best = -1, bidx = -1;
         for (int j = lane; j < NWB; j += 32) {
-            if (j == kb) continue;
+            if (j / WPW == w && ((tb >> (j % WPW)) & 1u)) continue;   // a thief itself
             const int r = ht_rest(*(volatile uint32_t*)&S.ht[j]);
             if (r > best) { best = r; bidx = j; }
         }
@@ -344,33 +371,27 @@ __global__ void __launch_bounds__(1024, 1) dfs_walker_kernel(const KParams P) {
             t = __shfl_sync(kFull, t, 0);
             kst = __shfl_sync(kFull, kst, 0);
             __syncwarp();                                    // lane 0's acquire -> all lanes
-            const uint32_t k_head = __shfl_sync(kFull, my_head, k * G);
             const unsigned long long* vring = rings + (size_t)vj * H;
-            unsigned long long* const kring = rings + (size_t)kb * H;
-            for (uint32_t q = lane; q < kst; q += 32u)       // kst <= kStealMax (64 for G = 16)
-                kring[(k_head + q) & (H - 1)] = vring[(t + q) & (H - 1)];
-            __syncwarp();
+            const uint32_t got = deliver(tb, kst, [&](uint32_t q) { return vring[(t + q) & (H - 1)]; });
             if (lane == 0) {
                 S.tailf[vj] = (t + kst) & 0xFFFFu;           // slots reusable by the owner
                 smem_unlock(&S.lock[vj]);
-                atom_add_release_cta(&S.ht[kb], kst << 16);  // publish into the thief's ring
             }
             __syncwarp();
-            if (wk == k) { my_head = k_head + kst; pub = my_head; active = true; }
             if (STATS && lane == 0) ++cnt[kCntIntraSteals];
-            return true;
+            return got;
         }
-        return false;
+        return 0u;
     };
 
-    // Alg 4 for thief walker k: two-choice victim block by cumulative ColdSeg load (reading
+    // Alg 4 for the thief walkers tb: two-choice victim block by cumulative ColdSeg load (reading
     // S14/S15), the walker with max cold_rest >= cold_cutoff, c_s entries from its ColdSeg bottom
-    auto steal_inter = [&](int k) -> bool {
+    auto steal_inter = [&](uint32_t tb) -> uint32_t {
         int token = 0;
         if (lane == 0) token = (*(volatile uint32_t*)&S.inter_token == 0u && smem_trylock(&S.inter_token)) ? 1 : 0;
         token = __shfl_sync(kFull, token, 0);
-        if (!token) return false;
-        bool got_work = false;
+        if (!token) return 0u;
+        uint32_t got_work = 0;
         const int nB = gridDim.x;
         int vb = -1;
         {
@@ -443,18 +464,13 @@ __global__ void __launch_bounds__(1024, 1) dfs_walker_kernel(const KParams P) {
                     bot = __shfl_sync(kFull, bot, 0);
                     kst = __shfl_sync(kFull, kst, 0);
                     __syncwarp();
-                    const int kb = w * WPW + k;
-                    unsigned long long* const kring = rings + (size_t)kb * H;
-                    const uint32_t k_head = __shfl_sync(kFull, my_head, k * G);
                     uint32_t* vtab = P.chunk_tab + ((size_t)vg << P.tab_log2);
-                    for (uint32_t q = lane; q < kst; q += 32u) {
+                    got_work = deliver(tb, kst, [&](uint32_t q) {
                         const uint32_t p = bot + q;
                         const uint32_t c = ld_relaxed_u32(&vtab[(p >> kChunkLog2) & tmask]);
-                        kring[(k_head + q) & (H - 1)] = c < P.n_chunks
-                            ? ld_cg_u64(P.pool + ((size_t)c << kChunkLog2) + (p & (kChunk - 1)))
-                            : pack_entry((uint32_t)P.root, P.m);   // owner exited on an error
-                    }
-                    __syncwarp();
+                        return c < P.n_chunks ? ld_cg_u64(P.pool + ((size_t)c << kChunkLog2) + (p & (kChunk - 1)))
+                                              : pack_entry((uint32_t)P.root, P.m);   // owner exited on an error
+                    });
                     if (lane == 0) {
                         uint32_t p = bot, left = kst;
                         while (left) {                       // chunk accounting (see the warp kernel)
@@ -469,12 +485,9 @@ __global__ void __launch_bounds__(1024, 1) dfs_walker_kernel(const KParams P) {
                             p += part; left -= part;
                         }
                         atomicSub(&P.block_cold[vb], (int)kst);
-                        atom_add_release_cta(&S.ht[kb], kst << 16);   // publish into the thief's ring
                     }
                     __syncwarp();
-                    if (wk == k) { my_head = k_head + kst; pub = my_head; active = true; }
                     if (STATS && lane == 0) ++cnt[kCntInterSteals];
-                    got_work = true;
                 }
             }
         }
@@ -711,12 +724,15 @@ __global__ void __launch_bounds__(1024, 1) dfs_walker_kernel(const KParams P) {
         // registers before it reserves, so only deregistered walkers may steal)
         const uint32_t idle_mask = __ballot_sync(kFull, !has_top && !active && sl == 0);
         if (idle_mask == 0) continue;
-        if (idle_mask != __ballot_sync(kFull, sl == 0)) {
-            // some walkers of this warp are busy: one Alg 3 attempt for the first idle walker
-            // every steal_period steps (the busy walkers wait for it)
+        uint32_t idle_w = 0;                                  // idle walkers, bit k = walker k
+#pragma unroll
+        for (int k = 0; k < WPW; ++k) idle_w |= ((idle_mask >> (k * G)) & 1u) << k;
+        if (idle_w != (1u << WPW) - 1u) {
+            // some walkers of this warp are busy: one Alg 3 steal for all idle walkers every
+            // steal_period steps (the busy walkers wait for it)
             if ((iter & P.steal_period_mask) == 0 && P.intra) {
-                const int k = (__ffs(idle_mask) - 1) / G;
-                if (steal_intra(k)) pop_if(wk == k);
+                const uint32_t got = steal_intra(idle_w);
+                if (got) pop_if(((got >> wk) & 1u) != 0);
             }
             continue;
         }
@@ -736,12 +752,9 @@ __global__ void __launch_bounds__(1024, 1) dfs_walker_kernel(const KParams P) {
                     if (lane == 0) { raise_error(P, kStatusETIMEOUT); S.done = 1; }
                     goto exit_loop;
                 }
-                // every walker of the warp tries Alg 3, then Alg 4, until one finds no victim
-                for (int k = 0; k < WPW; ++k) {
-                    if (P.intra && steal_intra(k)) { got |= 1u << k; continue; }
-                    if (P.inter && gridDim.x > 1 && steal_inter(k)) { got |= 1u << k; continue; }
-                    break;
-                }
+                // one steal for all walkers of the warp: Alg 3, else Alg 4
+                if (P.intra) got = steal_intra(idle_w);
+                if (!got && P.inter && gridDim.x > 1) got = steal_inter(idle_w);
                 if (got) break;
                 __nanosleep(backoff);
                 if (backoff < P.backoff_max_ns) backoff <<= 1;
