@@ -162,11 +162,14 @@ typedef struct dfs_options {
     int32_t walker_lanes;    /* lanes per walker: 32 = the warp kernel (one walker per warp, windows of
                                 `window` positions); 16, 8 or 4 = the sub-warp walker kernel (32/L
                                 independent walkers per warp, each with its own HotRing/ColdSeg and
-                                an L-position window); 0 = auto.
-                                deterministic, cluster >= 1 and window = 128 use the warp kernel   */
+                                an L-position window); 0 = auto: 4-lane walkers on
+                                low-degree graphs (m <= 4n, max degree <= 16) for batches with
+                                several traversals in flight and for path-like graphs (m < 2.2n),
+                                else the warp kernel.  deterministic, cluster >= 1 and window = 128
+                                use the warp kernel                                                */
     int32_t steal_period;    /* walker kernel: an idle walker in a warp that still has busy walkers
-                                tries one Alg 3 steal every steal_period steps (power of two <= 1024;
-                                0 = 1)                                                             */
+                                tries one Alg 3 steal (for all idle walkers of the warp) every
+                                steal_period steps (power of two <= 1024; 0 = 16)                  */
     int32_t donate;          /* walker kernel: 1 (default) = a walker about to push an entry while a
                                 sibling walker of its warp holds nothing hands the entry to that
                                 sibling instead; 0 = always push                    */
@@ -247,6 +250,20 @@ int64_t dfs_launch_count(const dfs_graph *g);
  * warps report every period); calling it again with the same len and a host buffer `out` copies the
  * last run's samples out and clears them; len = 0 disables. */
 int dfs_debug_timeline(dfs_graph *g, uint32_t len, uint32_t dt_ns, uint32_t *out);
+
+/* Diagnostics / tests: run a script of stack operations on the walkers of warp 0, block 0 of the
+ * sub-warp walker kernel (lanes = 16, 8 or 4 lanes per walker), using the kernel's own HotRing,
+ * ColdSeg and steal code (the paper's worked examples, Figs 2 and 3, are replayed this
+ * way by tests/test_gpu_stack_script.py).  script: n_ops records of 6 int32 {op, a, b, c, d, e}:
+ *   0 END; 1 SET w head tail top bottom (maps ColdSeg chunks for [0, top)); 2 RING w counter v i;
+ *   3 COLD w pos v i; 4 PUSH w v i; 5 POP w -> (v, i) or (-1, -1); 6 FLUSH w want keep;
+ *   7 REFILL w -> entries moved; 8 STEAL_INTRA thief-walker-mask -> receivers mask;
+ *   9 STEAL_INTER thief-walker-mask -> receivers mask; 10 DUMP w -> head tail top bottom;
+ *   11 READ_RING w counter -> (v, i); 12 READ_COLD w pos -> (v, i).
+ * Outputs are appended to out[0 .. out_len) (host memory).  opt supplies cutoffs, steal_half,
+ * ring_cap, ...; the handle's scratch is re-initialised before its next traversal. */
+int dfs_debug_stack_script(dfs_graph *g, int32_t lanes, const int32_t *script, int32_t n_ops,
+                           int32_t *out, int32_t out_len, const dfs_options *opt);
 
 void dfs_graph_destroy(dfs_graph *g);
 

@@ -115,6 +115,10 @@ struct KParams {
     int donate;                              // walker kernel: hand pushed entries to idle siblings
     const uint32_t* __restrict__ rec;        // vertex records (8 words per vertex: col[rp[v] .. +6),
                                              // rp[v], rp[v+1]; padding kFull), or null
+    const int32_t* script;                   // walker STATS kernel: stack-script mode (tests), or null
+    int script_len;
+    int32_t* script_out;
+    int script_out_len;
 };
 
 // vertex records (create time, on first use): record v = 8 words = one 32-byte
@@ -1659,16 +1663,24 @@ __global__ void dfs_leaf_init_kernel(const uint32_t* __restrict__ rp, const int3
 // CSR validation + narrowing of row_ptr to uint32 (step a1)
 __global__ void dfs_validate_rowptr_kernel(const int64_t* __restrict__ rp64, uint32_t* rp32, int64_t n,
                                            int64_t m, int* bad) {
+    // bad[0]: malformed flag; bad[1]: maximum out-degree (kernel selection)
     const size_t stride = (size_t)gridDim.x * blockDim.x;
+    int64_t dmax = 0;
     for (size_t v = blockIdx.x * (size_t)blockDim.x + threadIdx.x; v <= (size_t)n; v += stride) {
         const int64_t a = rp64[v];
         bool ok = a >= 0 && a <= m;
         if (v == 0) ok = ok && a == 0;
         if (v == (size_t)n) ok = ok && a == m;
-        if (v < (size_t)n) ok = ok && rp64[v + 1] >= a;
+        if (v < (size_t)n) {
+            const int64_t e = rp64[v + 1];
+            ok = ok && e >= a;
+            if (e - a > dmax) dmax = e - a;
+        }
         if (!ok) atomicExch(bad, 1);
         rp32[v] = (uint32_t)a;
     }
+    const int dm = __reduce_max_sync(kFull, (int)(dmax < 0x7FFFFFFF ? dmax : 0x7FFFFFFF));
+    if ((threadIdx.x & 31) == 0 && dm > 0) atomicMax(bad + 1, dm);
 }
 
 __global__ void dfs_validate_col_kernel(const int32_t* __restrict__ col, int64_t m, int64_t n, int* bad) {

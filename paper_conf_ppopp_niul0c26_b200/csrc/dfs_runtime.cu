@@ -112,6 +112,7 @@ struct dfs_graph {
     int device = 0;
     cudaStream_t stream = nullptr;
     int64_t n = 0, m = 0;
+    int64_t max_degree = 0;      // maximum out-degree (kernel selection)
     int sms = 0;
     int max_blocks = 0;          // co-resident 32-warp blocks (allocation bound)
     int max_clusters[4] = {0, 0, 0, 0};   // co-resident clusters of 1/2/4/8 CTAs (lazy)
@@ -297,13 +298,13 @@ dfs_graph* dfs_graph_create(const int64_t* row_ptr, const int32_t* col_idx, int6
     int* d_bad = nullptr;
     int64_t* d_rp64 = nullptr;                 // staging copy of a host row_ptr
     const bool rp_dev = is_device_ptr(row_ptr);
-    bool ok = cudaMalloc(&d_bad, sizeof(int)) == cudaSuccess &&
+    bool ok = cudaMalloc(&d_bad, 2 * sizeof(int)) == cudaSuccess &&
               (rp_dev || cudaMalloc(&d_rp64, (size_t)(n + 1) * sizeof(int64_t)) == cudaSuccess);
     if (!ok) {
         cudaGetLastError(); cudaFree(d_bad); cudaFree(d_rp64);
         free_graph(g); fail(DFS_ENOMEM); return nullptr;
     }
-    cudaMemset(d_bad, 0, sizeof(int));
+    cudaMemset(d_bad, 0, 2 * sizeof(int));
     const int64_t* rp_src = row_ptr;
     if (!rp_dev) {
         cudaMemcpy(d_rp64, row_ptr, (size_t)(n + 1) * sizeof(int64_t), cudaMemcpyHostToDevice);
@@ -320,8 +321,10 @@ dfs_graph* dfs_graph_create(const int64_t* row_ptr, const int32_t* col_idx, int6
         dfs_validate_col_kernel<<<blocks, 256>>>(g->d_col, m, n, d_bad);
         g->launches++;
     }
-    int hbad = 0;
-    cudaMemcpy(&hbad, d_bad, sizeof(int), cudaMemcpyDeviceToHost);
+    int hbad2[2] = {0, 0};
+    cudaMemcpy(hbad2, d_bad, 2 * sizeof(int), cudaMemcpyDeviceToHost);
+    const int hbad = hbad2[0];
+    g->max_degree = hbad2[1];
     cudaFree(d_bad);
     cudaFree(d_rp64);
     if (cudaGetLastError() != cudaSuccess) { free_graph(g); fail(DFS_ECUDA); return nullptr; }
@@ -395,8 +398,17 @@ int dfs_debug_timeline(dfs_graph* g, uint32_t len, uint32_t dt_ns, uint32_t* out
 // ------------------------------------------------------------------------------------------
 // one traversal on slot `sl`, stream-ordered on `s` (no synchronisation)
 // ------------------------------------------------------------------------------------------
+// stack-script mode of the walker STATS kernel (dfs_debug_stack_script)
+struct ScriptArgs {
+    const int32_t* d_script = nullptr;
+    int n_ops = 0;
+    int32_t* d_out = nullptr;
+    int out_len = 0;
+};
+
 static int launch_one(dfs_graph* g, Slot& sl, cudaStream_t s, int32_t root, int32_t* d_out,
-                      const dfs_options& o, int blocks, int warps, bool timed, bool cooperative) {
+                      const dfs_options& o, int blocks, int warps, bool timed, bool cooperative,
+                      const ScriptArgs* script = nullptr) {
     const uint32_t nwords = (uint32_t)((g->n + 31) / 32);
     const int rblocks = (int)std::min<int64_t>((std::max<int64_t>(nwords, sl.tab_dirty ? (int64_t)sl.tab_words : 0) + 255) / 256 + 1,
                                                (int64_t)g->sms * 8);
@@ -412,7 +424,7 @@ static int launch_one(dfs_graph* g, Slot& sl, cudaStream_t s, int32_t root, int3
     g->launches++;
     sl.tab_dirty = false;
 
-    KParams P;
+    KParams P = {};
     P.rp = g->d_rp; P.col = g->d_col; P.bitmap = sl.bitmap; P.parent = d_out;
     P.cold_tb = sl.cold_tb; P.chunk_tab = sl.tab; P.pool = sl.pool;
     P.chunk_consumed = sl.consumed; P.chunk_next = sl.next; P.block_cold = sl.block_cold;
@@ -446,6 +458,10 @@ static int launch_one(dfs_graph* g, Slot& sl, cudaStream_t s, int32_t root, int3
     P.timeline_dt_ns = tl ? g->timeline_dt_ns : 1;
     P.timeout_ns = (unsigned long long)o.timeout_ms * 1000000ull;
     P.seed = o.seed;
+    if (script) {
+        P.script = script->d_script; P.script_len = script->n_ops;
+        P.script_out = script->d_out; P.script_out_len = script->out_len;
+    }
     void* args[] = {(void*)&P};
     const int cl = o.cluster > 1 ? o.cluster : 1;
     // the cluster build has no bulk variant: cluster >= 1 takes precedence over bulk_copy
@@ -537,8 +553,18 @@ static int resolve_options(dfs_graph* g, const dfs_options* in, int num_roots, d
     if (o.steal_period < 0 || o.steal_period > 1024 || (o.steal_period & (o.steal_period - 1))) return DFS_EINVAL;
     const bool window_auto = o.window == 0;
     if (o.window == 0) o.window = (g->n > 0 && g->m >= 8 * g->n) ? 128 : 32;   // wide windows for dense lists
-    // kernel: the warp kernel (one walker per warp) or sub-warp walkers; auto = warp kernel
-    if (o.walker_lanes == 0) o.walker_lanes = 32;
+    // kernel (auto, measured on B200 — DESIGN.md §5): sub-warp walkers of 4 lanes where work is
+    // plentiful on low-degree graphs — batches (several traversals in flight) and path-like
+    // graphs (avg degree < 2.2: long unbranched runs, so every steal carries a long path); the
+    // warp kernel otherwise (road single roots: small stolen subtrees, walkers 1.5x slower;
+    // long lists / hubs: a 4-lane window needs 8x the steps of the 32-wide one)
+    if (o.walker_lanes == 0) {
+        const bool low_degree = g->m <= 4 * g->n && g->max_degree <= 16;
+        const bool batch = num_roots > 1 && o.concurrency != 1;
+        const bool pathlike = 10 * g->m < 22 * g->n;
+        o.walker_lanes = (low_degree && (batch || pathlike)) ? 4 : 32;
+    }
+    if (o.steal_period == 0) o.steal_period = 16;   // walker kernel (A/B on B200: batch -13%, road -27%)
     if (o.deterministic || o.cluster >= 1 || (o.window == 128 && !window_auto)) o.walker_lanes = 32;
     if (o.walker_lanes != 32) o.window = 32;
     if (o.records && o.walker_lanes != 32 && o.walker_lanes >= 8 && !g->d_rec) {
@@ -911,3 +937,48 @@ int dfs_run_batch(dfs_graph* g, const int32_t* roots, int32_t num_roots, int32_t
 }
 
 }  // extern "C"
+
+extern "C" int dfs_debug_stack_script(dfs_graph* g, int32_t lanes, const int32_t* script, int32_t n_ops,
+                                      int32_t* out, int32_t out_len, const dfs_options* opt) {
+    if (!g || !script || n_ops < 0 || (out_len > 0 && !out) || (lanes != 16 && lanes != 8 && lanes != 4))
+        return fail(DFS_EINVAL);
+    int rc = check_device(g);
+    if (rc != DFS_OK) return fail(rc);
+    dfs_options in;
+    dfs_options_default(&in);
+    if (opt) in = *opt;
+    in.walker_lanes = lanes; in.collect_stats = 1; in.deterministic = 0; in.cluster = 0; in.window = 0;
+    dfs_options o;
+    int blocks = 0, warps = 0, conc = 1;
+    rc = resolve_options(g, &in, 1, o, blocks, warps, conc);
+    if (rc != DFS_OK) return fail(rc);
+    Slot& sl = g->slots[0];
+    rc = ensure_slot(g, 0, std::max<int64_t>((int64_t)g->max_blocks * kMaxWarps, (int64_t)warps * (32 / lanes)));
+    if (rc != DFS_OK) return fail(rc);
+    if (!sl.parent && cudaMalloc(&sl.parent, (size_t)g->n * sizeof(int32_t)) != cudaSuccess) {
+        cudaGetLastError();
+        return fail(DFS_ENOMEM);
+    }
+    int32_t *d_script = nullptr, *d_out = nullptr;
+    if (cudaMalloc(&d_script, (size_t)n_ops * 6 * sizeof(int32_t) + 16) != cudaSuccess ||
+        cudaMalloc(&d_out, (size_t)out_len * sizeof(int32_t) + 16) != cudaSuccess) {
+        cudaGetLastError(); cudaFree(d_script); cudaFree(d_out);
+        return fail(DFS_ENOMEM);
+    }
+    cudaMemcpy(d_script, script, (size_t)n_ops * 6 * sizeof(int32_t), cudaMemcpyHostToDevice);
+    cudaMemset(d_out, 0xFF, (size_t)out_len * sizeof(int32_t) + 16);
+    ScriptArgs sa;
+    sa.d_script = d_script; sa.n_ops = n_ops; sa.d_out = d_out; sa.out_len = out_len;
+    cudaStream_t s = g->stream;
+    rc = launch_one(g, sl, s, 0, sl.parent, o, 1, warps, false, false, &sa);
+    if (rc == DFS_OK) {
+        if (cudaStreamSynchronize(s) != cudaSuccess ||
+            (out_len > 0 && cudaMemcpy(out, d_out, (size_t)out_len * sizeof(int32_t), cudaMemcpyDeviceToHost) != cudaSuccess)) {
+            cudaGetLastError();
+            rc = DFS_ECUDA;
+        }
+    }
+    sl.tab_dirty = true;                       // the script maps chunks it never returns
+    cudaFree(d_script); cudaFree(d_out);
+    return rc == DFS_OK ? DFS_OK : fail(rc);
+}

@@ -71,7 +71,7 @@ __global__ void __launch_bounds__(1024, 1) dfs_walker_kernel(const KParams P) {
     constexpr int WPW = 32 / G;                       // walkers per warp
     constexpr uint32_t GM = (1u << G) - 1u;
     constexpr int kPf = G < 8 ? G : 8;                // lanes prefetching candidates' row_ptr pairs
-    constexpr uint32_t kBatch = H / 2;                // flush / refill batch (reading S10)
+    constexpr uint32_t kBatch = H / 2;                // largest flush / refill batch (reading S10)
     constexpr uint32_t kStealMax = H / 4;             // entries per steal (ring space, see refill)
     extern __shared__ __align__(16) unsigned char smem_raw[];
     SmemW& S = *reinterpret_cast<SmemW*>(smem_raw);
@@ -91,6 +91,9 @@ __global__ void __launch_bounds__(1024, 1) dfs_walker_kernel(const KParams P) {
     const uint32_t tmask = (1u << P.tab_log2) - 1u;
     uint32_t* const my_tab = P.chunk_tab + ((size_t)gk << P.tab_log2);
     const uint32_t cap = P.ring_cap < (uint32_t)H ? P.ring_cap : (uint32_t)H;
+    // flush / refill batch: the paper's hot_size / 2 with capacity hot_size - 1 (Fig 2),
+    // i.e. (cap + 1) / 2 — H/2 at the default cap = H
+    const uint32_t batch = (cap + 1u) / 2u;
     const uint32_t hs = P.hot_cutoff >= 2 ? (uint32_t)P.hot_cutoff >> 1 : 1u;   // h_s (Alg 3 l.12)
     const uint32_t cs = P.cold_cutoff >= 2 ? (uint32_t)P.cold_cutoff >> 1 : 1u; // c_s (Alg 4 l.17)
 
@@ -262,7 +265,7 @@ __global__ void __launch_bounds__(1024, 1) dfs_walker_kernel(const KParams P) {
                 const uint32_t bot = (uint32_t)old;
                 const int avail = (int)(k_top - bot);
                 if (avail <= 0) { take = 0; break; }
-                take = avail < (int)kBatch ? (uint32_t)avail : kBatch;
+                take = avail < (int)batch ? (uint32_t)avail : batch;
                 const unsigned long long nw = ((unsigned long long)(k_top - take) << 32) | bot;
                 const unsigned long long got = atomicCAS(&P.cold_tb[kg], old, nw);
                 if (got == old) break;
@@ -495,6 +498,83 @@ __global__ void __launch_bounds__(1024, 1) dfs_walker_kernel(const KParams P) {
         return got_work;
     };
 
+    // ---------------------------------------------------------------- stack-script mode (tests)
+    // STATS builds only (dfs_debug_stack_script): warp 0 of block 0 drives its walkers' stack
+    // operations — the same lambdas the traversal uses — through a script of 6-int records, so the
+    // paper's worked examples (Figs 2 and 3) can be replayed on the real stack code.
+    if constexpr (STATS) {
+        if (P.script) {
+            if (blockIdx.x == 0 && w == 0) {
+                int oc = 0;                                   // output cursor (lane 0 writes)
+                auto put = [&](int32_t x) { if (lane == 0 && oc < P.script_out_len) P.script_out[oc] = x; ++oc; };
+                for (int pc = 0; pc < P.script_len; ++pc) {
+                    const int32_t* r = P.script + 6 * pc;
+                    const int op = r[0], k = r[1] & (WPW - 1);
+                    const int kb = w * WPW + k, kg = blockIdx.x * NWB + kb;
+                    uint32_t* const ktab = P.chunk_tab + ((size_t)kg << P.tab_log2);
+                    unsigned long long* const kring = rings + (size_t)kb * H;
+                    if (op == 0) break;
+                    if (op == 1) {                            // SET k head tail top bottom
+                        const uint32_t hd = (uint32_t)r[2] & 0xFFFFu, tl = (uint32_t)r[3] & 0xFFFFu;
+                        const uint32_t top = (uint32_t)r[4], bot = (uint32_t)r[5];
+                        uint32_t nh = 0;
+                        if (lane == 0) {
+                            S.ht[kb] = (hd << 16) | tl; S.tailf[kb] = tl;
+                            P.cold_tb[kg] = ((unsigned long long)top << 32) | bot;
+                            atomicAdd(&P.block_cold[blockIdx.x], (int)(top - bot));
+                            for (uint32_t c = 0; (unsigned long long)c * kChunk < top; ++c, ++nh) {
+                                const uint32_t id = pool_alloc(P);
+                                st_relaxed_u32(&P.chunk_consumed[id], 0u); st_relaxed_u32(&ktab[c & tmask], id);
+                            }
+                        }
+                        nh = __shfl_sync(kFull, nh, 0);
+                        __syncwarp();
+                        if (wk == k) { my_head = hd; pub = hd; tail_cache = tl; my_top = top; hi = nh; cold_lo = ~top; has_top = false; }
+                    } else if (op == 2 || op == 3) {          // RING k counter v i  /  COLD k pos v i
+                        if (lane == 0) {
+                            const unsigned long long e = pack_entry((uint32_t)r[3], (uint32_t)r[4]);
+                            const uint32_t q = (uint32_t)r[2];
+                            if (op == 2) kring[q & (H - 1)] = e;
+                            else P.pool[((size_t)ktab[(q >> kChunkLog2) & tmask] << kChunkLog2) + (q & (kChunk - 1))] = e;
+                        }
+                        __syncwarp();
+                    } else if (op == 4) {                     // PUSH k v i (Fig 2(c))
+                        const bool me = wk == k;
+                        st_shared_u64_if(me && sl == 0, ring + (my_head & (H - 1)), pack_entry((uint32_t)r[2], (uint32_t)r[3]));
+                        atom_add_release_cta_if(me && sl == 0, &S.ht[bk], 0x10000u);
+                        if (me) { ++my_head; pub = my_head; }
+                        __syncwarp();
+                    } else if (op == 5) {                     // POP k (Fig 2(d)) -> popped (v, i) or (-1, -1)
+                        pop_if(wk == k);
+                        const int got = __shfl_sync(kFull, (int)has_top, k * G);
+                        const uint32_t pv = __shfl_sync(kFull, u, k * G), pi = __shfl_sync(kFull, i, k * G);
+                        put(got ? (int32_t)pv : -1); put(got ? (int32_t)pi : -1);
+                        if (wk == k) has_top = false;
+                    } else if (op == 6) {                     // FLUSH k want keep (Fig 2(e))
+                        flush_walker(k, (uint32_t)r[2], (uint32_t)r[3]);
+                    } else if (op == 7) {                     // REFILL k (Fig 2(f)) -> entries moved
+                        put((int32_t)refill_walker(k));
+                    } else if (op == 8 || op == 9) {          // STEAL_INTRA / STEAL_INTER thief-mask (Fig 3)
+                        const uint32_t tb = (uint32_t)r[1] & ((1u << WPW) - 1u);
+                        put((int32_t)(op == 8 ? steal_intra(tb) : steal_inter(tb)));
+                    } else if (op == 10) {                    // DUMP k -> head tail top bottom
+                        const uint32_t x = S.ht[kb];
+                        const unsigned long long c = P.cold_tb[kg];
+                        put((int32_t)ht_head(x)); put((int32_t)ht_tail(x));
+                        put((int32_t)(uint32_t)(c >> 32)); put((int32_t)(uint32_t)c);
+                    } else if (op == 11 || op == 12) {        // READ_RING k counter / READ_COLD k pos -> v i
+                        const uint32_t q = (uint32_t)r[2];
+                        const unsigned long long e = op == 11 ? kring[q & (H - 1)]
+                            : P.pool[((size_t)ktab[(q >> kChunkLog2) & tmask] << kChunkLog2) + (q & (kChunk - 1))];
+                        put((int32_t)entry_v(e)); put((int32_t)entry_i(e));
+                    }
+                    __syncwarp();
+                }
+            }
+            return;
+        }
+    }
+
     // ---------------------------------------------------------------- main loop (Alg 2)
     for (;;) {
         if (__any_sync(kFull, has_top)) {
@@ -510,7 +590,7 @@ __global__ void __launch_bounds__(1024, 1) dfs_walker_kernel(const KParams P) {
                     while (fb) {
                         const int k = (__ffs(fb) - 1) / G;
                         fb &= fb - 1;
-                        if (!flush_walker(k, cap >= 2u ? cap / 2u : 1u, 0u)) { fail = true; break; }
+                        if (!flush_walker(k, batch, 0u)) { fail = true; break; }
                     }
                     if (fail) goto exit_loop;
                 }

@@ -28,7 +28,8 @@ STATUS = {0: "DFS_OK", -1: "DFS_EINVAL", -2: "DFS_ENOMEM", -3: "DFS_ECUDA", -4: 
 #: every symbol include/dfs.h declares (checked by tests/test_capi.py)
 EXPORTS = ["dfs_options_default", "dfs_graph_create", "dfs_run", "dfs_run_batch", "dfs_run_ex",
            "dfs_run_batch_ex", "dfs_set_stream", "dfs_graph_info", "dfs_launch_count",
-           "dfs_graph_destroy", "dfs_last_error", "dfs_strerror", "dfs_debug_timeline"]
+           "dfs_graph_destroy", "dfs_last_error", "dfs_strerror", "dfs_debug_timeline",
+           "dfs_debug_stack_script"]
 
 
 class DfsError(RuntimeError):
@@ -194,6 +195,8 @@ def load_library(path: Optional[str] = None):
         lib.dfs_launch_count.restype = I64
         lib.dfs_debug_timeline.argtypes = [P, ctypes.c_uint32, ctypes.c_uint32, P]
         lib.dfs_debug_timeline.restype = ctypes.c_int
+        lib.dfs_debug_stack_script.argtypes = [P, I32, P, I32, P, I32, ctypes.POINTER(_Options)]
+        lib.dfs_debug_stack_script.restype = ctypes.c_int
         lib.dfs_graph_destroy.argtypes = [P]
         lib.dfs_graph_destroy.restype = None
         lib.dfs_last_error.argtypes = []
@@ -347,6 +350,20 @@ class Graph:
         t = len_ // 3
         return (buf[:t].astype(np.int64) - 1, buf[t:2 * t].astype(np.int64),
                 buf[2 * t:3 * t].astype(np.int64))
+
+    def stack_script(self, lanes: int, ops, out_len: int = 256, options: Optional[Options] = None):
+        """Replay stack operations on the walker kernel's own code (dfs_debug_stack_script);
+        ``ops`` is a list of up to 6-int records; returns the int32 output values."""
+        rec = np.zeros((len(ops), 6), dtype=np.int32)
+        for q, r in enumerate(ops):
+            rec[q, :len(r)] = r
+        out = np.full(out_len, -7, dtype=np.int32)
+        o = options.to_c() if options is not None else None
+        rc = self._lib.dfs_debug_stack_script(self._h, int(lanes), rec.ctypes.data, len(ops), out.ctypes.data,
+                                              out_len, ctypes.byref(o) if o is not None else None)
+        if rc != 0:
+            raise DfsError(rc, "dfs_debug_stack_script")
+        return out
 
     def launch_count(self) -> int:
         return int(self._lib.dfs_launch_count(self._h))
