@@ -177,6 +177,10 @@ typedef struct dfs_options {
                                 list through its 32-byte vertex record (first 6 neighbours + its
                                 row_ptr pair; built once per handle on first use, 32 bytes per
                                 vertex of device memory); 0 = row_ptr then col_idx   */
+    int32_t spec_tail;       /* warp kernel, 128-wide windows: claim a descended child's next tree
+                                edge speculatively (as `speculate` does for 32-wide windows) while
+                                at most spec_tail blocks hold work — the serial tail of shallow
+                                power-law traversals; 0 = never                    */
 } dfs_options;
 
 typedef struct dfs_stats {

@@ -452,6 +452,7 @@ static int launch_one(dfs_graph* g, Slot& sl, cudaStream_t s, int32_t root, int3
     P.period_mask = (uint32_t)(o.spill_period > 0 ? o.spill_period : 32) - 1u;
     P.steal_period_mask = (uint32_t)(o.steal_period > 0 ? o.steal_period : 1) - 1u;
     P.donate = o.donate;
+    P.spec_tail = o.spec_tail > 0 ? o.spec_tail : 0;
     const bool tl = g->d_timeline && &sl == &g->slots[0];
     P.timeline = tl ? g->d_timeline : nullptr;
     P.timeline_len = tl ? (g->timeline_len / 3u) * 2u : 0;   // kernel: three regions of len/3

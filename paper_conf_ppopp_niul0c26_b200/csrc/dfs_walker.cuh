@@ -71,7 +71,6 @@ __global__ void __launch_bounds__(1024, 1) dfs_walker_kernel(const KParams P) {
     constexpr int WPW = 32 / G;                       // walkers per warp
     constexpr uint32_t GM = (1u << G) - 1u;
     constexpr int kPf = G < 8 ? G : 8;                // lanes prefetching candidates' row_ptr pairs
-    constexpr uint32_t kBatch = H / 2;                // largest flush / refill batch (reading S10)
     constexpr uint32_t kStealMax = H / 4;             // entries per steal (ring space, see refill)
     extern __shared__ __align__(16) unsigned char smem_raw[];
     SmemW& S = *reinterpret_cast<SmemW*>(smem_raw);
@@ -249,7 +248,7 @@ __global__ void __launch_bounds__(1024, 1) dfs_walker_kernel(const KParams P) {
 
     // refill walker k's empty HotRing from its ColdSeg top (Fig 2(f)); returns the
     // number of entries moved.  Ring space: a thief may still be copying <= kStealMax slots below
-    // head, so head + kBatch - tailf <= H holds with kBatch = H/2.
+    // head, so head + batch - tailf <= H holds with batch <= H/2.
     auto refill_walker = [&](int k) -> uint32_t {
         const int kb = w * WPW + k;
         const int kg = blockIdx.x * NWB + kb;

@@ -56,7 +56,7 @@ class _Options(ctypes.Structure):
                 ("bulk_copy", ctypes.c_int32), ("spill_period", ctypes.c_int32),
                 ("l2_persist_mb", ctypes.c_int32), ("walker_lanes", ctypes.c_int32),
                 ("steal_period", ctypes.c_int32), ("donate", ctypes.c_int32),
-                ("records", ctypes.c_int32)]
+                ("records", ctypes.c_int32), ("spec_tail", ctypes.c_int32)]
 
 
 class _Stats(ctypes.Structure):
@@ -113,6 +113,7 @@ class Options:
     steal_period: Optional[int] = None
     donate: Optional[bool] = None
     records: Optional[bool] = None
+    spec_tail: Optional[int] = None
 
     def to_c(self) -> _Options:
         o = _Options()
