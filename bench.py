@@ -395,7 +395,8 @@ def single_root_leg(a, workload, g, root0, undirected, desc, world, rank, local,
     achieved = kbytes / my_trav / 1e9            # rank 0's own launches (per-GPU kernel figure)
     roof = {"bound": "hbm", "achieved": round(achieved, 3), "peak": peak, "unit": "GB/s",
             "frac": round(achieved / peak, 6), "traffic": traffic_from_profile(workload),
-            "kernel": "b200dfs::dfs_persistent_kernel", "peak_source": peak_src,
+            "kernel": (f"b200dfs::dfs_walker_kernel<{st.walker_lanes}> (sub-warp walkers)" if st.walker_lanes != 32
+                       else f"b200dfs::dfs_persistent_kernel ({st.window}-wide windows)"), "peak_source": peak_src,
             "bytes_per_launch_avg": round(kbytes / steps, 1),
             "launch_ms_avg": round(my_trav * 1e3 / steps, 4),
             "kernel_share_of_step": round(my_trav / my_time, 4),
@@ -468,6 +469,8 @@ def batch_leg(a, g, world, rank, local, dev):
     if world > 1 and rank == 0 and not a.no_gather:
         sink = [torch.empty((sub, g.n), dtype=torch.int32, device=dev) for _ in range(world)]
 
+    lanes = []
+
     def one_pass(gather):
         counts = []
         launches0 = G.launch_count()
@@ -481,6 +484,7 @@ def batch_leg(a, g, world, rank, local, dev):
             if chunk:
                 _, st = G.run_batch(chunk, out=out_rows[:len(chunk)], options=o, stats=True)
                 counts.append(st.root_counts.copy())
+                lanes.append(st.walker_lanes)
             if gather and world > 1:
                 batch.gather_chunk_to_rank0(out_rows, len(chunk), min(rows, cap - c0), sub, sink, world, rank)
         e1.record()
@@ -515,12 +519,17 @@ def batch_leg(a, g, world, rank, local, dev):
         return None
     peak, peak_src = measured_peaks()
     conc = opts.get("concurrency", 0) or "auto (8)"
+    kl = lanes[0] if lanes else 32
     b = {"roots": k, "dfs_per_s": round(k / (t_trav * 1e-3), 3), "ms_per_dfs": round(t_trav / k, 4),
          "region_ms": round(t_trav, 3), "gteps": round(tot_edges / (t_trav * 1e-3) / 1e9, 4),
          "partition": f"contiguous slices of {k} seeded roots over {world} rank(s) (strong scaling)",
          "concurrency": conc, "rows_per_call": rows, "gpu_launches": int(launches), "clocks": clk,
          "roofline": {"bound": "hbm", "achieved": round(my_bytes / (my_ms * 1e-3) / 1e9, 3), "peak": peak,
                       "unit": "GB/s", "frac": round(my_bytes / (my_ms * 1e-3) / 1e9 / peak, 6),
+                      "traffic": traffic_from_profile("batch"), "traffic_what": "ncu dram read+write of one "
+                      "traversal-kernel launch of a K = 8 batch (profiles/r02/ncu/ncu_batch.md)",
+                      "kernel": (f"b200dfs::dfs_walker_kernel<{kl}> (sub-warp walkers)" if kl != 32
+                                 else "b200dfs::dfs_persistent_kernel"),
                       "peak_source": peak_src,
                       "what": "rank 0: SURVEY 8(d) B_min (4n + 12 n_r + 8 m_r) x its roots / its batch region time "
                               "(concurrent traversal kernels overlap, so the region is the kernel time)"},

@@ -177,10 +177,6 @@ typedef struct dfs_options {
                                 list through its 32-byte vertex record (first 6 neighbours + its
                                 row_ptr pair; built once per handle on first use, 32 bytes per
                                 vertex of device memory); 0 = row_ptr then col_idx   */
-    int32_t spec_tail;       /* warp kernel, 128-wide windows: claim a descended child's next tree
-                                edge speculatively (as `speculate` does for 32-wide windows) while
-                                at most spec_tail blocks hold work — the serial tail of shallow
-                                power-law traversals; 0 = never                    */
 } dfs_options;
 
 typedef struct dfs_stats {
@@ -211,6 +207,8 @@ typedef struct dfs_stats {
     int64_t dead_pops;       /* ... of which found nothing left to claim (every remaining target
                                 was claimed after the entry was pushed)                            */
     int64_t donations;       /* walker kernel: entries handed to idle sibling walkers             */
+    int32_t walker_lanes;    /* kernel that ran: 32 = warp kernel, else lanes per walker          */
+    int32_t window;          /* warp kernel window (32 or 128)                                    */
 } dfs_stats;
 
 void dfs_options_default(dfs_options *opt);

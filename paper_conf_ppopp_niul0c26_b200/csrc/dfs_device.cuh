@@ -119,7 +119,6 @@ struct KParams {
     int script_len;
     int32_t* script_out;
     int script_out_len;
-    int spec_tail;                           // 128-wide step: speculate while <= spec_tail blocks are busy
 };
 
 // vertex records (create time, on first use): record v = 8 words = one 32-byte
@@ -556,8 +555,7 @@ __global__ void __launch_bounds__(32 * WMAX, 1) dfs_persistent_kernel(const KPar
     // speculate: bits 0-1 = mode (0 off, 1 on, 2 on for 32-wide windows), bit 2 = issue the
     // child's first window before the claim returns (32-wide), bit 3 = also claim a popped
     // entry's next position speculatively (its probe at push time saw it unvisited)
-    // (128-wide windows: turned on while at most P.spec_tail blocks are busy — the serial tail)
-    bool spec_on = (P.speculate & 3) == 1 || ((P.speculate & 3) == 2 && VEC == 1);
+    const bool spec_on = (P.speculate & 3) == 1 || ((P.speculate & 3) == 2 && VEC == 1);
     const bool spec_pop = spec_on && (P.speculate & 8) != 0;
     const bool spec_early = spec_on && (P.speculate & 4) != 0;
     const uint32_t leaf_deg = P.leaf_skip ? 1u : 0u;   // children of degree <= this may be leaves
@@ -1261,14 +1259,6 @@ __global__ void __launch_bounds__(32 * WMAX, 1) dfs_persistent_kernel(const KPar
                     }
                 }
                 sample();
-                if constexpr (VEC == 4) {
-                    // serial tail (few busy blocks): claim the next tree edge
-                    // speculatively, as the 32-wide step does
-                    if (P.spec_tail) {
-                        const uint32_t bb = __shfl_sync(kFull, lane == 0 ? *(volatile unsigned int*)&P.ctl->busy : 0u, 0);
-                        spec_on = bb <= (uint32_t)P.spec_tail;
-                    }
-                }
                 if (P.spill) {
                     // demand-driven spill: many warps idle and a deep HotRing -> make the oldest
                     // half of it visible to other blocks (Alg 4 steals ColdSeg bottoms only)

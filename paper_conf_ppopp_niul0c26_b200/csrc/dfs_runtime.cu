@@ -452,7 +452,6 @@ static int launch_one(dfs_graph* g, Slot& sl, cudaStream_t s, int32_t root, int3
     P.period_mask = (uint32_t)(o.spill_period > 0 ? o.spill_period : 32) - 1u;
     P.steal_period_mask = (uint32_t)(o.steal_period > 0 ? o.steal_period : 1) - 1u;
     P.donate = o.donate;
-    P.spec_tail = o.spec_tail > 0 ? o.spec_tail : 0;
     const bool tl = g->d_timeline && &sl == &g->slots[0];
     P.timeline = tl ? g->d_timeline : nullptr;
     P.timeline_len = tl ? (g->timeline_len / 3u) * 2u : 0;   // kernel: three regions of len/3
@@ -628,8 +627,8 @@ static int check_device(const dfs_graph* g) {
     return cur == g->device ? DFS_OK : DFS_EDEVICE;
 }
 
-static void fill_stats(dfs_stats* stats, int blocks, int warps, float total_ms, float trav_ms, int64_t nv,
-                       int64_t mv, const unsigned long long* counters) {
+static void fill_stats(dfs_stats* stats, const dfs_options& o, int blocks, int warps, float total_ms, float trav_ms,
+                       int64_t nv, int64_t mv, const unsigned long long* counters) {
     int64_t* keep = stats->root_counts;
     std::memset(stats, 0, sizeof(*stats));
     stats->root_counts = keep;
@@ -658,6 +657,8 @@ static void fill_stats(dfs_stats* stats, int blocks, int warps, float total_ms, 
     stats->pops = (int64_t)counters[kCntPops];
     stats->dead_pops = (int64_t)counters[kCntDeadPops];
     stats->donations = (int64_t)counters[kCntDonations];
+    stats->walker_lanes = o.walker_lanes;
+    stats->window = o.window;
 }
 
 // per-root count buffer (2 x u64 per root) for stats calls
@@ -762,7 +763,7 @@ static int run_sequential(dfs_graph* g, const int32_t* roots, int32_t k, int32_t
         const int rc = finish_counts(g, k, stats, nv, mv);
         if (rc != DFS_OK) return fail(rc);
         int64_t* bc = stats->block_claims;
-        fill_stats(stats, blocks, warps, total_ms, trav_ms, nv, mv, counters);
+        fill_stats(stats, o, blocks, warps, total_ms, trav_ms, nv, mv, counters);
         stats->block_claims = bc;
         if (bc) {
             std::vector<unsigned long long> h((size_t)blocks);
@@ -847,7 +848,7 @@ static int run_concurrent(dfs_graph* g, const int32_t* roots, int32_t k, int32_t
         float ms = 0.f;
         cudaEventElapsedTime(&ms, s0.ev0, s0.evk1);
         unsigned long long counters[kNumWCounters] = {0};
-        fill_stats(stats, blocks, warps, ms, ms, nv, mv, counters);
+        fill_stats(stats, o, blocks, warps, ms, ms, nv, mv, counters);
     }
     return DFS_OK;
 }

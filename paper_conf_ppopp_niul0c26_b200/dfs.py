@@ -56,7 +56,7 @@ class _Options(ctypes.Structure):
                 ("bulk_copy", ctypes.c_int32), ("spill_period", ctypes.c_int32),
                 ("l2_persist_mb", ctypes.c_int32), ("walker_lanes", ctypes.c_int32),
                 ("steal_period", ctypes.c_int32), ("donate", ctypes.c_int32),
-                ("records", ctypes.c_int32), ("spec_tail", ctypes.c_int32)]
+                ("records", ctypes.c_int32)]
 
 
 class _Stats(ctypes.Structure):
@@ -73,7 +73,8 @@ class _Stats(ctypes.Structure):
                 ("cyc_claim", ctypes.c_int64), ("cyc_tail", ctypes.c_int64),
                 ("cyc_outside", ctypes.c_int64), ("root_counts", ctypes.c_void_p),
                 ("block_claims", ctypes.c_void_p), ("cluster_steals", ctypes.c_int64),
-                ("pops", ctypes.c_int64), ("dead_pops", ctypes.c_int64), ("donations", ctypes.c_int64)]
+                ("pops", ctypes.c_int64), ("dead_pops", ctypes.c_int64), ("donations", ctypes.c_int64),
+                ("walker_lanes", ctypes.c_int32), ("window", ctypes.c_int32)]
 
 
 @dataclass
@@ -113,7 +114,6 @@ class Options:
     steal_period: Optional[int] = None
     donate: Optional[bool] = None
     records: Optional[bool] = None
-    spec_tail: Optional[int] = None
 
     def to_c(self) -> _Options:
         o = _Options()
@@ -154,6 +154,8 @@ class Stats:
     pops: int = 0
     dead_pops: int = 0
     donations: int = 0
+    walker_lanes: int = 32
+    window: int = 32
     root_counts: Optional[np.ndarray] = None
     block_claims: Optional[np.ndarray] = None
 
