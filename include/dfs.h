@@ -160,7 +160,7 @@ typedef struct dfs_options {
                                 128-wide windows (A/B on B200: RMAT-24 -4.8%, road/path neutral),
                                 else off; -1 = off.  The limit stays set after the handle is gone  */
     int32_t walker_lanes;    /* lanes per walker: 32 = the warp kernel (one walker per warp, windows of
-                                `window` positions); 16, 8 or 4 = the sub-warp walker kernel (32/L
+                                `window` positions); 16, 8, 4 or 2 = the sub-warp walker kernel (32/L
                                 independent walkers per warp, each with its own HotRing/ColdSeg and
                                 an L-position window); 0 = auto: 4-lane walkers on
                                 low-degree graphs (m <= 4n, max degree <= 16) for batches with
@@ -254,7 +254,7 @@ int64_t dfs_launch_count(const dfs_graph *g);
 int dfs_debug_timeline(dfs_graph *g, uint32_t len, uint32_t dt_ns, uint32_t *out);
 
 /* Diagnostics / tests: run a script of stack operations on the walkers of warp 0, block 0 of the
- * sub-warp walker kernel (lanes = 16, 8 or 4 lanes per walker), using the kernel's own HotRing,
+ * sub-warp walker kernel (lanes = 16, 8, 4 or 2 lanes per walker), using the kernel's own HotRing,
  * ColdSeg and steal code (the paper's worked examples, Figs 2 and 3, are replayed this
  * way by tests/test_gpu_stack_script.py).  script: n_ops records of 6 int32 {op, a, b, c, d, e}:
  *   0 END; 1 SET w head tail top bottom (maps ColdSeg chunks for [0, top)); 2 RING w counter v i;

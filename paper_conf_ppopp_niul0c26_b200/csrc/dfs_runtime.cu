@@ -56,24 +56,29 @@ const void* const* kernel_table() {
 #undef DFS_K
 constexpr int kNumKernels = 24;
 
-// sub-warp walker kernels (dfs_walker.cuh): [G = 16, 8, 4][stats], then the vertex-record
+// sub-warp walker kernels (dfs_walker.cuh): [G = 16, 8, 4, 2][stats], then the vertex-record
 // variants [G = 16, 8][stats]; HotRing H = 16 * G entries per walker, so a 32-warp CTA holds
 // 128 KB of rings for every G
 #define DFS_WK(G, S, R) (const void*)dfs_walker_kernel<G, 16 * G, S, R>
 const void* const* walker_table() {
-    static const void* const t[10] = {DFS_WK(16, false, false), DFS_WK(16, true, false), DFS_WK(8, false, false),
+    static const void* const t[12] = {DFS_WK(16, false, false), DFS_WK(16, true, false), DFS_WK(8, false, false),
                                       DFS_WK(8, true, false), DFS_WK(4, false, false), DFS_WK(4, true, false),
+                                      DFS_WK(2, false, false), DFS_WK(2, true, false),
                                       DFS_WK(16, false, true), DFS_WK(16, true, true), DFS_WK(8, false, true),
                                       DFS_WK(8, true, true)};
     return t;
 }
 #undef DFS_WK
-constexpr int kNumWalkerKernels = 10;
-int walker_lanes_of(int kf) { return (kf % 6) < 2 ? 16 : (kf % 6) < 4 ? 8 : 4; }
-int walker_index(int lanes, bool rec) {
-    if (rec && lanes >= 8) return lanes == 16 ? 6 : 8;
-    return lanes == 16 ? 0 : lanes == 8 ? 2 : 4;
+constexpr int kNumWalkerKernels = 12;
+int walker_lanes_of(int kf) {
+    static const int lanes[12] = {16, 16, 8, 8, 4, 4, 2, 2, 16, 16, 8, 8};
+    return lanes[kf];
 }
+int walker_index(int lanes, bool rec) {
+    if (rec && lanes >= 8) return lanes == 16 ? 8 : 10;
+    return lanes == 16 ? 0 : lanes == 8 ? 2 : lanes == 4 ? 4 : 6;
+}
+bool valid_walker_lanes(int lanes) { return lanes == 16 || lanes == 8 || lanes == 4 || lanes == 2; }
 
 size_t smem_bytes(int warps) {
     return ((sizeof(SmemCtl) + 15) & ~size_t(15)) + (size_t)warps * kRing * sizeof(unsigned long long);
@@ -548,8 +553,7 @@ static int resolve_options(dfs_graph* g, const dfs_options* in, int num_roots, d
     if (o.reserved0 != 0) return DFS_EINVAL;
     if (o.spill_period < 0 || o.spill_period > 1024 || (o.spill_period & (o.spill_period - 1))) return DFS_EINVAL;
     if (o.cluster < 0 || o.cluster > 8 || (o.cluster > 1 && (o.cluster & (o.cluster - 1)))) return DFS_EINVAL;
-    if (o.walker_lanes != 0 && o.walker_lanes != 32 && o.walker_lanes != 16 && o.walker_lanes != 8 && o.walker_lanes != 4)
-        return DFS_EINVAL;
+    if (o.walker_lanes != 0 && o.walker_lanes != 32 && !valid_walker_lanes(o.walker_lanes)) return DFS_EINVAL;
     if (o.steal_period < 0 || o.steal_period > 1024 || (o.steal_period & (o.steal_period - 1))) return DFS_EINVAL;
     const bool window_auto = o.window == 0;
     if (o.window == 0) o.window = (g->n > 0 && g->m >= 8 * g->n) ? 128 : 32;   // wide windows for dense lists
@@ -942,7 +946,7 @@ int dfs_run_batch(dfs_graph* g, const int32_t* roots, int32_t num_roots, int32_t
 
 extern "C" int dfs_debug_stack_script(dfs_graph* g, int32_t lanes, const int32_t* script, int32_t n_ops,
                                       int32_t* out, int32_t out_len, const dfs_options* opt) {
-    if (!g || !script || n_ops < 0 || (out_len > 0 && !out) || (lanes != 16 && lanes != 8 && lanes != 4))
+    if (!g || !script || n_ops < 0 || (out_len > 0 && !out) || !valid_walker_lanes(lanes))
         return fail(DFS_EINVAL);
     int rc = check_device(g);
     if (rc != DFS_OK) return fail(rc);

@@ -24,7 +24,7 @@
 
 namespace b200dfs {
 
-constexpr int kMaxWalkersPerCta = 256;
+constexpr int kMaxWalkersPerCta = 512;
 constexpr int kCntDonations = kNumCounters;         // walker kernel only (Ctl::counters has 24)
 constexpr int kNumWCounters = kNumCounters + 1;
 
@@ -65,7 +65,7 @@ __device__ __forceinline__ unsigned long long ld_shared_u64_if(bool p, const uns
 // ------------------------------------------------------------------------------------------
 template <int G, int H, bool STATS, bool REC>
 __global__ void __launch_bounds__(1024, 1) dfs_walker_kernel(const KParams P) {
-    static_assert(G == 4 || G == 8 || G == 16, "G is 4, 8 or 16");
+    static_assert(G == 2 || G == 4 || G == 8 || G == 16, "G is 2, 4, 8 or 16");
     static_assert(!REC || G >= 8, "a vertex record spans 8 lanes");
     static_assert((H & (H - 1)) == 0 && H >= 32 && H <= 1024, "H is a power of two in [32, 1024]");
     constexpr int WPW = 32 / G;                       // walkers per warp

@@ -38,7 +38,7 @@ def G():
         yield h
 
 
-@pytest.mark.parametrize("lanes", [16, 8, 4])
+@pytest.mark.parametrize("lanes", [16, 8, 4, 2])
 def test_fig2_two_level_stack_on_kernel_code(G, lanes):
     d = _gold("fig2_two_level_stack.json")
     hs = d["hot_size"]
@@ -82,7 +82,7 @@ def test_fig2_two_level_stack_on_kernel_code(G, lanes):
     assert tuple(out[5:9]) == (A, 1, B, 2)
 
 
-@pytest.mark.parametrize("lanes", [8, 4])                 # >= 3 walkers per warp
+@pytest.mark.parametrize("lanes", [8, 4, 2])              # >= 3 walkers per warp
 def test_fig3a_intra_block_steal_on_kernel_code(G, lanes):
     d = _gold("fig3_steals.json")["intra"]
     e = d["expect"]
@@ -104,7 +104,7 @@ def test_fig3a_intra_block_steal_on_kernel_code(G, lanes):
     assert e["mask_before"] == "100" and e["mask_after"] == "110"   # (walker 1 became active)
 
 
-@pytest.mark.parametrize("lanes", [8, 4])
+@pytest.mark.parametrize("lanes", [8, 4, 2])
 def test_fig3b_inter_block_steal_on_kernel_code(G, lanes):
     d = _gold("fig3_steals.json")["inter"]
     e = d["expect"]

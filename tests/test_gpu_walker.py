@@ -16,7 +16,7 @@ pytestmark = pytest.mark.gpu
 if torch.cuda.is_available():
     from paper_conf_ppopp_niul0c26_b200 import DfsError, Graph, Options
 
-LANES = [16, 8, 4]
+LANES = [16, 8, 4, 2]
 
 
 def _valid(g, root, parent, undirected=True):
