@@ -514,6 +514,33 @@ def batch_leg(a, g, world, rank, local, dev):
             vals.append(int(res.ok))
     _, (tot_bytes, tot_edges, nval, nok) = batch.reduce_max_sum(
         [], [my_bytes, my_edges, float(len(vals)), float(sum(vals))], world, device=dev)
+    # e2e: the public C symbol dfs_run_batch with HOST buffers (roots in host memory, parent rows
+    # into pinned host memory), wall clock with a device sync on both sides; a bounded sample of
+    # E roots per rank (the full 1,024 x 96 MB of rows would not fit in host memory)
+    e2e = None
+    if not a.no_e2e:
+        import ctypes
+        from paper_conf_ppopp_niul0c26_b200 import dfs as dfsmod
+        lib = dfsmod.load_library()
+        E = min(16, len(mine))
+        hroots = np.ascontiguousarray(np.array(mine[:E], dtype=np.int32))
+        hout = torch.empty((max(E, 1), g.n), dtype=torch.int32).pin_memory()
+        h = ctypes.c_void_p(G._h)
+        assert lib.dfs_run_batch(h, hroots.ctypes.data, E, ctypes.c_void_p(hout.data_ptr())) == 0   # warm-up
+        if world > 1:
+            dist.barrier()
+        torch.cuda.synchronize()
+        t0 = time.perf_counter()
+        rc = lib.dfs_run_batch(h, hroots.ctypes.data, E, ctypes.c_void_p(hout.data_ptr()))
+        torch.cuda.synchronize()
+        el = time.perf_counter() - t0
+        assert rc == 0, rc
+        del hout
+        (el_max,), (roots_all,) = batch.reduce_max_sum([el], [float(E)], world, device=dev)
+        e2e = {"value": round(roots_all / el_max, 3), "unit": "DFS/s", "h2d_bytes_per_step": int(E * 4),
+               "d2h_bytes_per_step": int(E * g.n * 4), "roots_per_rank": E,
+               "what": f"dfs_run_batch(resident graph, {E} host roots, pinned host parents_out) per rank; "
+                       "wall clock, max over ranks"}
     G.close()
     if rank != 0:
         return None
@@ -535,6 +562,8 @@ def batch_leg(a, g, world, rank, local, dev):
                               "(concurrent traversal kernels overlap, so the region is the kernel time)"},
          "validation": {"rows_checked": int(nval), "rows_ok_I1_I6": int(nok),
                         "what": "4 rows of the last timed chunk per rank, oracle.check_tree I1-I6 exact"}}
+    if e2e is not None:
+        b["e2e"] = e2e
     if world == 1:
         b["with_gather"] = {"dfs_per_s": b["dfs_per_s"], "region_ms": b["region_ms"], "bytes_to_rank0": 0,
                             "what": "N=1: the parent rows are already on rank 0 (no exchange step)"}
