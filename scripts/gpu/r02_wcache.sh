@@ -6,6 +6,6 @@ timeout 900 python scripts/ab_libs.py --libs paper_conf_ppopp_niul0c26_b200/libd
 grep lib gpurun_out/ab_wcache_rmat.jsonl || tail -20 gpurun_out/ab_wcache_rmat.jsonl
 timeout 600 python scripts/ab_libs.py --libs paper_conf_ppopp_niul0c26_b200/libdfs.so ab/wcache/libdfs.so --config road24m --reps 3 --steps 6 > gpurun_out/ab_wcache_road.jsonl 2>&1
 grep lib gpurun_out/ab_wcache_road.jsonl || tail -20 gpurun_out/ab_wcache_road.jsonl
-timeout 900 ncu --metrics dram__bytes_read.sum,dram__bytes_write.sum,gpu__time_duration.sum --clock-control none -k regex:dfs_persistent_kernel --launch-skip 1 -c 1 --csv \
-  env DFS_LIB=ab/wcache/libdfs.so python scripts/ncu_run.py --config rmat24 > gpurun_out/ncu_wcache_rmat.csv 2>&1; echo ncu rc=$?
+DFS_LIB=ab/wcache/libdfs.so timeout 900 ncu --metrics dram__bytes_read.sum,dram__bytes_write.sum,gpu__time_duration.sum --clock-control none -k regex:dfs_persistent_kernel --launch-skip 1 -c 1 --csv \
+  python scripts/ncu_run.py --config rmat24 > gpurun_out/ncu_wcache_rmat.csv 2>&1; echo ncu rc=$?
 grep -E "dram__bytes|gpu__time" gpurun_out/ncu_wcache_rmat.csv | cut -c1-300
