@@ -80,6 +80,8 @@ def main():
             res = oracle.check_tree(g.row_ptr, g.col_idx, r, par, undirected=undirected)
             assert res.ok, (p, r, res)
         G.run(roots[0], out=out, options=o)
+        if a.batch:                                  # scratch slots of the batch: allocated untimed
+            G.run_batch(broots, out=bout, options=o)
     res = {p: {"step_ms": [], "trav_ms": [], "gteps": []} for p in names}
     s = 0
     for rep in range(a.reps):
