@@ -38,11 +38,6 @@
 #pragma once
 #include <cstdint>
 
-// DFS_WCACHE = 1: hub-window cache in the 128-wide step (A/B build; see the kernel)
-#ifndef DFS_WCACHE
-#define DFS_WCACHE 0
-#endif
-
 namespace b200dfs {
 
 constexpr uint32_t kFull = 0xffffffffu;
@@ -524,15 +519,6 @@ __global__ void __launch_bounds__(32 * WMAX, 1) dfs_persistent_kernel(const KPar
     unsigned long long* const ring = rings + (size_t)w * H;
     const uint32_t tmask = (1u << P.tab_log2) - 1u;
     uint32_t* const my_tab = P.chunk_tab + ((size_t)gw << P.tab_log2);
-#if DFS_WCACHE
-    // hub-window cache (128-wide step): the window of the last pushed entry, so that popping it
-    // back (the common case on shallow power-law graphs: the child's subtree pushed nothing)
-    // needs neither the row_ptr load nor the col_idx window reload.  col_idx is immutable, so
-    // a tag match {u, window base} is always a valid hit — no invalidation
-    int4* const wc = reinterpret_cast<int4*>(rings + (size_t)W * H) + (size_t)w * 32;
-    uint32_t* const wct = reinterpret_cast<uint32_t*>(reinterpret_cast<int4*>(rings + (size_t)W * H) + (size_t)W * 32) + 4 * w;
-    if (VEC == 4 && lane == 0) wct[0] = kFull;
-#endif
     const uint32_t hs = P.hot_cutoff >= 2 ? (uint32_t)P.hot_cutoff >> 1 : 1u;   // h_s (Alg 3 l.12)
     const uint32_t cs = P.cold_cutoff >= 2 ? (uint32_t)P.cold_cutoff >> 1 : 1u; // c_s (Alg 4 l.17)
 
@@ -1064,21 +1050,6 @@ __global__ void __launch_bounds__(32 * WMAX, 1) dfs_persistent_kernel(const KPar
             const uint32_t a = i & ~(uint32_t)(VEC - 1);
             if (!have_win || win_lanes < 32) {
                 if (!have_win) {
-#if DFS_WCACHE
-                    __syncwarp();
-                    const uint32_t cu = wct[0], ca = wct[1];
-                    if (need_end && cu == u && ca <= a && a < ca + kWin) {    // cached window (hit)
-                        const int sh = (int)((a - ca) / (uint32_t)VEC);
-                        end = wct[2]; need_end = false;
-                        int tnb[VEC];
-                        load_window(a, end, 32, tnb, 32 - sh);   // positions past the cached window
-                        const int4 x = wc[lane + sh < 32 ? lane + sh : 0];
-                        const bool cached = lane + sh < 32;
-                        nbv[0] = cached ? x.x : tnb[0]; nbv[1] = cached ? x.y : tnb[1];
-                        nbv[2] = cached ? x.z : tnb[2]; nbv[3] = cached ? x.w : tnb[3];
-                        win_lanes = 32;
-                    } else
-#endif
                     if (need_end) {                                   // popped entry: end unknown
                         const uint32_t e2 = __ldg(P.rp + u + 1);
                         load_window(a, P.m, kHeadLanes, nbv);
@@ -1255,12 +1226,6 @@ __global__ void __launch_bounds__(32 * WMAX, 1) dfs_persistent_kernel(const KPar
                     }
                 }
                 if (ni < end) {
-#if DFS_WCACHE
-                    if (ni < a + kWin) {                          // <u, ni> resumes inside this window
-                        wc[lane] = make_int4(nbv[0], nbv[1], nbv[2], nbv[3]);
-                        if (lane == 0) { wct[0] = u; wct[1] = a; wct[2] = end; }
-                    }
-#endif
                     if (!push_lean(u, ni)) goto exit_loop;
                 }
                 st_global_if(lane == 0, P.parent + v, (int32_t)u);             // Alg 1 l.10

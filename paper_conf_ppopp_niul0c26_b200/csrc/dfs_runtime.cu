@@ -81,8 +81,7 @@ int walker_index(int lanes, bool rec) {
 bool valid_walker_lanes(int lanes) { return lanes == 16 || lanes == 8 || lanes == 4 || lanes == 2; }
 
 size_t smem_bytes(int warps) {
-    return ((sizeof(SmemCtl) + 15) & ~size_t(15)) + (size_t)warps * kRing * sizeof(unsigned long long)
-           + (DFS_WCACHE ? (size_t)warps * (32 * 16 + 16) : 0);   // hub-window cache (128-wide step)
+    return ((sizeof(SmemCtl) + 15) & ~size_t(15)) + (size_t)warps * kRing * sizeof(unsigned long long);
 }
 size_t walker_smem_bytes(int warps, int lanes) {
     return ((sizeof(SmemW) + 15) & ~size_t(15)) + (size_t)warps * (32 / lanes) * (16 * lanes) * sizeof(unsigned long long);
