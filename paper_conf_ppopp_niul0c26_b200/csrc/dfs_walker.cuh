@@ -25,6 +25,9 @@
 namespace b200dfs {
 
 constexpr int kMaxWalkersPerCta = 512;
+#ifndef DFS_WALKER_FULLSCAN
+#define DFS_WALKER_FULLSCAN 0
+#endif
 constexpr int kCntDonations = kNumCounters;         // walker kernel only (Ctl::counters has 24)
 constexpr int kNumWCounters = kNumCounters + 1;
 
@@ -333,13 +336,24 @@ __global__ void __launch_bounds__(1024, 1) dfs_walker_kernel(const KParams P) {
 
     // Alg 3 for the thief walkers tb: the walker of this CTA with max hot_rest >= hot_cutoff
     // (siblings in this warp included); reserve from its tail under its lock, copy SMEM -> SMEM
+    // Victim scan: a window of 32 walkers per attempt starting at this warp's own walkers and
+    // rotating through the CTA (one shared load per lane), not all of the CTA's 32 x 32/G walkers
+    // as Alg 3 l.5-10 does for 32 warps: with 256 walkers per CTA the full scan was 16% of the
+    // batch's instructions.  DFS_WALKER_FULLSCAN = 1 builds the full scan (A/B).
+    uint32_t scan_off = 0;
     auto steal_intra = [&](uint32_t tb) -> uint32_t {
         int best = -1, bidx = -1;
-        for (int j = lane; j < NWB; j += 32) {
-            if (j / WPW == w && ((tb >> (j % WPW)) & 1u)) continue;   // a thief itself
+        auto consider = [&](int j) {
+            if (j / WPW == w && ((tb >> (j % WPW)) & 1u)) return;    // a thief itself
             const int r = ht_rest(*(volatile uint32_t*)&S.ht[j]);
             if (r > best) { best = r; bidx = j; }
-        }
+        };
+#if DFS_WALKER_FULLSCAN
+        for (int j = lane; j < NWB; j += 32) consider(j);
+#else
+        if (lane < NWB) consider((int)(((uint32_t)(w * WPW) + scan_off + (uint32_t)lane) % (uint32_t)NWB));
+        scan_off += 32u;
+#endif
         for (int att = 0; att < P.steal_tries; ++att) {
             const int mx = __reduce_max_sync(kFull, best);
             if (mx < P.hot_cutoff) break;
