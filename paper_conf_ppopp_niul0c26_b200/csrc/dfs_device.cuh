@@ -497,10 +497,12 @@ __global__ void __launch_bounds__(32 * WMAX, 1) dfs_persistent_kernel(const KPar
 #define DFS_SEQPF 0
 #endif
 #ifndef DFS_PF_LANES128
-#define DFS_PF_LANES128 2
+#define DFS_PF_LANES128 0
 #endif
-    // lanes whose candidates' row_ptr pairs are loaded with the probes: the first 8 positions
-    // (128-wide: DFS_PF_LANES128 lanes of 4 positions; A/B builds only)
+    // lanes whose candidates' row_ptr pairs are loaded with the probes: the first 8 positions of
+    // a 32-wide window; none for 128-wide windows (round 2: on RMAT-24 those speculative loads were
+    // 15% of the L2 sector requests and most missed — 0 lanes: 9.76 -> 8.88 ms, DRAM reads 6.46 ->
+    // 5.00 GB, profiles/r02/ab/pf_width_rmat.jsonl; DFS_PF_LANES128 = 1/2 rebuilds the old widths)
     constexpr int kPfLanes = VEC == 1 ? 8 : DFS_PF_LANES128;
     extern __shared__ __align__(16) unsigned char smem_raw[];
     SmemCtl& S = *reinterpret_cast<SmemCtl*>(smem_raw);
