@@ -503,7 +503,10 @@ __global__ void __launch_bounds__(32 * WMAX, 1) dfs_persistent_kernel(const KPar
     // a 32-wide window; none for 128-wide windows (round 2: on RMAT-24 those speculative loads were
     // 15% of the L2 sector requests and most missed — 0 lanes: 9.76 -> 8.88 ms, DRAM reads 6.46 ->
     // 5.00 GB, profiles/r02/ab/pf_width_rmat.jsonl; DFS_PF_LANES128 = 1/2 rebuilds the old widths)
-    constexpr int kPfLanes = VEC == 1 ? 8 : DFS_PF_LANES128;
+#ifndef DFS_PF_LANES32
+#define DFS_PF_LANES32 8
+#endif
+    constexpr int kPfLanes = VEC == 1 ? DFS_PF_LANES32 : DFS_PF_LANES128;
     extern __shared__ __align__(16) unsigned char smem_raw[];
     SmemCtl& S = *reinterpret_cast<SmemCtl*>(smem_raw);
     constexpr int kCtlBytes = (sizeof(SmemCtl) + 15) & ~15;
