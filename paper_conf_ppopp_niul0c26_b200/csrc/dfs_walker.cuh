@@ -73,7 +73,10 @@ __global__ void __launch_bounds__(1024, 1) dfs_walker_kernel(const KParams P) {
     static_assert((H & (H - 1)) == 0 && H >= 32 && H <= 1024, "H is a power of two in [32, 1024]");
     constexpr int WPW = 32 / G;                       // walkers per warp
     constexpr uint32_t GM = (1u << G) - 1u;
-    constexpr int kPf = G < 8 ? G : 8;                // lanes prefetching candidates' row_ptr pairs
+#ifndef DFS_WALKER_PF
+#define DFS_WALKER_PF 8
+#endif
+    constexpr int kPf = G < DFS_WALKER_PF ? G : DFS_WALKER_PF;   // lanes prefetching candidates' row_ptr pairs
     constexpr uint32_t kStealMax = H / 4;             // entries per steal (ring space, see refill)
     extern __shared__ __align__(16) unsigned char smem_raw[];
     SmemW& S = *reinterpret_cast<SmemW*>(smem_raw);
