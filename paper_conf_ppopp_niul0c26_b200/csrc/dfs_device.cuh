@@ -493,9 +493,6 @@ __global__ void __launch_bounds__(32 * WMAX, 1) dfs_persistent_kernel(const KPar
     constexpr uint32_t kBatch = H / 2;              // flush batch (reading S10)
     constexpr uint32_t kWin = 32u * VEC;            // positions per window
     constexpr int kHeadLanes = VEC == 1 ? 8 : 16;   // lanes fetched before a window's end is known
-#ifndef DFS_SEQPF
-#define DFS_SEQPF 0
-#endif
 #ifndef DFS_PF_LANES128
 #define DFS_PF_LANES128 0
 #endif
@@ -1020,15 +1017,6 @@ __global__ void __launch_bounds__(32 * WMAX, 1) dfs_persistent_kernel(const KPar
                     if (ni < end) {
                         if (!push_lean(u, ni)) goto exit_loop;
                     }
-#if DFS_SEQPF
-                    // sequential descent (v = u + 1, paths and spines with consecutive ids): the
-                    // next vertices' adjacency follows v's in col_idx and their row_ptr entries
-                    // follow v's — prefetch both into L2 ahead of the dependent chain
-                    if (v == u + 1u) {
-                        if (lane < DFS_SEQPF) asm volatile("prefetch.global.L2 [%0];" ::"l"(P.col + vre + 32u * lane));
-                        else if (lane == DFS_SEQPF) asm volatile("prefetch.global.L2 [%0];" ::"l"(P.rp + v + 8u));
-                    }
-#endif
                     par = u;
                     u = v; i = vrs; end = vre; spec_ok = spec_on;
                     nbv[0] = cnb; win_lanes = 32;                      // have_win stays true
