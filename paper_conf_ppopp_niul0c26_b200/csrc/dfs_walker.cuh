@@ -74,9 +74,12 @@ __global__ void __launch_bounds__(1024, 1) dfs_walker_kernel(const KParams P) {
     constexpr int WPW = 32 / G;                       // walkers per warp
     constexpr uint32_t GM = (1u << G) - 1u;
 #ifndef DFS_WALKER_PF
-#define DFS_WALKER_PF 8
+#define DFS_WALKER_PF 0
 #endif
-    constexpr int kPf = G < DFS_WALKER_PF ? G : DFS_WALKER_PF;   // lanes prefetching candidates' row_ptr pairs
+    // lanes prefetching their candidates' row_ptr pairs with the probes: none (round 2 A/B:
+    // path 10^8 7.21 -> 6.67 ms, batch neutral; profiles/r02/ab/walker_pf.jsonl) — a candidate
+    // claim loads its pair beside the claim atomic instead
+    constexpr int kPf = G < DFS_WALKER_PF ? G : DFS_WALKER_PF;
     constexpr uint32_t kStealMax = H / 4;             // entries per steal (ring space, see refill)
     extern __shared__ __align__(16) unsigned char smem_raw[];
     SmemW& S = *reinterpret_cast<SmemW*>(smem_raw);
