@@ -1087,7 +1087,10 @@ __global__ void __launch_bounds__(32 * WMAX, 1) dfs_persistent_kernel(const KPar
             // long list (hubs): the next window is pulled into L1 while this one's probes
             // resolve (a prefetch holds no registers; the window is loaded when it is reached)
             const bool have_nxt = a + kWin < end;
-            if (have_nxt && a + kWin + (uint32_t)VEC * lane < end)
+#ifndef DFS_NEXTWIN_PF
+#define DFS_NEXTWIN_PF 1
+#endif
+            if (DFS_NEXTWIN_PF && have_nxt && a + kWin + (uint32_t)VEC * lane < end)
                 asm volatile("prefetch.global.L1 [%0];" ::"l"(P.col + a + kWin + (uint32_t)VEC * lane));
             // speculative claim: the first valid position whose neighbour is not the parent we
             // came from (par = kFull: none to skip) is, if unvisited, exactly Alg 1's next tree
