@@ -173,10 +173,11 @@ typedef struct dfs_options {
     int32_t donate;          /* walker kernel: 1 (default) = a walker about to push an entry while a
                                 sibling walker of its warp holds nothing hands the entry to that
                                 sibling instead; 0 = always push                    */
-    int32_t records;         /* walker kernel with >= 8 lanes: 1 (default) = read a claimed child's
-                                list through its 32-byte vertex record (first 6 neighbours + its
+    int32_t records;         /* walker kernel with >= 8 lanes: 1 = read a claimed child's list
+                                through its 32-byte vertex record (first 6 neighbours + its
                                 row_ptr pair; built once per handle on first use, 32 bytes per
-                                vertex of device memory); 0 = row_ptr then col_idx   */
+                                vertex of device memory; DESIGN.md §4 — measured slower); 0
+                                (default) = row_ptr then col_idx                                   */
 } dfs_options;
 
 typedef struct dfs_stats {

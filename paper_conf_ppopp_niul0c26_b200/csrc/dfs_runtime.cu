@@ -234,7 +234,7 @@ void dfs_options_default(dfs_options* o) {
     o->steal_tries = 8;          // A/B on B200: road 16.8 -> 15.4 ms, grid -15%, others neutral
     o->bulk_copy = 1;            // A/B on B200: rmat24 -11%, caterpillar -18%, road -2%, path -1%
     o->donate = 1;               // walker kernel: hand pushed entries to idle sibling walkers
-    o->records = 1;              // walker kernel (>= 8 lanes): vertex records
+    o->records = 0;              // walker kernel (>= 8 lanes): vertex records — measured slower
 }
 
 int dfs_last_error(void) { return g_last_error; }
