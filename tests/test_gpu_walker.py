@@ -75,7 +75,7 @@ def test_walker_tree_inputs_bit_exact(lanes, name, build, roots):
     dict(inter_steal=False), dict(intra_steal=False), dict(blocks=3, warps_per_block=2),
     dict(blocks=1), dict(warps_per_block=1, blocks=5), dict(victim_policy=0), dict(speculate=0),
     dict(speculate=1), dict(leaf_skip=0), dict(leaf_skip=1), dict(pub_batch=4), dict(spill_period=1),
-    dict(records=0), dict(records=0, ring_cap=3), dict(donate=0), dict(donate=0, steal_period=1024),
+    dict(records=1), dict(records=1, ring_cap=3), dict(donate=0), dict(donate=0, steal_period=1024),
 ])
 def test_walker_stress(lanes, opts):
     g = graphgen.road(300, 200, seed=7)
