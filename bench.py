@@ -269,10 +269,19 @@ def main():
 
     import torch
     import torch.distributed as dist
-    torch.cuda.set_device(local)
+    # one rank per GPU over NCCL.  DFS_BENCH_BACKEND=gloo (test aid only: exercises the N > 1 code
+    # paths with several ranks sharing the GPUs of a smaller box; collectives on host tensors)
+    backend = os.environ.get("DFS_BENCH_BACKEND", "nccl")
+    gpu = local % max(1, torch.cuda.device_count()) if backend != "nccl" else local
+    torch.cuda.set_device(gpu)
     if world > 1:
-        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
-    dev = torch.device("cuda", local)
+        if backend == "nccl":
+            dist.init_process_group("nccl", device_id=torch.device("cuda", gpu))
+        else:
+            dist.init_process_group(backend)
+    dev = torch.device("cuda", gpu)
+    a.coll_dev = dev if backend == "nccl" else torch.device("cpu")
+    a.gpu = gpu
     import graphgen
 
     if a.config == "batch1024":
@@ -355,7 +364,7 @@ def single_root_leg(a, workload, g, root0, undirected, desc, world, rank, local,
 
     ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(steps)]
     trav_ms = []
-    clocks = ClockSampler(local).start()
+    clocks = ClockSampler(getattr(a, "gpu", local)).start()
     launches0 = G.launch_count()
     if world > 1:
         dist.barrier()
@@ -386,7 +395,7 @@ def single_root_leg(a, workload, g, root0, undirected, desc, world, rank, local,
 
     from paper_conf_ppopp_niul0c26_b200 import batch
     (t_job, _), (edges,) = batch.reduce_max_sum([my_time, my_trav], [float(my_edges)], world,
-                                                device=torch.device("cuda", local))
+                                                device=a.coll_dev)
     if rank != 0:
         G.close()
         return None
@@ -467,7 +476,7 @@ def batch_leg(a, g, world, rank, local, dev):
     sub = 8                                                   # rows per gather round
     sink = None
     if world > 1 and rank == 0 and not a.no_gather:
-        sink = [torch.empty((sub, g.n), dtype=torch.int32, device=dev) for _ in range(world)]
+        sink = [torch.empty((sub, g.n), dtype=torch.int32, device=a.coll_dev) for _ in range(world)]
 
     lanes = []
 
@@ -486,15 +495,16 @@ def batch_leg(a, g, world, rank, local, dev):
                 counts.append(st.root_counts.copy())
                 lanes.append(st.walker_lanes)
             if gather and world > 1:
-                batch.gather_chunk_to_rank0(out_rows, len(chunk), min(rows, cap - c0), sub, sink, world, rank)
+                src_rows = out_rows if a.coll_dev.type == "cuda" else out_rows.cpu()
+                batch.gather_chunk_to_rank0(src_rows, len(chunk), min(rows, cap - c0), sub, sink, world, rank)
         e1.record()
         torch.cuda.synchronize()
         ms = e0.elapsed_time(e1)
         launches = G.launch_count() - launches0
-        (t_max,), _ = batch.reduce_max_sum([ms], [], world, device=dev)
+        (t_max,), _ = batch.reduce_max_sum([ms], [], world, device=a.coll_dev)
         return t_max, ms, np.concatenate(counts) if counts else np.zeros((0, 2)), launches
 
-    clocks = ClockSampler(local).start()
+    clocks = ClockSampler(getattr(a, "gpu", local)).start()
     t_trav, my_ms, counts, launches = one_pass(False)
     t_gath = None
     if not a.no_gather and world > 1:
@@ -513,7 +523,7 @@ def batch_leg(a, g, world, rank, local, dev):
             assert res.ok, (r, res)
             vals.append(int(res.ok))
     _, (tot_bytes, tot_edges, nval, nok) = batch.reduce_max_sum(
-        [], [my_bytes, my_edges, float(len(vals)), float(sum(vals))], world, device=dev)
+        [], [my_bytes, my_edges, float(len(vals)), float(sum(vals))], world, device=a.coll_dev)
     # e2e: the public C symbol dfs_run_batch with HOST buffers (roots in host memory, parent rows
     # into pinned host memory), wall clock with a device sync on both sides; a bounded sample of
     # E roots per rank (the full 1,024 x 96 MB of rows would not fit in host memory)
@@ -536,7 +546,7 @@ def batch_leg(a, g, world, rank, local, dev):
         el = time.perf_counter() - t0
         assert rc == 0, rc
         del hout
-        (el_max,), (roots_all,) = batch.reduce_max_sum([el], [float(E)], world, device=dev)
+        (el_max,), (roots_all,) = batch.reduce_max_sum([el], [float(E)], world, device=a.coll_dev)
         e2e = {"value": round(roots_all / el_max, 3), "unit": "DFS/s", "h2d_bytes_per_step": int(E * 4),
                "d2h_bytes_per_step": int(E * g.n * 4), "roots_per_rank": E,
                "what": f"dfs_run_batch(resident graph, {E} host roots, pinned host parents_out) per rank; "
