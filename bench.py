@@ -469,7 +469,14 @@ def batch_leg(a, g, world, rank, local, dev):
         opts["concurrency"] = a.concurrency
     o = Options(**opts)
     cap = max(b - a_ for a_, b in (batch.partition(k, world, p) for p in range(world)))
-    rows = max(1, min(128, cap))                              # same on every rank
+    # rows per dfs_run_batch call: up to 512 (fewer call boundaries, each of which waits for the
+    # slowest in-flight traversal), bounded by 40% of the free device memory; the same on every rank
+    free_b, _ = torch.cuda.mem_get_info()
+    rows_fit = max(8, int(0.4 * free_b // (g.n * 4)))
+    if world > 1:
+        (rows_fit_min,), _ = batch.reduce_max_sum([-float(rows_fit)], [], world, device=a.coll_dev)
+        rows_fit = int(-rows_fit_min)
+    rows = max(1, min(512, cap, rows_fit))
     out_rows = torch.empty((rows, g.n), dtype=torch.int32, device=dev)
     G.run_batch(mine[:min(rows, 8)], out=out_rows[:min(rows, 8)], options=o)      # warm-up
     torch.cuda.synchronize()

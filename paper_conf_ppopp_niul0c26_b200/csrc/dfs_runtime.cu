@@ -14,6 +14,7 @@
 #include <cstdlib>
 #include <cstring>
 #include <new>
+#include <thread>
 #include <vector>
 
 #include "../../include/dfs.h"
@@ -109,6 +110,8 @@ struct Slot {
     bool tab_dirty = false;
     cudaStream_t stream = nullptr;          // own stream (slots >= 1 of a concurrent batch)
     cudaEvent_t ev0 = nullptr, ev1 = nullptr, evk0 = nullptr, evk1 = nullptr;
+    cudaEvent_t evq[2] = {nullptr, nullptr};   // completion of the last two traversals issued (batches)
+    int64_t issued = 0;                        // traversals issued on this slot in the current batch
 };
 
 }  // namespace
@@ -146,6 +149,8 @@ static void free_slot(Slot& s) {
     if (s.ev1) cudaEventDestroy(s.ev1);
     if (s.evk0) cudaEventDestroy(s.evk0);
     if (s.evk1) cudaEventDestroy(s.evk1);
+    if (s.evq[0]) cudaEventDestroy(s.evq[0]);
+    if (s.evq[1]) cudaEventDestroy(s.evq[1]);
     s = Slot();
 }
 
@@ -188,6 +193,8 @@ static int ensure_slot(dfs_graph* g, int k, int64_t n_warps) {
     if (!ok) { cudaGetLastError(); free_slot(s); return DFS_ENOMEM; }
     if (cudaEventCreate(&s.ev0) != cudaSuccess || cudaEventCreate(&s.ev1) != cudaSuccess ||
         cudaEventCreate(&s.evk0) != cudaSuccess || cudaEventCreate(&s.evk1) != cudaSuccess ||
+        cudaEventCreateWithFlags(&s.evq[0], cudaEventDisableTiming) != cudaSuccess ||
+        cudaEventCreateWithFlags(&s.evq[1], cudaEventDisableTiming) != cudaSuccess ||
         (k > 0 && cudaStreamCreateWithFlags(&s.stream, cudaStreamNonBlocking) != cudaSuccess)) {
         cudaGetLastError(); free_slot(s); return DFS_ECUDA;
     }
@@ -811,22 +818,43 @@ static int run_concurrent(dfs_graph* g, const int32_t* roots, int32_t k, int32_t
         cudaMemsetAsync(sl.status, 0, sizeof(int), sl.stream);
         cudaMemsetAsync(sl.count2, 0, 2 * sizeof(unsigned long long), sl.stream);
     }
-    for (int32_t q = 0; q < k; ++q) {
-        Slot& sl = g->slots[q % conc];
-        int32_t* d_out = out_dev ? out + (size_t)q * g->n : sl.parent;
-        int rc = launch_one(g, sl, sl.stream, roots[q], d_out, o, blocks, warps, false, false);
-        if (rc != DFS_OK) return fail(rc);
-        if (stats) {
-            dfs_count_kernel<<<g->sms * 4, 256, 0, sl.stream>>>(sl.bitmap, sl.bstride, g->d_rp, (uint32_t)g->n, g->d_counts + 2 * q);
-            g->launches++;
-        }
-        if (!out_dev) {
-            if (cudaMemcpyAsync(out + (size_t)q * g->n, sl.parent, (size_t)g->n * sizeof(int32_t),
-                                cudaMemcpyDeviceToHost, sl.stream) != cudaSuccess) {
-                cudaGetLastError();
-                return fail(DFS_ECUDA);
+    // dynamic issue: a root goes to whichever slot has room in its two-deep queue (the traversal
+    // issued two earlier on it has completed), so slots that draw short traversals take more
+    // roots and the batch does not end waiting for the slot that drew the long ones
+    for (int c = 0; c < conc; ++c) g->slots[c].issued = 0;
+    int32_t q = 0;
+    int rr = 0;                                          // round-robin start of the next sweep
+    while (q < k) {
+        bool any = false;
+        for (int t = 0; t < conc && q < k; ++t) {
+            const int c = (rr + t) % conc;
+            Slot& sl = g->slots[c];
+            if (sl.issued >= 2) {
+                const cudaError_t qe = cudaEventQuery(sl.evq[sl.issued & 1]);
+                if (qe == cudaErrorNotReady) continue;
+                if (qe != cudaSuccess) { cudaGetLastError(); return fail(DFS_ECUDA); }
             }
+            int32_t* d_out = out_dev ? out + (size_t)q * g->n : sl.parent;
+            int rc = launch_one(g, sl, sl.stream, roots[q], d_out, o, blocks, warps, false, false);
+            if (rc != DFS_OK) return fail(rc);
+            if (stats) {
+                dfs_count_kernel<<<g->sms * 4, 256, 0, sl.stream>>>(sl.bitmap, sl.bstride, g->d_rp, (uint32_t)g->n, g->d_counts + 2 * q);
+                g->launches++;
+            }
+            if (!out_dev) {
+                if (cudaMemcpyAsync(out + (size_t)q * g->n, sl.parent, (size_t)g->n * sizeof(int32_t),
+                                    cudaMemcpyDeviceToHost, sl.stream) != cudaSuccess) {
+                    cudaGetLastError();
+                    return fail(DFS_ECUDA);
+                }
+            }
+            cudaEventRecord(sl.evq[sl.issued & 1], sl.stream);
+            ++sl.issued;
+            ++q;
+            any = true;
+            rr = (c + 1) % conc;
         }
+        if (!any) std::this_thread::yield();
     }
     // join
     for (int c = 0; c < conc; ++c) {
