@@ -788,7 +788,8 @@ static int run_sequential(dfs_graph* g, const int32_t* roots, int32_t k, int32_t
 // concurrent path (§8(f)-2): `conc` slots, each on its own stream and a 1/conc share of the
 // SMs, take roots round-robin; no host synchronisation until the whole batch is issued
 static int run_concurrent(dfs_graph* g, const int32_t* roots, int32_t k, int32_t* out, bool out_dev,
-                          const dfs_options& o, int blocks, int warps, int conc, dfs_stats* stats) {
+                          const dfs_options& o, int blocks, int warps, int conc, dfs_stats* stats,
+                          int extra = 0) {
     for (int c = 0; c < conc; ++c) {
         Slot& sl = g->slots[c];
         if (sl.block_claims) { cudaFree(sl.block_claims); sl.block_claims = nullptr; }
@@ -835,7 +836,8 @@ static int run_concurrent(dfs_graph* g, const int32_t* roots, int32_t k, int32_t
                 if (qe != cudaSuccess) { cudaGetLastError(); return fail(DFS_ECUDA); }
             }
             int32_t* d_out = out_dev ? out + (size_t)q * g->n : sl.parent;
-            int rc = launch_one(g, sl, sl.stream, roots[q], d_out, o, blocks, warps, false, false);
+            // the first `extra` slots take one more block: all SMs in use (148 = 4 x 19 + 4 x 18)
+            int rc = launch_one(g, sl, sl.stream, roots[q], d_out, o, blocks + (c < extra ? 1 : 0), warps, false, false);
             if (rc != DFS_OK) return fail(rc);
             if (stats) {
                 dfs_count_kernel<<<g->sms * 4, 256, 0, sl.stream>>>(sl.bitmap, sl.bstride, g->d_rp, (uint32_t)g->n, g->d_counts + 2 * q);
@@ -905,7 +907,7 @@ static int run_many(dfs_graph* g, const int32_t* roots_host, int32_t k, int32_t*
     while (conc > 1) {
         int c = 0;
         rc = DFS_OK;
-        const int64_t owners = (int64_t)blocks * warps * (o.walker_lanes == 32 ? 1 : 32 / o.walker_lanes);
+        const int64_t owners = (int64_t)(blocks + (auto_blocks ? 1 : 0)) * warps * (o.walker_lanes == 32 ? 1 : 32 / o.walker_lanes);
         for (; c < conc; ++c) {
             rc = ensure_slot(g, c, c == 0 ? std::max<int64_t>(owners, (int64_t)g->max_blocks * kMaxWarps) : owners);
             if (rc != DFS_OK) break;
@@ -930,7 +932,8 @@ static int run_many(dfs_graph* g, const int32_t* roots_host, int32_t k, int32_t*
         }
         registered = true;
     }
-    rc = run_concurrent(g, roots_host, k, out, out_dev, o, blocks, warps, conc, stats);
+    const int extra = auto_blocks ? std::max(0, g->max_blocks - blocks * conc) : 0;
+    rc = run_concurrent(g, roots_host, k, out, out_dev, o, blocks, warps, conc, stats, extra);
     if (registered) { cudaHostUnregister(out); cudaGetLastError(); }
     return rc;
 }
