@@ -67,7 +67,10 @@ __device__ __forceinline__ unsigned long long ld_shared_u64_if(bool p, const uns
 // blockIdx.x * (W * 32 / G) + warp * (32 / G) + walker.
 // ------------------------------------------------------------------------------------------
 template <int G, int H, bool STATS, bool REC>
-__global__ void __launch_bounds__(1024, 1) dfs_walker_kernel(const KParams P) {
+#ifndef DFS_WALKER_LB
+#define DFS_WALKER_LB 1024
+#endif
+__global__ void __launch_bounds__(DFS_WALKER_LB, 1) dfs_walker_kernel(const KParams P) {
     static_assert(G == 2 || G == 4 || G == 8 || G == 16, "G is 2, 4, 8 or 16");
     static_assert(!REC || G >= 8, "a vertex record spans 8 lanes");
     static_assert((H & (H - 1)) == 0 && H >= 32 && H <= 1024, "H is a power of two in [32, 1024]");
