@@ -43,7 +43,11 @@ bool is_device_ptr(const void* p) {
 
 // the 24 instantiations of the persistent kernel: [bulk][cluster tier][vec128][wmax16][stats]
 // (the bulk variants without the cluster tier)
-#define DFS_K(V, W, S, C, B) (const void*)dfs_persistent_kernel<kRing, V, W, S, C, B>
+// DFS_WMAX_BIG: warps per CTA of the large instantiations (32: 64 registers per thread)
+#ifndef DFS_WMAX_BIG
+#define DFS_WMAX_BIG 32
+#endif
+#define DFS_K(V, W, S, C, B) (const void*)dfs_persistent_kernel<kRing, V, (W == 32 ? DFS_WMAX_BIG : W), S, C, B>
 const void* const* kernel_table() {
     static const void* const t[24] = {
         DFS_K(1, 32, false, false, false), DFS_K(1, 32, true, false, false), DFS_K(1, 16, false, false, false), DFS_K(1, 16, true, false, false),
@@ -80,6 +84,7 @@ int walker_index(int lanes, bool rec) {
     return lanes == 16 ? 0 : lanes == 8 ? 2 : lanes == 4 ? 4 : 6;
 }
 bool valid_walker_lanes(int lanes) { return lanes == 16 || lanes == 8 || lanes == 4 || lanes == 2; }
+constexpr int kWalkerMaxWarps = DFS_WALKER_LB / 32;
 
 size_t smem_bytes(int warps) {
     return ((sizeof(SmemCtl) + 15) & ~size_t(15)) + (size_t)warps * kRing * sizeof(unsigned long long);
@@ -286,7 +291,7 @@ dfs_graph* dfs_graph_create(const int64_t* row_ptr, const int32_t* col_idx, int6
     }
     if (!attr_ok) { cudaGetLastError(); delete g; fail(DFS_ECUDA); return nullptr; }
     int per_sm = 0;
-    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, dfs_persistent_kernel<kRing, 4, 32, false, false, false>, 1024, sm32) !=
+    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, dfs_persistent_kernel<kRing, 4, DFS_WMAX_BIG, false, false, false>, 32 * DFS_WMAX_BIG, sm32) !=
             cudaSuccess || per_sm < 1) {
         cudaGetLastError(); per_sm = 1;
     }
@@ -537,7 +542,7 @@ static int max_clusters(dfs_graph* g, int cl, int warps, int window, bool stats)
     cudaLaunchAttribute at[1];
     at[0].id = cudaLaunchAttributeClusterDimension;
     at[0].val.clusterDim.x = (unsigned)cl; at[0].val.clusterDim.y = 1; at[0].val.clusterDim.z = 1;
-    cfg.gridDim = dim3((unsigned)(g->max_blocks / cl * cl)); cfg.blockDim = dim3(1024);
+    cfg.gridDim = dim3((unsigned)(g->max_blocks / cl * cl)); cfg.blockDim = dim3(32 * DFS_WMAX_BIG);
     cfg.dynamicSmemBytes = smem_bytes(32); cfg.attrs = at; cfg.numAttrs = 1;
     int n = 0;
     if (cudaOccupancyMaxActiveClusters(&n, kfn, &cfg) != cudaSuccess) { cudaGetLastError(); n = 0; }
@@ -590,6 +595,11 @@ static int resolve_options(dfs_graph* g, const dfs_options* in, int num_roots, d
     if (o.concurrency < 0 || o.concurrency > kMaxSlots) return DFS_EINVAL;
     warps = o.warps_per_block <= 0 ? 32 : o.warps_per_block;
     if (warps > 32) return DFS_EINVAL;
+    // the walker kernel is compiled for CTAs of up to kWalkerMaxWarps warps (DFS_WALKER_LB threads:
+    // 28 warps x 72 registers measured faster than 32 x 64 — fewer register rematerialisations;
+    // DESIGN.md §5); auto and larger requests get that
+    if (o.walker_lanes != 32 && warps > kWalkerMaxWarps) warps = kWalkerMaxWarps;
+    if (o.walker_lanes == 32 && warps > DFS_WMAX_BIG) warps = DFS_WMAX_BIG;
     conc = o.concurrency == 0 ? 8 : o.concurrency;       // auto: 8 in flight (B200 sweep)
     if (o.deterministic) conc = 1;
     if (conc > num_roots) conc = std::max(1, num_roots);

@@ -25,6 +25,11 @@
 namespace b200dfs {
 
 constexpr int kMaxWalkersPerCta = 512;
+// CTA size the walker kernel is compiled for (threads): 28 warps x 72 registers (round-2 sweep,
+// DESIGN.md §5); the runtime launches it with at most DFS_WALKER_LB / 32 warps
+#ifndef DFS_WALKER_LB
+#define DFS_WALKER_LB 896
+#endif
 #ifndef DFS_WALKER_FULLSCAN
 #define DFS_WALKER_FULLSCAN 0
 #endif
@@ -67,9 +72,6 @@ __device__ __forceinline__ unsigned long long ld_shared_u64_if(bool p, const uns
 // blockIdx.x * (W * 32 / G) + warp * (32 / G) + walker.
 // ------------------------------------------------------------------------------------------
 template <int G, int H, bool STATS, bool REC>
-#ifndef DFS_WALKER_LB
-#define DFS_WALKER_LB 1024
-#endif
 __global__ void __launch_bounds__(DFS_WALKER_LB, 1) dfs_walker_kernel(const KParams P) {
     static_assert(G == 2 || G == 4 || G == 8 || G == 16, "G is 2, 4, 8 or 16");
     static_assert(!REC || G >= 8, "a vertex record spans 8 lanes");
