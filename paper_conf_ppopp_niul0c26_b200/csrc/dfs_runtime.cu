@@ -942,7 +942,8 @@ static int run_many(dfs_graph* g, const int32_t* roots_host, int32_t k, int32_t*
         }
         registered = true;
     }
-    const int extra = auto_blocks ? std::max(0, g->max_blocks - blocks * conc) : 0;
+    // (not with the cluster tier: its grids are whole clusters)
+    const int extra = (auto_blocks && o.cluster < 1) ? std::max(0, g->max_blocks - blocks * conc) : 0;
     rc = run_concurrent(g, roots_host, k, out, out_dev, o, blocks, warps, conc, stats, extra);
     if (registered) { cudaHostUnregister(out); cudaGetLastError(); }
     return rc;
