@@ -1,0 +1,8 @@
+# round-2 session 2: re-verify the last committed build (smoke, all GPU tests, default bench)
+set -x
+nvidia-smi --query-gpu=name,clocks.sm,clocks.max.sm --format=csv
+python -c "import __graft_entry__ as g; g.smoke()" > gpurun_out/smoke.log 2>&1; echo smoke rc=$?
+timeout 1500 python -m pytest tests -m gpu -q -rf --timeout 600 --durations=10 > gpurun_out/pytest_gpu.log 2>&1; echo pytest rc=$?
+tail -4 gpurun_out/pytest_gpu.log
+timeout 900 python bench.py --steps 20 --warmup 5 > gpurun_out/bench.json 2> gpurun_out/bench.err; echo bench rc=$?
+tail -3 gpurun_out/bench.err
