@@ -113,8 +113,6 @@ struct KParams {
     uint32_t period_mask;                    // spill_period - 1
     uint32_t steal_period_mask;              // walker kernel: steal_period - 1
     int donate;                              // walker kernel: hand pushed entries to idle siblings
-    const uint2* __restrict__ adj;           // edge-annotated adjacency (32-wide windows, DFS_ADJ):
-                                             // adj[j] = {col_idx[j], row_ptr[col_idx[j]]} (+32 padding)
     const uint32_t* __restrict__ rec;        // vertex records (8 words per vertex: col[rp[v] .. +6),
                                              // rp[v], rp[v+1]; padding kFull), or null
     const int32_t* script;                   // walker STATS kernel: stack-script mode (tests), or null
@@ -122,12 +120,6 @@ struct KParams {
     int32_t* script_out;
     int script_out_len;
 };
-
-// DFS_ADJ = 1: the 32-wide step reads the edge-annotated adjacency instead of col_idx + row_ptr
-// (A/B build; measured neutral on road and 21% slower on the caterpillar)
-#ifndef DFS_ADJ
-#define DFS_ADJ 0
-#endif
 
 // vertex records (create time, on first use): record v = 8 words = one 32-byte
 // sector: the first 6 entries of v's adjacency list (kFull past its end), then row_ptr[v] and
@@ -143,23 +135,6 @@ __global__ void dfs_records_kernel(const uint32_t* __restrict__ rp, const int32_
         for (int k = 0; k < 6; ++k) w[k] = s + k < e ? (uint32_t)col[s + k] : kFull;
         rec[2 * v] = make_uint4(w[0], w[1], w[2], w[3]);
         rec[2 * v + 1] = make_uint4(w[4], w[5], s, e);
-    }
-}
-
-// edge-annotated adjacency (create time, on first use of the 32-wide warp kernel):
-// adj[j] = {col_idx[j], row_ptr[col_idx[j]]} for j < m, then 32 padding entries {kFull, 0} so a
-// window's head lanes may read past the last list.  The 32-wide step issues a claimed child's
-// window load with its claim: the window address arrives with the child's id.
-__global__ void dfs_adj_kernel(const uint32_t* __restrict__ rp, const int32_t* __restrict__ col, uint32_t m,
-                               uint2* __restrict__ adj) {
-    const size_t stride = (size_t)gridDim.x * blockDim.x;
-    for (size_t j = blockIdx.x * (size_t)blockDim.x + threadIdx.x; j < (size_t)m + 32; j += stride) {
-        if (j < m) {
-            const uint32_t x = (uint32_t)col[j];
-            adj[j] = make_uint2(x, rp[x]);
-        } else {
-            adj[j] = make_uint2(kFull, 0u);
-        }
     }
 }
 
@@ -239,12 +214,6 @@ __device__ __forceinline__ uint32_t ld_cg_if(bool p, const uint32_t* a, uint32_t
 __device__ __forceinline__ uint2 ld_cg_u2_if(bool p, const uint32_t* a, uint32_t dx, uint32_t dy) {
     uint2 r = make_uint2(dx, dy);
     asm volatile("{ .reg .pred q; setp.ne.u32 q, %2, 0; @q ld.global.cg.v2.u32 {%0, %1}, [%3]; }"
-                 : "+r"(r.x), "+r"(r.y) : "r"((uint32_t)p), "l"(a));
-    return r;
-}
-__device__ __forceinline__ uint2 ld_nc_u2_if(bool p, const uint2* a, uint32_t dx, uint32_t dy) {
-    uint2 r = make_uint2(dx, dy);
-    asm volatile("{ .reg .pred q; setp.ne.u32 q, %2, 0; @q ld.global.nc.v2.u32 {%0, %1}, [%3]; }"
                  : "+r"(r.x), "+r"(r.y) : "r"((uint32_t)p), "l"(a));
     return r;
 }
@@ -535,10 +504,6 @@ __global__ void __launch_bounds__(32 * WMAX, 1) dfs_persistent_kernel(const KPar
 #define DFS_PF_LANES32 8
 #endif
     constexpr int kPfLanes = VEC == 1 ? DFS_PF_LANES32 : DFS_PF_LANES128;
-    // edge-annotated adjacency for 32-wide windows: the window entry of a neighbour
-    // carries the start of its list, so a claimed child's window load is issued with the claim
-    // instead of after a dependent row_ptr load (one dependent load per DFS level, not two)
-    constexpr bool kAdj = DFS_ADJ && VEC == 1;
     extern __shared__ __align__(16) unsigned char smem_raw[];
     SmemCtl& S = *reinterpret_cast<SmemCtl*>(smem_raw);
     constexpr int kCtlBytes = (sizeof(SmemCtl) + 15) & ~15;
@@ -584,7 +549,6 @@ __global__ void __launch_bounds__(32 * WMAX, 1) dfs_persistent_kernel(const KPar
     bool need_end = false;       // end must be re-read from row_ptr
     uint32_t u = 0, i = 0, end = 0;
     int nbv[VEC];                // this lane's neighbours in the current window
-    uint32_t nbs = 0;            // kAdj: start of this lane's neighbour's list (row_ptr[nbv[0]])
 #pragma unroll
     for (int e = 0; e < VEC; ++e) nbv[e] = -1;
     uint32_t my_head = 0;        // owner's true HotRing head (16-bit wrap)
@@ -630,17 +594,6 @@ __global__ void __launch_bounds__(32 * WMAX, 1) dfs_persistent_kernel(const KPar
             nb[0] = x.x; nb[1] = x.y; nb[2] = x.z; nb[3] = x.w;
         } else {
             nb[0] = (int)ld_nc_if(ld, P.col + q, kFull);
-        }
-    };
-    // 32-wide window entry at CSR position q: the neighbour and, with the annotated adjacency,
-    // the start of its list
-    auto ldw = [&](bool p, uint32_t q, int& nb, uint32_t& ns) {
-        if constexpr (kAdj) {
-            const uint2 x = ld_nc_u2_if(p, P.adj + q, kFull, 0u);
-            nb = (int)x.x; ns = x.y;
-        } else {
-            nb = (int)ld_nc_if(p, P.col + q, kFull);
-            (void)ns;
         }
     };
     // lanes of the current window that hold data (the rest are loaded on demand)
@@ -962,20 +915,19 @@ __global__ void __launch_bounds__(32 * WMAX, 1) dfs_persistent_kernel(const KPar
                 if (!have_win) {
                     if (need_end) {                                   // popped entry: end unknown
                         const uint32_t e2 = __ldg(P.rp + u + 1);
-                        ldw(lane < kHeadLanes && i + lane < P.m, i + lane, nbv[0], nbs);
+                        nbv[0] = (int)ld_nc_if(lane < kHeadLanes && i + lane < P.m, P.col + i + lane, kFull);
                         win_lanes = kHeadLanes;
                         end = e2; need_end = false;
                     } else {
-                        ldw(i + lane < end, i + lane, nbv[0], nbs);
+                        nbv[0] = (int)ld_nc_if(i + lane < end, P.col + i + lane, kFull);
                         win_lanes = 32;
                     }
                     have_win = true;
                 }
                 if (win_lanes < 32) {
                     if (end > i + (uint32_t)win_lanes) {
-                        int t; uint32_t ts = 0;
-                        ldw(lane >= win_lanes && i + lane < end, i + lane, t, ts);
-                        if (lane >= win_lanes) { nbv[0] = t; nbs = ts; }
+                        const int t = (int)ld_nc_if(lane >= win_lanes && i + lane < end, P.col + i + lane, kFull);
+                        if (lane >= win_lanes) nbv[0] = t;
                     }
                     win_lanes = 32;
                 }
@@ -985,30 +937,22 @@ __global__ void __launch_bounds__(32 * WMAX, 1) dfs_persistent_kernel(const KPar
             const bool valid = i + (uint32_t)lane < end;
             // long list (hubs): the next window is in flight while this one's probes resolve
             const bool have_nxt = i + 32u < end;
-            int nxt1; uint32_t nxt1s = 0;
-            ldw(have_nxt && i + 32u + lane < end, i + 32u + lane, nxt1, nxt1s);
+            const int nxt1 = (int)ld_nc_if(have_nxt && i + 32u + lane < end, P.col + i + 32u + lane, kFull);
             // speculative claim (fresh child only): the first position whose neighbour is not the
             // parent we came from is, if unvisited, exactly Alg 1's next tree edge
             const uint32_t vb = __ballot_sync(kFull, spec_ok && valid && (uint32_t)nb != par);
             const int sk = __ffs(vb) - 1;
             const uint32_t sv = vb ? (uint32_t)__shfl_sync(kFull, nb, sk & 31) : u;
             uint32_t s_old = atom_or_if(vb != 0 && lane == 0, P.bitmap + 2u * (sv >> 5), 1u << (sv & 31));
-            // the child's list [s_rs, s_re): with the annotated adjacency its start came with the
-            // window (a shuffle) and only the end is loaded, in parallel with the child's window
-            const uint32_t s_rs = kAdj ? (uint32_t)__shfl_sync(kFull, nbs, sk & 31) : ld_nc_if(vb != 0, P.rp + sv, 0u);
-            const uint32_t s_re = ld_nc_if(vb != 0, P.rp + sv + 1, 0u);
+            const uint32_t s_rs = ld_nc_if(vb != 0, P.rp + sv, 0u), s_re = ld_nc_if(vb != 0, P.rp + sv + 1, 0u);
             // probe the visited bits; lanes holding the first 8 positions prefetch their
-            // candidates' row_ptr pairs (kAdj: only the ends)
+            // candidates' row_ptr pairs
             const uint2 wl = ld_cg_u2_if(valid, P.bitmap + 2u * ((uint32_t)nb >> 5), kFull, 0u);   // {visited, leaf}
             const bool pf = valid && lane < kPfLanes;
-            const uint32_t prs = kAdj ? nbs : ld_nc_if(pf, P.rp + nb, 0u), pre = ld_nc_if(pf, P.rp + nb + 1, 0u);
+            const uint32_t prs = ld_nc_if(pf, P.rp + nb, 0u), pre = ld_nc_if(pf, P.rp + nb + 1, 0u);
             // early child window (speculate & 4): issued once the row_ptr pair arrives, before
-            // the claim returns (the probes are already in flight); kAdj: issued at once for the
-            // first kHeadLanes positions (its end is not known yet; the rest on demand)
-            int cnb = kFull; uint32_t cnbs = 0;
-            if constexpr (kAdj) ldw(spec_early && vb != 0 && lane < kHeadLanes, s_rs + lane, cnb, cnbs);
-            else cnb = (int)ld_nc_if(spec_early && vb != 0 && s_rs + lane < s_re, P.col + s_rs + lane, kFull);
-            int cwl = kAdj && spec_early ? kHeadLanes : 32;          // lanes of cnb that hold data
+            // the claim returns (the probes are already in flight)
+            int cnb = (int)ld_nc_if(spec_early && vb != 0 && s_rs + lane < s_re, P.col + s_rs + lane, kFull);
             const bool unv = valid && !((wl.x >> (nb & 31)) & 1u) && lane != sk;   // sk is claimed either way
             const bool lf = unv && ((wl.y >> (nb & 31)) & 1u);
             bool cand = unv && !lf;
@@ -1033,7 +977,7 @@ __global__ void __launch_bounds__(32 * WMAX, 1) dfs_persistent_kernel(const KPar
             uint32_t v = sv, vrs = s_rs, vre = s_re;
             int kpos = sk;
             if (won) {
-                if (!spec_early) { ldw(vrs + lane < vre, vrs + lane, cnb, cnbs); cwl = 32; }
+                if (!spec_early) cnb = (int)ld_nc_if(vrs + lane < vre, P.col + vrs + lane, kFull);
             } else {
                 if (STATS && vb && lane == 0) ++cnt[kCntFailedClaims];
                 // claim the first unvisited candidate in CSR order; on a lost race try the next
@@ -1041,18 +985,11 @@ __global__ void __launch_bounds__(32 * WMAX, 1) dfs_persistent_kernel(const KPar
                 while (any) {
                     const int k = __ffs(any) - 1;
                     const uint32_t cv = (uint32_t)__shfl_sync(kFull, nb, k);
-                    uint32_t crs, cre = __shfl_sync(kFull, pre, k & (kPfLanes - 1));
-                    if constexpr (kAdj) {
-                        crs = (uint32_t)__shfl_sync(kFull, nbs, k);
-                        if (k >= kPfLanes) cre = __ldg(P.rp + cv + 1);
-                    } else {
-                        crs = __shfl_sync(kFull, prs, k & (kPfLanes - 1));
-                        if (k >= kPfLanes) { crs = __ldg(P.rp + cv); cre = __ldg(P.rp + cv + 1); }
-                    }
+                    uint32_t crs = __shfl_sync(kFull, prs, k & (kPfLanes - 1)), cre = __shfl_sync(kFull, pre, k & (kPfLanes - 1));
+                    if (k >= kPfLanes) { crs = __ldg(P.rp + cv); cre = __ldg(P.rp + cv + 1); }
                     const uint32_t bit = 1u << (cv & 31);
                     uint32_t old = atom_or_if(lane == 0, P.bitmap + 2u * (cv >> 5), bit);
-                    ldw(crs + lane < cre, crs + lane, cnb, cnbs);          // overlaps the claim
-                    cwl = 32;
+                    cnb = (int)ld_nc_if(crs + lane < cre, P.col + crs + lane, kFull);   // overlaps the claim
                     old = __shfl_sync(kFull, old, 0);
                     if (!(old & bit)) { won = true; v = cv; vrs = crs; vre = cre; kpos = k; break; }
                     if (STATS && lane == 0) ++cnt[kCntFailedClaims];
@@ -1082,7 +1019,7 @@ __global__ void __launch_bounds__(32 * WMAX, 1) dfs_persistent_kernel(const KPar
                     }
                     par = u;
                     u = v; i = vrs; end = vre; spec_ok = spec_on;
-                    nbv[0] = cnb; nbs = cnbs; win_lanes = cwl;         // have_win stays true
+                    nbv[0] = cnb; win_lanes = 32;                      // have_win stays true
                 }
             }
             if (advance) {
@@ -1092,14 +1029,11 @@ __global__ void __launch_bounds__(32 * WMAX, 1) dfs_persistent_kernel(const KPar
                 i = next_i;
                 if (i < end && d < 32u) {
                     int x = __shfl_down_sync(kFull, nb, d);
-                    const uint32_t xs = kAdj ? __shfl_down_sync(kFull, nbs, d) : 0u;
-                    int y; uint32_t ys = 0;
-                    ldw(lane >= 32 - (int)d && i + lane < end, i + lane, y, ys);
+                    const int y = (int)ld_nc_if(lane >= 32 - (int)d && i + lane < end, P.col + i + lane, kFull);
                     nbv[0] = lane >= 32 - (int)d ? y : x;
-                    if (kAdj) nbs = lane >= 32 - (int)d ? ys : xs;
                     spec_ok = spec_on; par = kFull;               // next position: claim at once
                 } else if (have_nxt) {                            // next window already loaded
-                    nbv[0] = nxt1; nbs = nxt1s;
+                    nbv[0] = nxt1;
                     spec_ok = false;
                 } else {
                     have_win = false;                             // i >= end: Alg 1 l.14: pop

@@ -137,8 +137,6 @@ struct dfs_graph {
     int32_t* d_col = nullptr;    // col_idx (+8 padding for 128-bit window loads)
     uint32_t* d_leaf = nullptr;  // leaf map: ceil(n/32) words (dfs_leaf_*_kernel)
     uint32_t* d_rec = nullptr;   // vertex records: 8 words per vertex (built on first use)
-    uint2* d_adj = nullptr;      // edge-annotated adjacency, m + 32 entries (built on first use
-                                 // of the 32-wide warp kernel)
     Slot slots[kMaxSlots];
     int64_t launches = 0;
     unsigned int* d_timeline = nullptr;   // diagnostics (dfs_debug_timeline)
@@ -166,7 +164,7 @@ static void free_graph(dfs_graph* g) {
     int cur = 0;
     cudaGetDevice(&cur);
     cudaSetDevice(g->device);
-    cudaFree(g->d_rp); cudaFree(g->d_col); cudaFree(g->d_leaf); cudaFree(g->d_rec); cudaFree(g->d_adj); cudaFree(g->d_timeline); cudaFree(g->d_counts);
+    cudaFree(g->d_rp); cudaFree(g->d_col); cudaFree(g->d_leaf); cudaFree(g->d_rec); cudaFree(g->d_timeline); cudaFree(g->d_counts);
     for (int k = 0; k < kMaxSlots; ++k) free_slot(g->slots[k]);
     cudaSetDevice(cur);
     delete g;
@@ -485,7 +483,6 @@ static int launch_one(dfs_graph* g, Slot& sl, cudaStream_t s, int32_t root, int3
     const int cl = o.cluster > 1 ? o.cluster : 1;
     // the cluster build has no bulk variant: cluster >= 1 takes precedence over bulk_copy
     P.rec = g->d_rec;
-    P.adj = g->d_adj;
     const bool rec = wl != 32 && wl >= 8 && o.records && g->d_rec;
     const void* kfn = wl != 32 ? walker_table()[walker_index(wl, rec) + (o.collect_stats ? 1 : 0)]
                                : kernel_table()[(o.cluster >= 1 ? 8 : o.bulk_copy ? 16 : 0) + (o.window == 128 ? 4 : 0) +
@@ -595,18 +592,6 @@ static int resolve_options(dfs_graph* g, const dfs_options* in, int num_roots, d
         if (cudaDeviceSynchronize() != cudaSuccess) { cudaGetLastError(); cudaFree(g->d_rec); g->d_rec = nullptr; return DFS_ECUDA; }
     }
     if (o.window != 32 && o.window != 128) return DFS_EINVAL;
-#if DFS_ADJ
-    if (o.walker_lanes == 32 && o.window == 32 && !g->d_adj) {
-        // edge-annotated adjacency for the 32-wide step (8 bytes per edge), built once per handle
-        if (cudaMalloc(&g->d_adj, ((size_t)g->m + 32) * sizeof(uint2)) != cudaSuccess) {
-            cudaGetLastError(); g->d_adj = nullptr; return DFS_ENOMEM;
-        }
-        const int blocks_a = (int)std::min<int64_t>((g->m + 32 + 255) / 256, (int64_t)g->sms * 16);
-        dfs_adj_kernel<<<blocks_a, 256>>>(g->d_rp, g->d_col, (uint32_t)g->m, g->d_adj);
-        g->launches++;
-        if (cudaDeviceSynchronize() != cudaSuccess) { cudaGetLastError(); cudaFree(g->d_adj); g->d_adj = nullptr; return DFS_ECUDA; }
-    }
-#endif
     if (o.concurrency < 0 || o.concurrency > kMaxSlots) return DFS_EINVAL;
     warps = o.warps_per_block <= 0 ? 32 : o.warps_per_block;
     if (warps > 32) return DFS_EINVAL;
