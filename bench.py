@@ -539,7 +539,7 @@ def batch_leg(a, g, world, rank, local, dev):
         import ctypes
         from paper_conf_ppopp_niul0c26_b200 import dfs as dfsmod
         lib = dfsmod.load_library()
-        E = min(16, len(mine))
+        E = min(64, len(mine))
         hroots = np.ascontiguousarray(np.array(mine[:E], dtype=np.int32))
         hout = torch.empty((max(E, 1), g.n), dtype=torch.int32).pin_memory()
         h = ctypes.c_void_p(G._h)

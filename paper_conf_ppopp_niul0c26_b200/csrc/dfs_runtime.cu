@@ -99,6 +99,11 @@ struct Slot {
     uint32_t* bitmap = nullptr;
     uint32_t bstride = 1;                   // bitmap layout of the last launch (1, or 2 = {visited, leaf})
     int32_t* parent = nullptr;              // lazily allocated for host outputs
+    int32_t* parent2 = nullptr;             // second row buffer: concurrent batches into host memory
+                                            // copy one row while the next traversal fills the other
+    cudaStream_t cstream = nullptr;         // device->host copies of the slot's rows (batches)
+    cudaEvent_t evt[2] = {nullptr, nullptr};   // traversal into buffer b done (copy may start)
+    cudaEvent_t evc[2] = {nullptr, nullptr};   // copy out of buffer b done (buffer reusable)
     unsigned long long* cold_tb = nullptr;
     uint32_t* tab = nullptr;
     unsigned long long* pool = nullptr;
@@ -146,10 +151,15 @@ struct dfs_graph {
 };
 
 static void free_slot(Slot& s) {
-    cudaFree(s.bitmap); cudaFree(s.parent); cudaFree(s.cold_tb); cudaFree(s.tab); cudaFree(s.pool);
+    cudaFree(s.bitmap); cudaFree(s.parent); cudaFree(s.parent2); cudaFree(s.cold_tb); cudaFree(s.tab); cudaFree(s.pool);
     cudaFree(s.consumed); cudaFree(s.next); cudaFree(s.block_cold); cudaFree(s.ctl); cudaFree(s.count2);
     cudaFree(s.status); cudaFree(s.block_claims);
     if (s.stream) cudaStreamDestroy(s.stream);
+    if (s.cstream) cudaStreamDestroy(s.cstream);
+    for (int b = 0; b < 2; ++b) {
+        if (s.evt[b]) cudaEventDestroy(s.evt[b]);
+        if (s.evc[b]) cudaEventDestroy(s.evc[b]);
+    }
     if (s.ev0) cudaEventDestroy(s.ev0);
     if (s.ev1) cudaEventDestroy(s.ev1);
     if (s.evk0) cudaEventDestroy(s.evk0);
@@ -803,11 +813,26 @@ static int run_concurrent(dfs_graph* g, const int32_t* roots, int32_t k, int32_t
     for (int c = 0; c < conc; ++c) {
         Slot& sl = g->slots[c];
         if (sl.block_claims) { cudaFree(sl.block_claims); sl.block_claims = nullptr; }
-        if (!out_dev && !sl.parent) {
-            if (cudaMalloc(&sl.parent, (size_t)g->n * sizeof(int32_t)) != cudaSuccess) {
+        if (!out_dev) {
+            // host rows: two device row buffers and a copy stream per slot, so the copy of one
+            // row overlaps the slot's next traversal (double buffering)
+            if ((!sl.parent && cudaMalloc(&sl.parent, (size_t)g->n * sizeof(int32_t)) != cudaSuccess) ||
+                (!sl.parent2 && cudaMalloc(&sl.parent2, (size_t)g->n * sizeof(int32_t)) != cudaSuccess)) {
                 cudaGetLastError();
                 return fail(DFS_ENOMEM);
             }
+            if (!sl.cstream) {
+                if (cudaStreamCreateWithFlags(&sl.cstream, cudaStreamNonBlocking) != cudaSuccess) {
+                    cudaGetLastError(); sl.cstream = nullptr; return fail(DFS_ECUDA);
+                }
+                for (int b = 0; b < 2; ++b) {
+                    if (cudaEventCreateWithFlags(&sl.evt[b], cudaEventDisableTiming) != cudaSuccess ||
+                        cudaEventCreateWithFlags(&sl.evc[b], cudaEventDisableTiming) != cudaSuccess) {
+                        cudaGetLastError(); return fail(DFS_ECUDA);
+                    }
+                }
+            }
+            // the copy stream starts after the handle's stream like the slot stream (below)
         }
     }
     // fork: every slot stream waits for the handle's stream; slot 0 gets its own stream too
@@ -826,6 +851,7 @@ static int run_concurrent(dfs_graph* g, const int32_t* roots, int32_t k, int32_t
     for (int c = 0; c < conc; ++c) {
         Slot& sl = g->slots[c];
         cudaStreamWaitEvent(sl.stream, s0.ev0, 0);
+        if (!out_dev) cudaStreamWaitEvent(sl.cstream, s0.ev0, 0);
         cudaMemsetAsync(sl.status, 0, sizeof(int), sl.stream);
         cudaMemsetAsync(sl.count2, 0, 2 * sizeof(unsigned long long), sl.stream);
     }
@@ -845,7 +871,10 @@ static int run_concurrent(dfs_graph* g, const int32_t* roots, int32_t k, int32_t
                 if (qe == cudaErrorNotReady) continue;
                 if (qe != cudaSuccess) { cudaGetLastError(); return fail(DFS_ECUDA); }
             }
-            int32_t* d_out = out_dev ? out + (size_t)q * g->n : sl.parent;
+            const int buf = (int)(sl.issued & 1);
+            int32_t* d_out = out_dev ? out + (size_t)q * g->n : (buf ? sl.parent2 : sl.parent);
+            // host rows: the buffer's previous row must have left for the host first
+            if (!out_dev && sl.issued >= 2) cudaStreamWaitEvent(sl.stream, sl.evc[buf], 0);
             // the first `extra` slots take one more block: all SMs in use (148 = 4 x 19 + 4 x 18)
             int rc = launch_one(g, sl, sl.stream, roots[q], d_out, o, blocks + (c < extra ? 1 : 0), warps, false, false);
             if (rc != DFS_OK) return fail(rc);
@@ -854,11 +883,15 @@ static int run_concurrent(dfs_graph* g, const int32_t* roots, int32_t k, int32_t
                 g->launches++;
             }
             if (!out_dev) {
-                if (cudaMemcpyAsync(out + (size_t)q * g->n, sl.parent, (size_t)g->n * sizeof(int32_t),
-                                    cudaMemcpyDeviceToHost, sl.stream) != cudaSuccess) {
+                // the row's copy runs on the slot's copy stream, overlapping its next traversal
+                cudaEventRecord(sl.evt[buf], sl.stream);
+                cudaStreamWaitEvent(sl.cstream, sl.evt[buf], 0);
+                if (cudaMemcpyAsync(out + (size_t)q * g->n, d_out, (size_t)g->n * sizeof(int32_t),
+                                    cudaMemcpyDeviceToHost, sl.cstream) != cudaSuccess) {
                     cudaGetLastError();
                     return fail(DFS_ECUDA);
                 }
+                cudaEventRecord(sl.evc[buf], sl.cstream);
             }
             cudaEventRecord(sl.evq[sl.issued & 1], sl.stream);
             ++sl.issued;
@@ -868,11 +901,15 @@ static int run_concurrent(dfs_graph* g, const int32_t* roots, int32_t k, int32_t
         }
         if (!any) std::this_thread::yield();
     }
-    // join
+    // join (host rows: the copy streams too)
     for (int c = 0; c < conc; ++c) {
         Slot& sl = g->slots[c];
         cudaEventRecord(sl.ev1, sl.stream);
         cudaStreamWaitEvent(base, sl.ev1, 0);
+        if (!out_dev && sl.issued > 0) {
+            cudaEventRecord(sl.ev1, sl.cstream);
+            cudaStreamWaitEvent(base, sl.ev1, 0);
+        }
     }
     cudaEventRecord(s0.evk1, base);
     if (cudaStreamSynchronize(base) != cudaSuccess) { cudaGetLastError(); return fail(DFS_ECUDA); }

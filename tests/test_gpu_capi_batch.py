@@ -89,6 +89,22 @@ def test_batch_default_concurrency_every_row(graph):
             _valid(g, int(r), out16[q].cpu().numpy())
 
 
+def test_batch_host_rows_double_buffered():
+    """Host (pinned) output rows of a concurrent batch: every slot runs many more traversals than
+    its two device row buffers, so each buffer is reused while the previous row's copy to the host
+    is in flight (copy stream + events); every row must still be the right traversal."""
+    g = graphgen.road(256, 256, seed=0x5EED)
+    roots = graphgen.random_roots(g, 40, seed=45)
+    with Graph(g.row_ptr, g.col_idx) as G:
+        for conc in (4, 8):
+            hb = torch.full((len(roots), g.n), 31337, dtype=torch.int32).pin_memory()
+            G.run_batch(roots, out=hb, options=Options(concurrency=conc))
+            for q, r in enumerate(roots):
+                row = hb[q].numpy()
+                assert row[int(r)] == -1, (conc, q)                        # the row of root q
+                _valid(g, int(r), row)
+
+
 @pytest.mark.parametrize("opts", [dict(), dict(hot_cutoff=2, cold_cutoff=2, steal_half=False),
                                   dict(window=128), dict(warps_per_block=8, blocks=40)])
 def test_both_steal_tiers_move_work(opts):
