@@ -162,8 +162,7 @@ typedef struct dfs_options {
     int32_t walker_lanes;    /* lanes per walker: 32 = the warp kernel (one walker per warp, windows of
                                 `window` positions); 16, 8, 4 or 2 = the sub-warp walker kernel (32/L
                                 independent walkers per warp, each with its own HotRing/ColdSeg and
-                                an L-position window); 1 = thread walkers (32 per
-                                warp, a 4-position window scanned in registers); 0 = auto: 4-lane walkers on
+                                an L-position window); 0 = auto: 4-lane walkers on
                                 low-degree graphs (m <= 4n, max degree <= 16) for batches with
                                 several traversals in flight and for path-like graphs (m < 2.2n),
                                 else the warp kernel.  deterministic, cluster >= 1 and window = 128

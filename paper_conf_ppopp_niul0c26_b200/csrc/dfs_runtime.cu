@@ -62,46 +62,35 @@ const void* const* kernel_table() {
 constexpr int kNumKernels = 24;
 
 // sub-warp walker kernels (dfs_walker.cuh): [G = 16, 8, 4, 2][stats], then the vertex-record
-// variants [G = 16, 8][stats], then the thread walkers [G = 1][stats]; HotRing H = 16 * G entries
-// per walker, so a 32-warp CTA holds 128 KB of rings for every G
+// variants [G = 16, 8][stats]; HotRing H = 16 * G entries per walker, so a 32-warp CTA holds
+// 128 KB of rings for every G
 #define DFS_WK(G, S, R) (const void*)dfs_walker_kernel<G, 16 * G, S, R>
-// thread walkers: 32-entry HotRings (a 16-entry ring flushes every 8 pushes), so at most
-// kG1MaxWarps warps fit in shared memory
-#ifndef DFS_G1_RING
-#define DFS_G1_RING 32
-#endif
-constexpr int kG1Ring = DFS_G1_RING;
-constexpr int kG1MaxWarps = DFS_G1_RING >= 32 ? 24 : 28;
-#define DFS_WK1(S) (const void*)dfs_walker_kernel<1, kG1Ring, S, false>
 const void* const* walker_table() {
-    static const void* const t[14] = {DFS_WK(16, false, false), DFS_WK(16, true, false), DFS_WK(8, false, false),
+    static const void* const t[12] = {DFS_WK(16, false, false), DFS_WK(16, true, false), DFS_WK(8, false, false),
                                       DFS_WK(8, true, false), DFS_WK(4, false, false), DFS_WK(4, true, false),
                                       DFS_WK(2, false, false), DFS_WK(2, true, false),
                                       DFS_WK(16, false, true), DFS_WK(16, true, true), DFS_WK(8, false, true),
-                                      DFS_WK(8, true, true), DFS_WK1(false), DFS_WK1(true)};
+                                      DFS_WK(8, true, true)};
     return t;
 }
 #undef DFS_WK
-#undef DFS_WK1
-constexpr int kNumWalkerKernels = 14;
+constexpr int kNumWalkerKernels = 12;
 int walker_lanes_of(int kf) {
-    static const int lanes[14] = {16, 16, 8, 8, 4, 4, 2, 2, 16, 16, 8, 8, 1, 1};
+    static const int lanes[12] = {16, 16, 8, 8, 4, 4, 2, 2, 16, 16, 8, 8};
     return lanes[kf];
 }
 int walker_index(int lanes, bool rec) {
     if (rec && lanes >= 8) return lanes == 16 ? 8 : 10;
-    return lanes == 16 ? 0 : lanes == 8 ? 2 : lanes == 4 ? 4 : lanes == 2 ? 6 : 12;
+    return lanes == 16 ? 0 : lanes == 8 ? 2 : lanes == 4 ? 4 : 6;
 }
-bool valid_walker_lanes(int lanes) { return lanes == 16 || lanes == 8 || lanes == 4 || lanes == 2 || lanes == 1; }
+bool valid_walker_lanes(int lanes) { return lanes == 16 || lanes == 8 || lanes == 4 || lanes == 2; }
 constexpr int kWalkerMaxWarps = DFS_WALKER_LB / 32;
 
 size_t smem_bytes(int warps) {
     return ((sizeof(SmemCtl) + 15) & ~size_t(15)) + (size_t)warps * kRing * sizeof(unsigned long long);
 }
-int walker_ring(int lanes) { return lanes == 1 ? kG1Ring : 16 * lanes; }
-int walker_max_warps(int lanes) { return lanes == 1 ? std::min(kWalkerMaxWarps, kG1MaxWarps) : kWalkerMaxWarps; }
 size_t walker_smem_bytes(int warps, int lanes) {
-    return ((sizeof(SmemW) + 15) & ~size_t(15)) + (size_t)warps * (32 / lanes) * walker_ring(lanes) * sizeof(unsigned long long);
+    return ((sizeof(SmemW) + 15) & ~size_t(15)) + (size_t)warps * (32 / lanes) * (16 * lanes) * sizeof(unsigned long long);
 }
 
 // per-traversal scratch set
@@ -307,7 +296,7 @@ dfs_graph* dfs_graph_create(const int64_t* row_ptr, const int32_t* col_idx, int6
     for (int kf = 0; kf < kNumWalkerKernels; ++kf) {
         const int lanes = walker_lanes_of(kf);
         if (cudaFuncSetAttribute(walker_table()[kf], cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                 (int)walker_smem_bytes(std::min(32, walker_max_warps(lanes)), lanes)) != cudaSuccess)
+                                 (int)walker_smem_bytes(32, lanes)) != cudaSuccess)
             attr_ok = false;
     }
     if (!attr_ok) { cudaGetLastError(); delete g; fail(DFS_ECUDA); return nullptr; }
@@ -619,7 +608,7 @@ static int resolve_options(dfs_graph* g, const dfs_options* in, int num_roots, d
     // the walker kernel is compiled for CTAs of up to kWalkerMaxWarps warps (DFS_WALKER_LB threads:
     // 28 warps x 72 registers measured faster than 32 x 64 — fewer register rematerialisations;
     // DESIGN.md §5); auto and larger requests get that
-    if (o.walker_lanes != 32 && warps > walker_max_warps(o.walker_lanes)) warps = walker_max_warps(o.walker_lanes);
+    if (o.walker_lanes != 32 && warps > kWalkerMaxWarps) warps = kWalkerMaxWarps;
     if (o.walker_lanes == 32 && warps > DFS_WMAX_BIG) warps = DFS_WMAX_BIG;
     conc = o.concurrency == 0 ? 8 : o.concurrency;       // auto: 8 in flight (B200 sweep)
     if (o.deterministic) conc = 1;

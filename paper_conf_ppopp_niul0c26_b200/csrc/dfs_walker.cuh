@@ -24,7 +24,7 @@
 
 namespace b200dfs {
 
-constexpr int kMaxWalkersPerCta = 1024;          // G = 1: 32 walkers per warp
+constexpr int kMaxWalkersPerCta = 512;
 // CTA size the walker kernel is compiled for (threads): 28 warps x 72 registers (round-2 sweep,
 // DESIGN.md §5); the runtime launches it with at most DFS_WALKER_LB / 32 warps
 #ifndef DFS_WALKER_LB
@@ -73,11 +73,10 @@ __device__ __forceinline__ unsigned long long ld_shared_u64_if(bool p, const uns
 // ------------------------------------------------------------------------------------------
 template <int G, int H, bool STATS, bool REC>
 __global__ void __launch_bounds__(DFS_WALKER_LB, 1) dfs_walker_kernel(const KParams P) {
-    static_assert(G == 1 || G == 2 || G == 4 || G == 8 || G == 16, "G is 1, 2, 4, 8 or 16");
+    static_assert(G == 2 || G == 4 || G == 8 || G == 16, "G is 2, 4, 8 or 16");
     static_assert(!REC || G >= 8, "a vertex record spans 8 lanes");
-    static_assert((H & (H - 1)) == 0 && H >= 16 && H <= 1024, "H is a power of two in [16, 1024]");
+    static_assert((H & (H - 1)) == 0 && H >= 32 && H <= 1024, "H is a power of two in [32, 1024]");
     constexpr int WPW = 32 / G;                       // walkers per warp
-    constexpr uint32_t WALL = WPW == 32 ? kFull : (1u << WPW) - 1u;   // all walkers of a warp
     constexpr uint32_t GM = (1u << G) - 1u;
 #ifndef DFS_WALKER_PF
 #define DFS_WALKER_PF 0
@@ -134,7 +133,6 @@ __global__ void __launch_bounds__(DFS_WALKER_LB, 1) dfs_walker_kernel(const KPar
     bool has_top = false, have_win = false, need_end = false, active = false;
     uint32_t u = 0, i = 0, end = 0;
     int nb = -1;                                      // this lane's neighbour: position i + sl
-    int nb4[4] = {-1, -1, -1, -1};                    // G = 1: the walker's window, positions i .. i+3
     uint32_t my_head = 0, pub = 0, tail_cache = 0;    // HotRing (owner view)
     uint32_t my_top = 0, hi = 0, cold_lo = 0;         // ColdSeg top, mapped chunks, "empty at" hint
     bool spec_ok = false;
@@ -581,7 +579,7 @@ __global__ void __launch_bounds__(DFS_WALKER_LB, 1) dfs_walker_kernel(const KPar
                     } else if (op == 7) {                     // REFILL k (Fig 2(f)) -> entries moved
                         put((int32_t)refill_walker(k));
                     } else if (op == 8 || op == 9) {          // STEAL_INTRA / STEAL_INTER thief-mask (Fig 3)
-                        const uint32_t tb = (uint32_t)r[1] & WALL;
+                        const uint32_t tb = (uint32_t)r[1] & ((1u << WPW) - 1u);
                         put((int32_t)(op == 8 ? steal_intra(tb) : steal_inter(tb)));
                     } else if (op == 10) {                    // DUMP k -> head tail top bottom
                         const uint32_t x = S.ht[kb];
@@ -621,167 +619,6 @@ __global__ void __launch_bounds__(DFS_WALKER_LB, 1) dfs_walker_kernel(const KPar
                     if (fail) goto exit_loop;
                 }
             }
-          if constexpr (G == 1) {
-            // ===== thread walkers (G = 1): every lane is a walker; its window is the 4 positions
-            // i .. i+3 of its list, scanned in order in registers (no shuffles: the 32 walkers of
-            // a warp share every instruction).  Same steps as below: speculative first claim,
-            // probes of the {visited, leaf} pairs, bulk leaf claims, in-order claim of the first
-            // unvisited candidate, leaf skip, push <u, next> (or donate it), pop.
-            constexpr int V = 4;
-            auto pick = [](const int (&a)[V], int k) -> int {   // a[k] by selects (no local memory)
-                return k == 0 ? a[0] : (k == 1 ? a[1] : (k == 2 ? a[2] : a[3]));
-            };
-            {   // window of a popped top (end not yet known) or one that must be reloaded
-                const bool lw = act && !have_win;
-                const uint32_t e2 = ld_nc_if(lw && need_end, P.rp + u + 1, end);
-                const uint32_t lim = need_end ? P.m : end;
-#pragma unroll
-                for (int k = 0; k < V; ++k) {
-                    const int x = (int)ld_nc_if(lw && i + (uint32_t)k < lim, P.col + i + k, kFull);
-                    if (lw) nb4[k] = x;
-                }
-                if (lw) { end = e2; need_end = false; have_win = true; }
-            }
-            count(kCntWindows, act);
-            uint32_t vm = 0;                                  // positions of the window in [i, end)
-#pragma unroll
-            for (int k = 0; k < V; ++k) if (act && i + (uint32_t)k < end) vm |= 1u << k;
-            // speculative claim: the first position whose neighbour is not the parent we came from
-            // is, if unvisited, exactly Alg 1's next tree edge
-            uint32_t sm = 0;
-            if (spec_ok) {
-#pragma unroll
-                for (int k = 0; k < V; ++k) if (((vm >> k) & 1u) && (uint32_t)nb4[k] != par) sm |= 1u << k;
-            }
-            const bool dospec = sm != 0;
-            const int sk = dospec ? __ffs(sm) - 1 : -1;
-            const uint32_t sv = dospec ? (uint32_t)pick(nb4, sk) : u;
-            uint32_t s_old = atom_or_if(dospec, P.bitmap + 2u * (sv >> 5), 1u << (sv & 31));
-            const uint32_t s_rs = ld_nc_if(dospec, P.rp + sv, 0u), s_re = ld_nc_if(dospec, P.rp + sv + 1, 0u);
-            uint2 wl[V];                                      // probes: {visited, leaf} pairs
-#pragma unroll
-            for (int k = 0; k < V; ++k)
-                wl[k] = ld_cg_u2_if((vm >> k) & 1u, P.bitmap + 2u * ((uint32_t)nb4[k] >> 5), kFull, 0u);
-            int cnb[V];                                       // the child's first window
-#pragma unroll
-            for (int k = 0; k < V; ++k)
-                cnb[k] = (int)ld_nc_if(spec_early && dospec && s_rs + (uint32_t)k < s_re, P.col + s_rs + k, kFull);
-            uint32_t cm = 0, lcm = 0;                         // unvisited candidates / leaves
-#pragma unroll
-            for (int k = 0; k < V; ++k) {
-                const uint32_t x = (uint32_t)nb4[k];
-                if (((vm >> k) & 1u) && k != sk && !((wl[k].x >> (x & 31)) & 1u)) {
-                    if ((wl[k].y >> (x & 31)) & 1u) lcm |= 1u << k; else cm |= 1u << k;
-                }
-            }
-            // bulk leaf claims (reading S24): fire-and-forget red.or, parent = u in every order
-            if (__any_sync(kFull, lcm != 0)) {
-#pragma unroll
-                for (int k = 0; k < V; ++k) {
-                    const bool lf = (lcm >> k) & 1u;
-                    red_or_if(lf, P.bitmap + 2u * ((uint32_t)nb4[k] >> 5), 1u << (nb4[k] & 31));
-                    st_global_if(lf, P.parent + nb4[k], (int32_t)u);            // Alg 1 l.10
-                    count(kCntClaims, lf);
-                }
-                if (P.block_claims) my_claims += __popc(lcm);
-            }
-            bool won = dospec && !(s_old & (1u << (sv & 31)));
-            count(kCntFailedClaims, dospec && !won);
-            uint32_t v = sv, vrs = s_rs, vre = s_re;
-            int kpos = sk;
-            if (!spec_early) {
-#pragma unroll
-                for (int k = 0; k < V; ++k) cnb[k] = (int)ld_nc_if(won && vrs + (uint32_t)k < vre, P.col + vrs + k, kFull);
-            }
-            // claim the first unvisited candidate in CSR order; on a lost race the next one (the
-            // walkers that still search advance together)
-            bool need = act && !won;
-            while (__any_sync(kFull, need && cm != 0)) {
-                const bool tr = need && cm != 0;
-                const int k = tr ? __ffs(cm) - 1 : 0;
-                const uint32_t cv = (uint32_t)pick(nb4, k);
-                const uint32_t bit = 1u << (cv & 31);
-                const uint32_t crs = ld_nc_if(tr, P.rp + cv, 0u), cre = ld_nc_if(tr, P.rp + cv + 1, 0u);
-                const uint32_t old = atom_or_if(tr, P.bitmap + 2u * (cv >> 5), bit);
-                int cw[V];                                    // overlaps the claim
-#pragma unroll
-                for (int q = 0; q < V; ++q) cw[q] = (int)ld_nc_if(tr && crs + (uint32_t)q < cre, P.col + crs + q, kFull);
-                const bool ok = tr && !(old & bit);
-                if (ok) {
-                    won = true; v = cv; vrs = crs; vre = cre; kpos = k; need = false;
-#pragma unroll
-                    for (int q = 0; q < V; ++q) cnb[q] = cw[q];
-                }
-                if (tr) cm &= ~(1u << k);                     // tried: won, or lost the race
-                count(kCntFailedClaims, tr && !ok);
-            }
-            // ---- descend (Alg 1 l.8-11) or continue u's scan
-            const uint32_t later = kpos >= 0 ? cm & ~((2u << kpos) - 1u) : cm;
-            const uint32_t ni = later ? i + (uint32_t)(__ffs(later) - 1) : i + (uint32_t)V;
-            st_global_if(won, P.parent + v, (int32_t)u);                        // Alg 1 l.10
-            count(kCntClaims, won);
-            if (P.block_claims && won) ++my_claims;
-            // leaf skip: v's list is empty or exactly [u]
-            const bool leafskip = won && P.leaf_skip && vre - vrs <= 1u && (vre == vrs || (uint32_t)cnb[0] == u);
-            const uint32_t next_i = leafskip ? ni : i + (uint32_t)V;
-            const bool advance = act && (!won || leafskip);
-            const bool descend = won && !leafskip;
-            bool exhausted = false;
-            if (advance) {
-                const uint32_t d = next_i - i;
-                i = next_i;
-                if (i >= end) {
-                    exhausted = true; have_win = false;       // Alg 1 l.14: pop
-                } else if (d < (uint32_t)V) {                 // leaf skip: shift the window down
-                    int t[V];
-#pragma unroll
-                    for (int k = 0; k < V; ++k) {
-                        const int src = k + (int)d;
-                        const int y = (int)ld_nc_if(src >= V && i + (uint32_t)k < end, P.col + i + k, kFull);
-                        t[k] = src < V ? pick(nb4, src) : y;
-                    }
-#pragma unroll
-                    for (int k = 0; k < V; ++k) nb4[k] = t[k];
-                    spec_ok = spec_on; par = kFull;
-                } else {
-                    have_win = false; spec_ok = false;        // next window: loaded next step
-                }
-            }
-            // push <u, ni> unless u is exhausted, or donate it to an idle sibling walker (see below)
-            bool do_push = descend && ni < end;
-            if (P.donate) {
-                const uint32_t pm = __ballot_sync(kFull, do_push);
-                const uint32_t im = __ballot_sync(kFull, !act);
-                if (pm && im) {
-                    const uint32_t below = (1u << lane) - 1u;
-                    const int rp_ = __popc(pm & below), ri_ = __popc(im & below);
-                    const bool give = do_push && rp_ < __popc(im);
-                    const bool recv = !act && ri_ < __popc(pm);
-                    const int srcl = recv ? (int)__fns(pm, 0, ri_ + 1) : lane;
-                    const uint32_t du = __shfl_sync(kFull, u, srcl);
-                    const uint32_t dni = __shfl_sync(kFull, ni, srcl);
-                    const uint32_t dend = __shfl_sync(kFull, end, srcl);
-                    atom_add_relaxed_cta_if(recv && !active, &S.lbusy, 1u);
-                    count(kCntDonations, recv);
-                    if (recv) {
-                        has_top = true; active = true;
-                        u = du; i = dni; end = dend;
-                        have_win = false; need_end = false; spec_ok = spec_pop; par = kFull;
-                    }
-                    if (give) do_push = false;
-                }
-            }
-            st_shared_u64_if(do_push, ring + (my_head & (H - 1)), pack_entry(u, ni));
-            atom_add_release_cta_if(do_push, &S.ht[bk], 0x10000u);
-            if (do_push) { ++my_head; pub = my_head; }
-            if (descend) {
-                par = u; u = v; i = vrs; end = vre; spec_ok = spec_on;
-#pragma unroll
-                for (int k = 0; k < V; ++k) nb4[k] = cnb[k];
-                have_win = true; need_end = false;
-            }
-            if (__any_sync(kFull, exhausted)) pop_if(exhausted);           // Alg 1 l.14
-          } else {
             // ---- window of walkers whose top came from a pop (end not yet known)
             {
                 const bool lw = act && !have_win;
@@ -933,7 +770,6 @@ __global__ void __launch_bounds__(DFS_WALKER_LB, 1) dfs_walker_kernel(const KPar
                 nb = cnb; have_win = true; need_end = false;
             }
             if (__any_sync(kFull, exhausted)) pop_if(exhausted);           // Alg 1 l.14
-          }
             // ---- periodic work: demand-driven spill, done flag and watchdog
             if ((++iter & P.period_mask) == 0) {
                 if (P.spill) {
@@ -995,7 +831,7 @@ __global__ void __launch_bounds__(DFS_WALKER_LB, 1) dfs_walker_kernel(const KPar
         uint32_t idle_w = 0;                                  // idle walkers, bit k = walker k
 #pragma unroll
         for (int k = 0; k < WPW; ++k) idle_w |= ((idle_mask >> (k * G)) & 1u) << k;
-        if (idle_w != WALL) {
+        if (idle_w != (1u << WPW) - 1u) {
             // some walkers of this warp are busy: one Alg 3 steal for all idle walkers every
             // steal_period steps (the busy walkers wait for it)
             if ((iter & P.steal_period_mask) == 0 && P.intra) {

@@ -1,4 +1,4 @@
-"""GPU parity of the sub-warp walker kernel (dfs_walker.cuh; dfs_options.walker_lanes = 16/8/4/2, and 1 = thread walkers).
+"""GPU parity of the sub-warp walker kernel (dfs_walker.cuh; dfs_options.walker_lanes = 16/8/4).
 
 Same bars as the warp kernel: I1-I6 exact on every graph and option
 set (I4 = reach set bit-exact), bit-exact with Alg 1 on tree inputs (unique spanning tree), steal
@@ -16,7 +16,7 @@ pytestmark = pytest.mark.gpu
 if torch.cuda.is_available():
     from paper_conf_ppopp_niul0c26_b200 import DfsError, Graph, Options
 
-LANES = [16, 8, 4, 2, 1]
+LANES = [16, 8, 4, 2]
 
 
 def _valid(g, root, parent, undirected=True):
