@@ -816,10 +816,13 @@ static int run_concurrent(dfs_graph* g, const int32_t* roots, int32_t k, int32_t
         if (!out_dev) {
             // host rows: two device row buffers and a copy stream per slot, so the copy of one
             // row overlaps the slot's next traversal (double buffering)
-            if ((!sl.parent && cudaMalloc(&sl.parent, (size_t)g->n * sizeof(int32_t)) != cudaSuccess) ||
-                (!sl.parent2 && cudaMalloc(&sl.parent2, (size_t)g->n * sizeof(int32_t)) != cudaSuccess)) {
+            if (!sl.parent && cudaMalloc(&sl.parent, (size_t)g->n * sizeof(int32_t)) != cudaSuccess) {
                 cudaGetLastError();
                 return fail(DFS_ENOMEM);
+            }
+            if (!sl.parent2 && cudaMalloc(&sl.parent2, (size_t)g->n * sizeof(int32_t)) != cudaSuccess) {
+                cudaGetLastError();                       // one buffer: copies do not overlap
+                sl.parent2 = nullptr;
             }
             if (!sl.cstream) {
                 if (cudaStreamCreateWithFlags(&sl.cstream, cudaStreamNonBlocking) != cudaSuccess) {
@@ -871,10 +874,11 @@ static int run_concurrent(dfs_graph* g, const int32_t* roots, int32_t k, int32_t
                 if (qe == cudaErrorNotReady) continue;
                 if (qe != cudaSuccess) { cudaGetLastError(); return fail(DFS_ECUDA); }
             }
-            const int buf = (int)(sl.issued & 1);
+            const int nbuf = sl.parent2 ? 2 : 1;
+            const int buf = (int)(sl.issued % nbuf);
             int32_t* d_out = out_dev ? out + (size_t)q * g->n : (buf ? sl.parent2 : sl.parent);
             // host rows: the buffer's previous row must have left for the host first
-            if (!out_dev && sl.issued >= 2) cudaStreamWaitEvent(sl.stream, sl.evc[buf], 0);
+            if (!out_dev && sl.issued >= nbuf) cudaStreamWaitEvent(sl.stream, sl.evc[buf], 0);
             // the first `extra` slots take one more block: all SMs in use (148 = 4 x 19 + 4 x 18)
             int rc = launch_one(g, sl, sl.stream, roots[q], d_out, o, blocks + (c < extra ? 1 : 0), warps, false, false);
             if (rc != DFS_OK) return fail(rc);
