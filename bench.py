@@ -65,6 +65,7 @@ def parse(argv=None):
     ap.add_argument("--no-validate", action="store_true")
     ap.add_argument("--no-batch", action="store_true", help="skip the batch1024 sub-record")
     ap.add_argument("--no-rmat", action="store_true", help="skip the rmat24 sub-record")
+    ap.add_argument("--no-span", action="store_true", help="skip the span (eccentricity floor) record")
     ap.add_argument("--no-gather", action="store_true", help="batch: skip the with-gather pass")
     ap.add_argument("--cpu-seconds", type=float, default=12.0)
     ap.add_argument("--nroots", type=int, default=64)
@@ -321,6 +322,51 @@ def main():
         dist.destroy_process_group()
 
 
+# ------------------------------------------------------------------------------ span
+def bfs_eccentricity(row_ptr, col_idx, r):
+    """Largest BFS distance from r (level-synchronous frontier BFS in numpy; not the oracle)."""
+    rp = np.asarray(row_ptr, dtype=np.int64)
+    col = np.asarray(col_idx)
+    dist_ = np.full(len(rp) - 1, -1, np.int32)
+    dist_[r] = 0
+    f = np.array([r], dtype=np.int64)
+    d = 0
+    while True:
+        s = rp[f]
+        c = rp[f + 1] - s
+        tot = int(c.sum())
+        if tot == 0:
+            break
+        nb = col[np.repeat(s - (np.cumsum(c) - c), c) + np.arange(tot)]
+        nb = np.unique(nb[dist_[nb] < 0])
+        if nb.size == 0:
+            break
+        d += 1
+        dist_[nb] = d
+        f = nb.astype(np.int64)
+    return d
+
+
+def span_record(g, my_roots, step_ms, clk, k=2):
+    """The latency floor of the first k timed roots ("span"): any traversal that
+    builds a tree needs ecc(root) sequential claims, each at least one L2 hit (~250 cycles) plus
+    one global atomic (~318 cycles) after its parent's claim (B300_MICROARCH L2/ATOMG latencies),
+    at the SM clock sampled during the timed region."""
+    mhz = (clk or {}).get("sm_mhz") or 1965.0
+    per_level_us = 570.0 / mhz
+    out = []
+    for r in list(dict.fromkeys(my_roots))[:k]:
+        ecc = bfs_eccentricity(g.row_ptr, g.col_idx, int(r))
+        ms = [t for rr, t in zip(my_roots, step_ms) if rr == r]
+        med = float(np.median(ms))
+        floor = ecc * per_level_us / 1e3
+        out.append({"root": int(r), "bfs_ecc": ecc, "ms_median": round(med, 4), "floor_ms": round(floor, 4),
+                    "frac_of_floor": round(floor / med, 4)})
+    return {"roots": out, "per_level_cycles": 570,
+            "what": "latency floor = BFS eccentricity x (L2 hit + atomic) per level; no tree-building traversal "
+                    "from that root can be faster; the DFS's own span is longer (scripts/span_sim.c)"}
+
+
 # ------------------------------------------------------------------------------ single root
 def single_root_leg(a, workload, g, root0, undirected, desc, world, rank, local, headline):
     """Single-root traversals on one GPU per rank (weak-scaled replicas for N > 1).  Returns the
@@ -429,6 +475,8 @@ def single_root_leg(a, workload, g, root0, undirected, desc, world, rank, local,
            "ms_per_dfs": round(ms_per_dfs, 4), "dfs_per_s": round(steps * world / t_job, 3),
            "ms_per_dfs_median": round(float(np.median(step_ms)), 4),
            "gpu_launches": int(launches), "clocks": clk, "roofline": roof, "validation": valid}
+    if headline and not a.no_span and workload in ("road24m", "grid256", "rmat24"):   # (deep configs: 10^6+ BFS levels)
+        rec["span"] = span_record(g, my_roots, step_ms, clk)
     if headline and not a.no_cpu_baseline and world == 1:
         v, ms, cnt, core = cpu_oracle_pinned(g, roots, a.cpu_seconds)
         rec["cpu_baseline"] = {"value": round(v, 6), "unit": "GTEPS", "cores": 1, "kind": "oracle",

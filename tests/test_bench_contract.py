@@ -47,6 +47,8 @@ def test_product_arm_json_line():
     assert e["d2h_bytes_per_step"] >= 4 * d["config"]["n"]          # the parent array comes back
     assert {"sm_mhz", "sm_max_mhz", "reasons"} <= d["clocks"].keys()
     assert d["validation"] and all(v["i6"] == 1 for v in d["validation"].values())
+    sp = d["span"]["roots"][0]                                       # headline root 0 of the grid
+    assert sp["root"] == 0 and sp["bfs_ecc"] == 255 + 255 and 0 < sp["frac_of_floor"] <= 1
 
 
 def test_gpus_flag_relaunches_under_torchrun():
