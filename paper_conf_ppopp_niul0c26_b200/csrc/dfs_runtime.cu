@@ -824,16 +824,14 @@ static int run_concurrent(dfs_graph* g, const int32_t* roots, int32_t k, int32_t
                 cudaGetLastError();                       // one buffer: copies do not overlap
                 sl.parent2 = nullptr;
             }
-            if (!sl.cstream) {
-                if (cudaStreamCreateWithFlags(&sl.cstream, cudaStreamNonBlocking) != cudaSuccess) {
-                    cudaGetLastError(); sl.cstream = nullptr; return fail(DFS_ECUDA);
+            for (int b = 0; b < 2; ++b) {
+                if ((!sl.evt[b] && cudaEventCreateWithFlags(&sl.evt[b], cudaEventDisableTiming) != cudaSuccess) ||
+                    (!sl.evc[b] && cudaEventCreateWithFlags(&sl.evc[b], cudaEventDisableTiming) != cudaSuccess)) {
+                    cudaGetLastError(); return fail(DFS_ECUDA);
                 }
-                for (int b = 0; b < 2; ++b) {
-                    if (cudaEventCreateWithFlags(&sl.evt[b], cudaEventDisableTiming) != cudaSuccess ||
-                        cudaEventCreateWithFlags(&sl.evc[b], cudaEventDisableTiming) != cudaSuccess) {
-                        cudaGetLastError(); return fail(DFS_ECUDA);
-                    }
-                }
+            }
+            if (!sl.cstream && cudaStreamCreateWithFlags(&sl.cstream, cudaStreamNonBlocking) != cudaSuccess) {
+                cudaGetLastError(); sl.cstream = nullptr; return fail(DFS_ECUDA);
             }
             // the copy stream starts after the handle's stream like the slot stream (below)
         }
