@@ -121,12 +121,6 @@ struct KParams {
     int script_out_len;
 };
 
-// DFS_PIPE: the 32-wide step issues the next level's speculative claim as soon as this level's
-// claim has won; 0 rebuilds the unpipelined step for A/B
-#ifndef DFS_PIPE
-#define DFS_PIPE 1
-#endif
-
 // vertex records (create time, on first use): record v = 8 words = one 32-byte
 // sector: the first 6 entries of v's adjacency list (kFull past its end), then row_ptr[v] and
 // row_ptr[v+1].  A walker of >= 8 lanes loads a claimed child's record with one coalesced request,
@@ -563,11 +557,6 @@ __global__ void __launch_bounds__(32 * WMAX, 1) dfs_persistent_kernel(const KPar
     bool spec_ok = false;        // speculative claim allowed on the current window (fresh child,
                                  // or a popped entry with speculate & 8)
     uint32_t par = kFull;        // parent of u when spec_ok (kFull: no position to skip)
-    // pipelined claim (32-wide step, DFS_PIPE): the next step's speculative claim, issued as soon
-    // as this step's claim is known to have won — its target, result and row_ptr pair
-    bool piped = false;
-    uint32_t p_vb = 0, p_sv = 0, p_old = 0, p_rs = 0, p_re = 0;
-    int p_sk = -1;
     // speculate: bits 0-1 = mode (0 off, 1 on, 2 on for 32-wide windows), bit 2 = issue the
     // child's first window before the claim returns (32-wide), bit 3 = also claim a popped
     // entry's next position speculatively (its probe at push time saw it unvisited)
@@ -951,18 +940,11 @@ __global__ void __launch_bounds__(32 * WMAX, 1) dfs_persistent_kernel(const KPar
             const int nxt1 = (int)ld_nc_if(have_nxt && i + 32u + lane < end, P.col + i + 32u + lane, kFull);
             // speculative claim (fresh child only): the first position whose neighbour is not the
             // parent we came from is, if unvisited, exactly Alg 1's next tree edge
-            uint32_t vb, sv, s_old, s_rs, s_re;
-            int sk;
-            if (DFS_PIPE && piped) {                              // claimed at the end of the last step
-                vb = p_vb; sk = p_sk; sv = p_sv; s_old = p_old; s_rs = p_rs; s_re = p_re;
-                piped = false;
-            } else {
-                vb = __ballot_sync(kFull, spec_ok && valid && (uint32_t)nb != par);
-                sk = __ffs(vb) - 1;
-                sv = vb ? (uint32_t)__shfl_sync(kFull, nb, sk & 31) : u;
-                s_old = atom_or_if(vb != 0 && lane == 0, P.bitmap + 2u * (sv >> 5), 1u << (sv & 31));
-                s_rs = ld_nc_if(vb != 0, P.rp + sv, 0u); s_re = ld_nc_if(vb != 0, P.rp + sv + 1, 0u);
-            }
+            const uint32_t vb = __ballot_sync(kFull, spec_ok && valid && (uint32_t)nb != par);
+            const int sk = __ffs(vb) - 1;
+            const uint32_t sv = vb ? (uint32_t)__shfl_sync(kFull, nb, sk & 31) : u;
+            uint32_t s_old = atom_or_if(vb != 0 && lane == 0, P.bitmap + 2u * (sv >> 5), 1u << (sv & 31));
+            const uint32_t s_rs = ld_nc_if(vb != 0, P.rp + sv, 0u), s_re = ld_nc_if(vb != 0, P.rp + sv + 1, 0u);
             // probe the visited bits; lanes holding the first 8 positions prefetch their
             // candidates' row_ptr pairs
             const uint2 wl = ld_cg_u2_if(valid, P.bitmap + 2u * ((uint32_t)nb >> 5), kFull, 0u);   // {visited, leaf}
@@ -1019,21 +1001,6 @@ __global__ void __launch_bounds__(32 * WMAX, 1) dfs_persistent_kernel(const KPar
             bool advance = !won;
             if (won) {
                 if (STATS) unproductive = false;
-                if (DFS_PIPE && spec_on) {
-                    // pipelined claim: the first position of v's list whose neighbour is not u is
-                    // exactly what the next step (top v, par u, a fresh window) claims first;
-                    // claim it now, before this step's bookkeeping, so that its round trip
-                    // overlaps the push, the parent store and the loop.  A non-empty ballot means
-                    // v has a neighbour other than u, so v is not a leaf and the step descends.
-                    const uint32_t vb2 = __ballot_sync(kFull, vrs + (uint32_t)lane < vre && (uint32_t)cnb != u);
-                    if (vb2) {
-                        p_vb = vb2; p_sk = __ffs(vb2) - 1;
-                        p_sv = (uint32_t)__shfl_sync(kFull, cnb, p_sk);
-                        p_old = atom_or_if(lane == 0, P.bitmap + 2u * (p_sv >> 5), 1u << (p_sv & 31));
-                        p_rs = ld_nc_if(true, P.rp + p_sv, 0u); p_re = ld_nc_if(true, P.rp + p_sv + 1, 0u);
-                        piped = true;
-                    }
-                }
                 // descend (Alg 1 l.8-11): push <u, next candidate> unless u is exhausted —
                 // positions whose probe saw a claimed target stay claimed, so skipping them keeps
                 // Alg 1's order — then v becomes the register top with its first window loaded
