@@ -121,13 +121,6 @@ struct KParams {
     int script_out_len;
 };
 
-// DFS_HYB = 1 (A/B build): the 128-wide kernel runs the 32-wide step on lists of <= 32
-// positions (per vertex, chosen when the child's window is loaded) — RMAT's serial tail walks
-// low-degree vertices at ~1 us per claim with 128-wide windows
-#ifndef DFS_HYB
-#define DFS_HYB 0
-#endif
-
 // vertex records (create time, on first use): record v = 8 words = one 32-byte
 // sector: the first 6 entries of v's adjacency list (kFull past its end), then row_ptr[v] and
 // row_ptr[v+1].  A walker of >= 8 lanes loads a claimed child's record with one coalesced request,
@@ -564,9 +557,6 @@ __global__ void __launch_bounds__(32 * WMAX, 1) dfs_persistent_kernel(const KPar
     bool spec_ok = false;        // speculative claim allowed on the current window (fresh child,
                                  // or a popped entry with speculate & 8)
     uint32_t par = kFull;        // parent of u when spec_ok (kFull: no position to skip)
-    // DFS_HYB (128-wide kernel): the current window holds a list of <= 32 positions in the
-    // 32-wide format (lane k = position i + k in nbv[0]) and the 32-wide step runs on it
-    bool narrow = false;
     // speculate: bits 0-1 = mode (0 off, 1 on, 2 on for 32-wide windows), bit 2 = issue the
     // child's first window before the claim returns (32-wide), bit 3 = also claim a popped
     // entry's next position speculatively (its probe at push time saw it unvisited)
@@ -1054,113 +1044,6 @@ __global__ void __launch_bounds__(32 * WMAX, 1) dfs_persistent_kernel(const KPar
                     spec_ok = spec_pop; par = kFull;
                 }
             }
-          } else if (DFS_HYB && narrow && have_win && win_lanes == 32) {
-            // ===== 32-wide step inside the 128-wide kernel (DFS_HYB): the top's list has at most
-            // 32 positions left, lane k holds position i + k.  Same logic as the VEC == 1 step
-            // (speculative first claim, probes, bulk leaf claims, in-order fallback, leaf skip);
-            // a child with a longer list gets a 128-wide window and leaves this mode.
-            constexpr int kPf32 = 8;
-            const bool sp_on = (P.speculate & 3) == 1 || (P.speculate & 3) == 2;
-            const bool sp_early = sp_on && (P.speculate & 4) != 0;
-            if (STATS && lane == 0) ++cnt[kCntWindows];
-            const int nb = nbv[0];
-            const bool valid = i + (uint32_t)lane < end;
-            const uint32_t vb = __ballot_sync(kFull, spec_ok && valid && (uint32_t)nb != par);
-            const int sk = __ffs(vb) - 1;
-            const uint32_t sv = vb ? (uint32_t)__shfl_sync(kFull, nb, sk & 31) : u;
-            uint32_t s_old = atom_or_if(vb != 0 && lane == 0, P.bitmap + 2u * (sv >> 5), 1u << (sv & 31));
-            const uint32_t s_rs = ld_nc_if(vb != 0, P.rp + sv, 0u), s_re = ld_nc_if(vb != 0, P.rp + sv + 1, 0u);
-            const uint2 wl = ld_cg_u2_if(valid, P.bitmap + 2u * ((uint32_t)nb >> 5), kFull, 0u);   // {visited, leaf}
-            const bool pf = valid && lane < kPf32;
-            const uint32_t prs = ld_nc_if(pf, P.rp + nb, 0u), pre = ld_nc_if(pf, P.rp + nb + 1, 0u);
-            // the child's first window: 32-wide if its list is short, else 128-wide
-            int cnb[VEC];
-#pragma unroll
-            for (int f = 0; f < VEC; ++f) cnb[f] = -1;
-            bool cnarrow = true;
-            auto load_child = [&](uint32_t rs, uint32_t re, bool p) {
-                cnarrow = re - rs <= 32u;
-                if (cnarrow) cnb[0] = (int)ld_nc_if(p && rs + lane < re, P.col + rs + lane, kFull);
-                else if (p) load_window(rs & ~(uint32_t)(VEC - 1), re, 32, cnb);
-            };
-            if (sp_early && vb != 0) load_child(s_rs, s_re, true);
-            const bool unv = valid && !((wl.x >> (nb & 31)) & 1u) && lane != sk;
-            const bool lf = unv && ((wl.y >> (nb & 31)) & 1u);
-            bool cand = unv && !lf;
-            if (__any_sync(kFull, lf)) {
-                red_or_if(lf, P.bitmap + 2u * ((uint32_t)nb >> 5), 1u << (nb & 31));
-                st_global_if(lf, P.parent + nb, (int32_t)u);                    // Alg 1 l.10
-                if (STATS || P.block_claims || P.timeline) {
-                    const uint32_t nl = __popc(__ballot_sync(kFull, lf));
-                    my_claims += nl;
-                    if (STATS && lane == 0) cnt[kCntClaims] += nl;
-                }
-            }
-            s_old = __shfl_sync(kFull, s_old, 0);
-            bool won = vb != 0 && !(s_old & (1u << (sv & 31)));
-            uint32_t v = sv, vrs = s_rs, vre = s_re;
-            int kpos = sk;
-            if (won) {
-                if (!sp_early) load_child(vrs, vre, true);
-            } else {
-                if (STATS && vb && lane == 0) ++cnt[kCntFailedClaims];
-                uint32_t any = __ballot_sync(kFull, cand);
-                while (any) {
-                    const int k = __ffs(any) - 1;
-                    const uint32_t cv = (uint32_t)__shfl_sync(kFull, nb, k);
-                    uint32_t crs = __shfl_sync(kFull, prs, k & (kPf32 - 1)), cre = __shfl_sync(kFull, pre, k & (kPf32 - 1));
-                    if (k >= kPf32) { crs = __ldg(P.rp + cv); cre = __ldg(P.rp + cv + 1); }
-                    const uint32_t bit = 1u << (cv & 31);
-                    uint32_t old = atom_or_if(lane == 0, P.bitmap + 2u * (cv >> 5), bit);
-                    load_child(crs, cre, true);                     // overlaps the claim
-                    old = __shfl_sync(kFull, old, 0);
-                    if (!(old & bit)) { won = true; v = cv; vrs = crs; vre = cre; kpos = k; break; }
-                    if (STATS && lane == 0) ++cnt[kCntFailedClaims];
-                    if (lane == k) cand = false;
-                    any = __ballot_sync(kFull, cand);
-                }
-            }
-            uint32_t next_i = i + 32u;
-            bool advance = !won;
-            if (won) {
-                if (STATS && lane == 0) ++cnt[kCntClaims];
-                ++my_claims;
-                const uint32_t later = __ballot_sync(kFull, cand && lane > kpos);
-                const uint32_t ni = later ? i + (uint32_t)(__ffs(later) - 1) : i + 32u;
-                st_global_if(lane == 0, P.parent + v, (int32_t)u);             // Alg 1 l.10
-                int first = cnb[0];
-                if (!cnarrow) {
-                    const uint32_t sel = vrs & 3u;
-                    first = sel == 0u ? cnb[0] : (sel == 1u ? cnb[1] : (sel == 2u ? cnb[2] : cnb[3]));
-                }
-                if (vre - vrs <= leaf_deg && (vre == vrs || (uint32_t)__shfl_sync(kFull, first, 0) == u)) {
-                    next_i = ni; advance = true;                  // leaf skip: stay on u
-                } else {
-                    if (ni < end) {
-                        if (!push_lean(u, ni)) goto exit_loop;
-                    }
-                    par = u;
-                    u = v; i = vrs; end = vre; spec_ok = spec_on || cnarrow;
-                    narrow = cnarrow; win_lanes = 32;              // have_win stays true
-#pragma unroll
-                    for (int f = 0; f < VEC; ++f) nbv[f] = cnb[f];
-                }
-            }
-            if (advance) {
-                const uint32_t d = next_i - i;
-                i = next_i;
-                if (i < end && d < 32u) {                         // leaf skip: shift the window
-                    int x = __shfl_down_sync(kFull, nb, d);
-                    const int y = (int)ld_nc_if(lane >= 32 - (int)d && i + lane < end, P.col + i + lane, kFull);
-                    nbv[0] = lane >= 32 - (int)d ? y : x;
-                    spec_ok = true; par = kFull;
-                } else {
-                    have_win = false; narrow = false;             // i >= end: Alg 1 l.14: pop
-                    has_top = pop(u, i);
-                    need_end = true;
-                    spec_ok = spec_pop; par = kFull;
-                }
-            }
           } else {
             // ===== lean expansion step (Alg 1 l.5-12 over one window) =====
             // Window = positions [a, a + kWin), a = i rounded down to a multiple of VEC; lane k
@@ -1284,18 +1167,7 @@ __global__ void __launch_bounds__(32 * WMAX, 1) dfs_persistent_kernel(const KPar
             uint32_t v = sv, vrs = s_rs, vre = s_re;
             int kl = sk, ke = se;                                 // window slot of v
             int cnb[VEC];
-            bool cnarrow = false;                                 // DFS_HYB: cnb is 32-wide
-            auto load_child = [&](uint32_t rs, uint32_t re) {
-                cnarrow = DFS_HYB && re - rs <= 32u;
-                if (cnarrow) {
-                    cnb[0] = (int)ld_nc_if(rs + lane < re, P.col + rs + lane, kFull);
-#pragma unroll
-                    for (int f = 1; f < VEC; ++f) cnb[f] = -1;
-                } else {
-                    load_window(rs & ~(uint32_t)(VEC - 1), re, 32, cnb);
-                }
-            };
-            if (won) load_child(vrs, vre);
+            if (won) load_window(vrs & ~(uint32_t)(VEC - 1), vre, 32, cnb);
             for (;;) {
                 if (won) {
                     // leaf skip: v's list is empty or exactly [u] — Alg 1 would descend, find
@@ -1305,7 +1177,7 @@ __global__ void __launch_bounds__(32 * WMAX, 1) dfs_persistent_kernel(const KPar
                     if (P.leaf_skip && vre == vrs + 1u) {
                         int first = cnb[0];
                         if constexpr (VEC == 4) {                // selects, not a local-memory index
-                            const uint32_t sel = cnarrow ? 0u : vrs & 3u;
+                            const uint32_t sel = vrs & 3u;
                             first = sel == 0u ? cnb[0] : (sel == 1u ? cnb[1] : (sel == 2u ? cnb[2] : cnb[3]));
                         }
                         leaf = (uint32_t)__shfl_sync(kFull, first, 0) == u;
@@ -1337,7 +1209,7 @@ __global__ void __launch_bounds__(32 * WMAX, 1) dfs_persistent_kernel(const KPar
                 if (k >= kPfLanes) { crs = __ldg(P.rp + cv); cre = __ldg(P.rp + cv + 1); }
                 const uint32_t bit = 1u << (cv & 31);
                 uint32_t old = atom_or_if(lane == 0, P.bitmap + 2u * (cv >> 5), bit);
-                load_child(crs, cre);                             // overlaps the claim
+                load_window(crs & ~(uint32_t)(VEC - 1), cre, 32, cnb);   // overlaps the claim
                 old = __shfl_sync(kFull, old, 0);
                 if (!(old & bit)) { won = true; v = cv; vrs = crs; vre = cre; kl = k; ke = e; continue; }
                 if (STATS && lane == 0) ++cnt[kCntFailedClaims];
@@ -1366,8 +1238,8 @@ __global__ void __launch_bounds__(32 * WMAX, 1) dfs_persistent_kernel(const KPar
                 }
                 st_global_if(lane == 0, P.parent + v, (int32_t)u);             // Alg 1 l.10
                 par = u;
-                u = v; i = vrs; end = vre; spec_ok = spec_on || cnarrow;
-                have_win = true; need_end = false; win_lanes = 32; narrow = cnarrow;
+                u = v; i = vrs; end = vre; spec_ok = spec_on;
+                have_win = true; need_end = false; win_lanes = 32;
 #pragma unroll
                 for (int f = 0; f < VEC; ++f) nbv[f] = cnb[f];
             } else {
