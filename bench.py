@@ -543,15 +543,40 @@ def batch_leg(a, g, world, rank, local, dev):
         torch.cuda.synchronize()
         e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         e0.record()
-        for c0 in range(0, cap, rows):
-            chunk = mine[c0:c0 + rows]
-            if chunk:
-                _, st = G.run_batch(chunk, out=out_rows[:len(chunk)], options=o, stats=True)
-                counts.append(st.root_counts.copy())
-                lanes.append(st.walker_lanes)
-            if gather and world > 1:
-                src_rows = out_rows if a.coll_dev.type == "cuda" else out_rows.cpu()
-                batch.gather_chunk_to_rank0(src_rows, len(chunk), min(rows, cap - c0), sub, sink, world, rank)
+        if gather and world > 1 and rows >= 2 * sub:
+            # exchange overlapped with the traversals: chunks of `grows` rows alternate between
+            # two halves of the row buffer; chunk c's rows go to rank 0 (async NCCL gathers on
+            # the communicator's stream) while chunk c + 1 traverses into the other half, and a
+            # half is reused only after its gathers completed
+            grows = max(sub, (rows // 2) // sub * sub)
+            halves = [out_rows[:grows], out_rows[grows:2 * grows]]
+            pending = [[], []]
+            for ci, c0 in enumerate(range(0, cap, grows)):
+                buf = halves[ci % 2]
+                for w, _ in pending[ci % 2]:
+                    w.wait()
+                pending[ci % 2] = []
+                chunk = mine[c0:c0 + grows]
+                if chunk:
+                    _, st = G.run_batch(chunk, out=buf[:len(chunk)], options=o, stats=True)
+                    counts.append(st.root_counts.copy())
+                    lanes.append(st.walker_lanes)
+                src_rows = buf if a.coll_dev.type == "cuda" else buf.cpu()
+                pending[ci % 2] = batch.gather_chunk_to_rank0(src_rows, len(chunk), min(grows, cap - c0), sub,
+                                                              sink, world, rank, async_op=True)
+            for pw in pending:
+                for w, _ in pw:
+                    w.wait()
+        else:
+            for c0 in range(0, cap, rows):
+                chunk = mine[c0:c0 + rows]
+                if chunk:
+                    _, st = G.run_batch(chunk, out=out_rows[:len(chunk)], options=o, stats=True)
+                    counts.append(st.root_counts.copy())
+                    lanes.append(st.walker_lanes)
+                if gather and world > 1:
+                    src_rows = out_rows if a.coll_dev.type == "cuda" else out_rows.cpu()
+                    batch.gather_chunk_to_rank0(src_rows, len(chunk), min(rows, cap - c0), sub, sink, world, rank)
         e1.record()
         torch.cuda.synchronize()
         ms = e0.elapsed_time(e1)
@@ -636,7 +661,8 @@ def batch_leg(a, g, world, rank, local, dev):
         b["with_gather"] = {"dfs_per_s": round(k / (t_gath * 1e-3), 3), "region_ms": round(t_gath, 3),
                             "bytes_to_rank0": int((k - (hi - lo)) * g.n * 4),
                             "what": f"each chunk's parent rows gathered to rank 0 (NCCL gather, {sub}-row rounds "
-                                    "into a reused rank-0 device buffer)"}
+                                    "into a reused rank-0 device buffer), overlapped with the next chunk's "
+                                    "traversals (double-buffered rows, async gathers)"}
     if world == 1 and not a.no_cpu_baseline:
         v, done, nth, el = cpu_oracle_pool(g, roots, a.cpu_seconds)
         b["cpu_baseline"] = {"value": round(v, 4), "unit": "DFS/s", "cores": nth, "kind": "oracle",

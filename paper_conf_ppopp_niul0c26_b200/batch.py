@@ -170,16 +170,21 @@ def reduce_max_sum(maxvals: Sequence[float], sumvals: Sequence[float], world: in
 
 
 def gather_chunk_to_rank0(rows, have: int, nrows: int, sub: int, sink, world: int, rank: int,
-                          group=None, dst: int = 0) -> int:
+                          group=None, dst: int = 0, async_op: bool = False):
     """The C5 exchange step for one chunk of parent rows (bench.py batch pass 2): every rank
     sends rows [0, nrows) of ``rows`` (a (>= nrows, n) int32 tensor whose first ``have`` rows are
     valid; the rest are sent as -3 padding so every rank makes the same calls) to ``dst`` in
     rounds of ``sub`` rows; ``dst`` receives each round into ``sink`` (world tensors of
     (sub, n) — a reused buffer: the result sink).  Returns the number of rounds (the same on
-    every rank).  Tensors live on the process group's device (CUDA for NCCL, CPU for gloo)."""
+    every rank).  Tensors live on the process group's device (CUDA for NCCL, CPU for gloo).
+
+    ``async_op=True`` returns the list of the rounds' work handles instead: with NCCL the
+    gathers then run on the communicator's stream while the caller launches the next chunk's
+    traversals (``rows`` must stay untouched until the handles are waited on)."""
     import torch
     import torch.distributed as dist
     rounds = 0
+    works = []
     n = rows.shape[1]
     for s0 in range(0, nrows, sub):
         take = max(0, min(sub, have - s0))
@@ -189,6 +194,9 @@ def gather_chunk_to_rank0(rows, have: int, nrows: int, sub: int, sink, world: in
             src = torch.full((sub, n), -3, dtype=rows.dtype, device=rows.device)
             if take > 0:
                 src[:take] = rows[s0:s0 + take]
-        dist.gather(src.contiguous(), gather_list=sink if rank == dst else None, dst=dst, group=group)
+        w = dist.gather(src.contiguous(), gather_list=sink if rank == dst else None, dst=dst, group=group,
+                        async_op=async_op)
+        if async_op:
+            works.append((w, src))                     # keep the padded source alive
         rounds += 1
-    return rounds
+    return works if async_op else rounds

@@ -122,6 +122,19 @@ def _worker_bench_exchange(rank, world, port, q):
                                                   sink, world, rank)
             if rank == 0:
                 received.append([t.clone() for t in sink])
+        # the async variant (bench pass 2 overlaps it with the next chunk's traversals) delivers
+        # the same rows once its work handles are waited on
+        received_async = []
+        for s0 in range(0, nrows, sub):
+            works = batch.gather_chunk_to_rank0(rows[s0:], max(0, have - s0), min(sub, nrows - s0), sub,
+                                                sink, world, rank, async_op=True)
+            assert len(works) == 1
+            for w, _ in works:
+                w.wait()
+            if rank == 0:
+                received_async.append([t.clone() for t in sink])
+        if rank == 0:
+            assert all(all(torch.equal(x, y) for x, y in zip(ra, rs)) for ra, rs in zip(received_async, received))
         q.put((rank, mx, sm, rounds, received))
     finally:
         dist.destroy_process_group()
