@@ -223,8 +223,10 @@ dfs_graph *dfs_graph_create(const int64_t *row_ptr, const int32_t *col_idx, int6
 int dfs_run(dfs_graph *g, int32_t root, int32_t *parent_out);
 
 /* num_roots independent traversals; row i of parents_out (num_roots x n, row-major, host or
- * device) receives the result for roots[i] (roots: host or device).  North-star batch entry;
- * multi-GPU batches partition roots across processes above this call. */
+ * device) receives the result for roots[i] (roots: host or device; repeated roots are allowed,
+ * each row is its own traversal).  num_roots = 0 is a no-op returning DFS_OK (roots and
+ * parents_out may then be NULL); num_roots < 0 or a NULL array otherwise: DFS_EINVAL.
+ * North-star batch entry; multi-GPU batches partition roots across processes above this call. */
 int dfs_run_batch(dfs_graph *g, const int32_t *roots, int32_t num_roots, int32_t *parents_out);
 
 /* dfs_run with explicit options (may be NULL = defaults) and optional stats (may be NULL). */

@@ -1003,10 +1003,10 @@ int dfs_run(dfs_graph* g, int32_t root, int32_t* parent_out) {
 
 int dfs_run_batch_ex(dfs_graph* g, const int32_t* roots, int32_t num_roots, int32_t* parents_out,
                      const dfs_options* opt, dfs_stats* stats) {
-    if (!g || !roots || !parents_out || num_roots < 0) return fail(DFS_EINVAL);
+    if (!g || num_roots < 0 || (num_roots > 0 && (!roots || !parents_out))) return fail(DFS_EINVAL);
     int rc = check_device(g);
     if (rc != DFS_OK) return fail(rc);
-    if (num_roots == 0) return DFS_OK;
+    if (num_roots == 0) return DFS_OK;                          // nothing to do (arrays may be NULL)
     std::vector<int32_t> hroots((size_t)num_roots);
     if (is_device_ptr(roots)) {
         if (cudaMemcpy(hroots.data(), roots, (size_t)num_roots * sizeof(int32_t), cudaMemcpyDeviceToHost) != cudaSuccess) {

@@ -89,6 +89,20 @@ def test_batch_default_concurrency_every_row(graph):
             _valid(g, int(r), out16[q].cpu().numpy())
 
 
+def test_batch_empty_and_repeated_roots():
+    """num_roots = 0 is a no-op (NULL arrays accepted); repeated roots give independent rows."""
+    g = graphgen.road(128, 96, seed=3)
+    lib = dfsmod.load_library()
+    with Graph(g.row_ptr, g.col_idx) as G:
+        assert lib.dfs_run_batch(ctypes.c_void_p(G._h), None, 0, None) == 0
+        assert lib.dfs_run_batch(ctypes.c_void_p(G._h), None, -1, None) == -1
+        assert G.run_batch([]).shape == (0, g.n)
+        roots = [7, 7, 7, 7, 7, 7, 7, 7, 7, 0]
+        out = G.run_batch(roots)
+        for q, r in enumerate(roots):
+            _valid(g, r, out[q].cpu().numpy())
+
+
 def test_batch_host_rows_double_buffered():
     """Host (pinned) output rows of a concurrent batch: every slot runs many more traversals than
     its two device row buffers, so each buffer is reused while the previous row's copy to the host
