@@ -418,3 +418,41 @@ def test_bulk_copy_flush_refill_exact():
                 _exact(g, root, G.run(root, options=o))
                 p, st = G.run(root, options=Options(bulk_copy=True, ring_cap=rc, collect_stats=True), stats=True)
                 _valid(g, root, p)
+
+
+def test_two_handles_from_two_host_threads():
+    """Distinct handles are independent (dfs.h): two host threads, each with its own handle and
+    its own stream, run single roots and batches at the same time; every result is valid, and a
+    failing call in one thread sets that thread's dfs_last_error only."""
+    import threading
+    graphs = [graphgen.road(300, 200, seed=21), graphgen.rmat(14, 8, seed=22)]
+    errors, results = [None, None], [None, None]
+
+    def work(t):
+        try:
+            g = graphs[t]
+            roots = [int(x) for x in graphgen.random_roots(g, 6, seed=30 + t)]
+            s = torch.cuda.Stream()
+            with torch.cuda.stream(s), Graph(g.row_ptr, g.col_idx) as G:
+                singles = [G.run(r).cpu().numpy() for r in roots[:3]]
+                rows = G.run_batch(roots).cpu().numpy()
+                lib = G._lib
+                bad = lib.dfs_run_ex(G._h, g.n + 5, None, None, None)
+                results[t] = (roots, singles, rows, bad, lib.dfs_last_error())
+        except Exception as e:  # noqa: BLE001 — reported by the main thread
+            errors[t] = e
+
+    ths = [threading.Thread(target=work, args=(t,)) for t in range(2)]
+    for th in ths:
+        th.start()
+    for th in ths:
+        th.join(timeout=600)
+    assert errors == [None, None], errors
+    for t in range(2):
+        g = graphs[t]
+        roots, singles, rows, bad, last = results[t]
+        assert bad == -1 and last == -1                       # DFS_EINVAL, this thread's code
+        for r, p in zip(roots[:3], singles):
+            _valid(g, r, p, undirected=True)
+        for q, r in enumerate(roots):
+            _valid(g, r, rows[q], undirected=True)
