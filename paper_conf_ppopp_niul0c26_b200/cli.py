@@ -2,11 +2,14 @@
 
     python -m paper_conf_ppopp_niul0c26_b200.cli --mtx graph.mtx --roots 64 --csv perf.csv
     python -m paper_conf_ppopp_niul0c26_b200.cli --config road24m --roots 8
+    python -m paper_conf_ppopp_niul0c26_b200.cli --config road24m --roots 256 --batch   # DFS/s
 
 Mirrors the paper's measurement methodology: a set of source vertices (here: the
 given ones, or `--roots` seeded vertices with out-degree > 0), one traversal per source, and the
 average of traversed edges / runtime (MTEPS).  Writes one CSV row per source (the artifact's
-per-graph perf CSV, is the model).  Every traversal runs in libdfs.so.
+per-graph perf CSV, is the model).  `--batch` runs all sources as one
+`dfs_run_batch` (K traversals in flight, BASELINE configs[4]) and reports DFS/s.  Every traversal
+runs in libdfs.so.
 """
 from __future__ import annotations
 
@@ -29,6 +32,8 @@ def main(argv=None) -> int:
     ap.add_argument("--csv", help="write per-source results here")
     ap.add_argument("--save-parents", metavar="NPY",
                     help="also save the (sources x n) int32 parent arrays (numpy .npy) for checking")
+    ap.add_argument("--batch", action="store_true",
+                    help="one dfs_run_batch over all sources (concurrent traversals); reports DFS/s")
     ap.add_argument("--set", action="append", default=[], metavar="KEY=VALUE",
                     help="dfs_options field, e.g. --set hot_cutoff=32 --set cold_cutoff=64")
     a = ap.parse_args(argv)
@@ -59,6 +64,28 @@ def main(argv=None) -> int:
     if a.save_parents:
         import numpy as np
         saved = np.empty((len(roots), g.n), dtype=np.int32)
+    if a.batch:
+        bout = torch.empty((len(roots), g.n), dtype=torch.int32, device="cuda")
+        G.run_batch(roots[:2], out=bout[:2], options=options)  # warm-up (scratch slots)
+        bout, st = G.run_batch(roots, out=bout, options=options, stats=True)
+        if saved is not None:
+            saved[:] = bout.cpu().numpy()
+        G.close()
+        if saved is not None:
+            np.save(a.save_parents, saved)
+        per = [dict(root=r, n_visited=int(st.root_counts[q, 0]), m_visited=int(st.root_counts[q, 1]))
+               for q, r in enumerate(roots)]
+        if a.csv:
+            with open(a.csv, "w", newline="") as f:
+                w = csv.DictWriter(f, fieldnames=list(per[0]))
+                w.writeheader()
+                w.writerows(per)
+        tot_e = sum(r["m_visited"] for r in per)
+        print(json.dumps(dict(graph=name, n=g.n, m=g.m, sources=len(per), load_s=round(load_s, 2), batch=True,
+                              kernel=("walkers x%d lanes" % st.walker_lanes) if st.walker_lanes != 32 else "warp",
+                              ms=round(st.kernel_ms, 3), dfs_per_s=round(len(per) / st.kernel_ms * 1e3, 2),
+                              aggregate_mteps=round(tot_e / st.kernel_ms / 1e3, 2))))
+        return 0
     for q, r in enumerate(roots):
         _, st = G.run(r, out=out, options=options, stats=True)
         if saved is not None:

@@ -381,6 +381,18 @@ def test_cli_on_matrix_market(tmp_path, capsys):
     parents = np.load(npy)
     for q, r in enumerate((0, 17)):
         _valid(gdm, r, parents[q], undirected=False)
+    # --batch: one dfs_run_batch over all sources (concurrent traversals), DFS/s summary, rows valid
+    assert cli.main(["--mtx", str(p), "--roots", "6", "--batch", "--csv", str(out_csv),
+                     "--save-parents", str(npy)]) == 0
+    summary = _json.loads(capsys.readouterr().out.strip().splitlines()[-1])
+    assert summary["batch"] is True and summary["sources"] == 6 and summary["dfs_per_s"] > 0
+    rows = out_csv.read_text().strip().splitlines()
+    parents = np.load(npy)
+    assert len(rows) == 7 and parents.shape == (6, g.n)
+    for q, line in enumerate(rows[1:]):
+        r = int(line.split(",")[0])
+        assert int(line.split(",")[1]) == g.n
+        _valid(gm, r, parents[q])
 
 
 @pytest.mark.parametrize("cl", [2, 4])
