@@ -437,6 +437,9 @@ def single_root_leg(a, workload, g, root0, undirected, desc, world, rank, local,
     # SURVEY §8(d)'s 4n reset term over the whole step time
     kbytes = sum(12.0 * n_r[r] + 8.0 * m_r[r] for r in my_roots)
     sbytes = kbytes + 4.0 * g.n * steps
+    # SURVEY §8(d)'s B_sec: the same accesses at 32-byte sector granularity (random accesses)
+    secbytes = sum(4.0 * g.n + 64.0 * n_r[r] + 32.0 * n_r[r] * (1.0 + 4.0 * (m_r[r] / max(1, n_r[r])) / 32.0)
+                   + 32.0 * m_r[r] for r in my_roots)
     my_trav = sum(trav_ms) / 1e3
 
     from paper_conf_ppopp_niul0c26_b200 import batch
@@ -458,7 +461,12 @@ def single_root_leg(a, workload, g, root0, undirected, desc, world, rank, local,
             "step": {"bytes_B_min_avg": round(sbytes / steps, 1),
                      "achieved": round(sbytes / my_time / 1e9, 3),
                      "frac": round(sbytes / my_time / 1e9 / peak, 6),
-                     "what": "SURVEY 8(d) B_min = 4n + 12 n_r + 8 m_r over the whole step (reset + traversal + finalize)"}}
+                     "what": "SURVEY 8(d) B_min = 4n + 12 n_r + 8 m_r over the whole step (reset + traversal + finalize)"},
+            "step_sector": {"bytes_B_sec_avg": round(secbytes / steps, 1),
+                            "achieved": round(secbytes / my_time / 1e9, 3),
+                            "frac": round(secbytes / my_time / 1e9 / peak, 6),
+                            "what": "SURVEY 8(d) B_sec = 4n + 64 n_r + 32 n_r (1 + 4 d/32) + 32 m_r (32-byte sectors "
+                                    "for random accesses) over the whole step"}}
     gteps = edges / t_job / 1e9
     ms_per_dfs = t_job * 1e3 / steps
     rec = {"metric": METRIC, "value": round(gteps, 6), "unit": "GTEPS", "n_gpus": world,
